@@ -1,0 +1,397 @@
+"""Pins of the CPU oracle against things other than itself (runs without a GPU).
+
+Each test names the passage (PAPER.md P:Lx-y) or the mathematical fact it
+pins.  These must pass before any CUDA result is compared with the oracle.
+"""
+from __future__ import annotations
+
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+import ttgen
+from tests import brute
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+# ---------------------------------------------------------------- Fig.2 ropes
+def test_fig2_linearisation_and_ropes():
+    """Left-biased linearisation + ropes of the Fig.2 worked example."""
+    rows = []
+    for line in open(os.path.join(GOLDEN, "fig2_ropes.txt")):
+        line = line.strip()
+        if not line or line.startswith("#"):
+            continue
+        lhs, rhs = line.split("|")
+        lab, *ch = [int(x) for x in lhs.split()]
+        pre, skip = [int(x) for x in rhs.split()]
+        rows.append((lab, ch, pre, skip))
+    labels = [r[0] for r in rows]
+    children = [[labels.index(c) for c in r[1]] for r in rows]
+    t = oracle.build_generic(children, root=0)
+    got_label = t.i64(oracle.F_LABEL)  # label index (0-based) in preorder
+    got_skip = t.i64(oracle.F_SKIP)
+    for lab, ch, pre, skip in rows:
+        p = pre - 1
+        assert labels[got_label[p]] == lab
+        assert got_skip[p] + 1 == skip
+    # guided push order at node 1 is "first 5, then 2": reversed children
+    assert [labels[c] for c in reversed(children[0])] == [5, 2]
+
+
+def _subtree_sizes(ch):
+    n = len(ch)
+    size = np.ones(n, np.int64)
+    for v in range(n - 1, -1, -1):
+        for c in ch[v]:
+            if c >= 0:
+                size[v] += size[c]
+    return size
+
+
+def _check_preorder_skip(t):
+    """skip[n] = n + |subtree(n)| and first child = n + 1 (preorder)."""
+    ch = t.children()
+    size = _subtree_sizes(ch)
+    skip = t.i64(oracle.F_SKIP)
+    assert np.array_equal(skip, np.arange(t.n_nodes) + size)
+    for v in range(t.n_nodes):
+        kids = [c for c in ch[v] if c >= 0]
+        if kids:
+            assert kids[0] == v + 1
+            # each next child starts where the previous subtree ends
+            for a, b in zip(kids, kids[1:]):
+                assert b == skip[a]
+
+
+# ------------------------------------------------------------------ kd-tree
+@pytest.mark.parametrize("n,dim,leaf", [(2000, 3, 1), (3000, 7, 8), (777, 2, 3)])
+def test_kd_build_invariants(n, dim, leaf):
+    p = ttgen.gaussian_mixture(n, dim, seed=11, components=4)
+    p[::50] = p[0]  # duplicates
+    t = oracle.build_kd(p, leaf)
+    _check_preorder_skip(t)
+    order = t.tree_order()
+    assert np.array_equal(np.sort(order), np.arange(n))  # every point in exactly one leaf
+    pb, pc_ = t.i64(oracle.F_PBEGIN), t.i64(oracle.F_PCOUNT)
+    sd, split = t.i64(oracle.F_SPLITDIM), t.f32(oracle.F_SPLIT)
+    lo, hi = t.f32(oracle.F_LO, dim), t.f32(oracle.F_HI, dim)
+    ch = t.children()
+    for v in range(t.n_nodes):
+        pts = p[order[pb[v]:pb[v] + pc_[v]]]
+        assert np.array_equal(lo[v], pts.min(0)) and np.array_equal(hi[v], pts.max(0))  # tight box
+        if sd[v] < 0:
+            assert 1 <= pc_[v] <= leaf
+            continue
+        ext = (hi[v] - lo[v]).astype(np.float32)
+        assert sd[v] == int(np.argmax(ext))  # largest extent, lowest dim on ties
+        L, R = ch[v, 0], ch[v, 1]
+        assert pc_[L] == pc_[v] // 2 and pc_[R] == pc_[v] - pc_[v] // 2  # median split
+        lp = p[order[pb[L]:pb[L] + pc_[L]], sd[v]]
+        rp = p[order[pb[R]:pb[R] + pc_[R]], sd[v]]
+        assert lp.max() <= split[v] <= rp.min()
+        assert split[v] in rp
+
+
+# ------------------------------------------------------------------ oct-tree
+def test_oct_build_invariants():
+    b = ttgen.plummer(3000, seed=12)
+    t = oracle.build_oct(b)
+    _check_preorder_skip(t)
+    order = t.tree_order()
+    assert np.array_equal(np.sort(order), np.arange(len(b)))
+    c, side = t.root_cube()
+    codes = brute.morton63(b, c, side)
+    pb, pcn, lvl = t.i64(oracle.F_PBEGIN), t.i64(oracle.F_PCOUNT), t.i64(oracle.F_LEVEL)
+    body = t.i64(oracle.F_BODY)
+    com = np.stack([t.f32(oracle.F_COMX), t.f32(oracle.F_COMY), t.f32(oracle.F_COMZ)], 1)
+    mass = t.f32(oracle.F_MASS)
+    ch = t.children()
+    for v in range(t.n_nodes):
+        ids = order[pb[v]:pb[v] + pcn[v]]
+        # all bodies of a node share the octant path of its depth (cube containment)
+        sh = np.uint64(63 - 3 * lvl[v])
+        if lvl[v] > 0:
+            assert len(np.unique(codes[ids] >> sh)) == 1
+        kids = [k for k in ch[v] if k >= 0]
+        if body[v] >= 0:
+            assert pcn[v] == 1 and ids[0] == body[v] and not kids
+        else:
+            assert len(kids) >= 1  # a cell may hold a single non-empty octant
+            # children in increasing octant order
+            octs = [int((codes[order[pb[k]]] >> np.uint64(63 - 3 * (lvl[v] + 1))) & np.uint64(7)) for k in kids]
+            assert octs == sorted(octs) and len(set(octs)) == len(octs)
+        # COM = mass-weighted mean of the bodies (fp64 brute), rounded to fp32
+        bb = b[ids].astype(np.float64)
+        M = bb[:, 3].sum()
+        want = (bb[:, :3] * bb[:, 3:4]).sum(0) / M
+        np.testing.assert_allclose(com[v], want, rtol=2e-6, atol=1e-6)
+        np.testing.assert_allclose(mass[v], M, rtol=2e-7)
+
+
+def test_oct_bucket_for_identical_bodies():
+    """Identical positions cannot be separated: a bucket cell at depth 32 (R9)."""
+    b = ttgen.plummer(64, seed=13)
+    b[5, :3] = b[6, :3] = b[7, :3]
+    t = oracle.build_oct(b)
+    assert t.height == 33
+    assert np.array_equal(np.sort(t.tree_order()), np.arange(64))
+
+
+# ------------------------------------------------------------------- vp-tree
+def test_vp_build_invariants():
+    p = ttgen.gaussian_mixture(1500, 5, seed=14, components=3)
+    t = oracle.build_vp(p)
+    _check_preorder_skip(t)
+    order = t.tree_order()
+    assert np.array_equal(np.sort(order), np.arange(len(p)))
+    vp, rin, rout = t.i64(oracle.F_VP), t.f32(oracle.F_RIN), t.f32(oracle.F_ROUT)
+    pb, pcn = t.i64(oracle.F_PBEGIN), t.i64(oracle.F_PCOUNT)
+    ch = t.children()
+    for v in range(t.n_nodes):
+        ids = order[pb[v]:pb[v] + pcn[v]]
+        assert ids[0] == vp[v] == ids.min()  # vantage = smallest id of the set
+        d = np.sqrt(brute.pinned_d2(p[[vp[v]]], p)[0])
+        cin, cout = ch[v, 0], ch[v, 1]
+        nrest = pcn[v] - 1
+        if cin >= 0:
+            ii = order[pb[cin]:pb[cin] + pcn[cin]]
+            assert len(ii) == nrest // 2
+            assert np.all(d[ii] <= rin[v]) and rin[v] in d[ii]
+        if cout >= 0:
+            oo = order[pb[cout]:pb[cout] + pcn[cout]]
+            assert np.all(d[oo] >= rout[v]) and rout[v] in d[oo]
+        if cin >= 0 and cout >= 0:
+            assert rin[v] <= rout[v]
+
+
+# ------------------------------------------------------------------------ PC
+def test_pc_vs_bruteforce():
+    """Fig.4 recursion == all-pairs count (R1 closed ball, self counted)."""
+    p = ttgen.uniform(2048, 3, seed=21)
+    p[100:110] = p[5]  # exact duplicates sit on the boundary of every test
+    t = oracle.build_kd(p, 1)
+    for r in (0.0, 0.05, 0.1, 0.3):
+        got = oracle.pc(t, p, r).out[0]
+        assert np.array_equal(got, brute.pc_counts(p, p, r))
+        assert got.min() >= 1
+        # the pair relation is symmetric: rn(a-b) = -rn(b-a), so the number of
+        # ordered pairs i != j is even
+        assert (int(got.sum()) - len(p)) % 2 == 0
+
+
+def test_pc_bucket_leaves_and_queries():
+    p = ttgen.gaussian_mixture(3000, 7, seed=22, components=5)
+    q = ttgen.gaussian_mixture(500, 7, seed=23, components=5)
+    t = oracle.build_kd(p, 8)
+    got = oracle.pc(t, q, 0.12).out[0]
+    assert np.array_equal(got, brute.pc_counts(q, p, 0.12))
+    assert np.array_equal(oracle.pc(t, q, np.inf).out[0], np.full(len(q), len(p)))  # r = inf -> N
+    # monotone in r
+    a = oracle.pc(t, q, 0.05).out[0]
+    assert np.all(a <= got)
+
+
+def test_pc_visit_count_matches_paper_shape():
+    """Config 1 shape: ~220 visits/point, count ~38 (sanity, not parity)."""
+    p = ttgen.uniform(10_000, 3, seed=1)
+    t = oracle.build_kd(p, 1)
+    r = oracle.pc(t, p, 0.1, stats=True)
+    assert 150 < r.visits.mean() < 300
+    assert 30 < r.out[0].mean() < 45
+    assert t.n_nodes == 19_999
+
+
+# ------------------------------------------------------------------------ BH
+def test_bh_theta0_equals_direct_sum():
+    """theta = 0 -> dsq = +inf -> every cell opened -> O(n^2) direct sum (R8)."""
+    b = ttgen.plummer(1500, seed=31)
+    t = oracle.build_oct(b)
+    assert oracle.bh_dsq_root(t, 0.0) == np.inf
+    got = oracle.bh(t, b, 0.0, 0.05, self_ids=np.arange(len(b))).out[0]
+    want = brute.direct_sum(b, 0.05)
+    err = np.linalg.norm(got - want, axis=1) / np.linalg.norm(want, axis=1)
+    assert err.max() < 1e-11
+
+
+def test_bh_two_body_closed_form():
+    """a_0 = m_1 r / (r^2 + eps^2)^{3/2} for two bodies whenever the root cell
+    opens (theta <= 0.5 here; at larger theta the root is 'far enough' and each body
+    sees the root monopole, which includes itself -- Fig.9a has no self test
+    for cells)."""
+    b = np.array([[0.1, 0.2, 0.3, 0.5], [0.4, -0.2, 0.7, 0.25]], np.float32)
+    t = oracle.build_oct(b)
+    for theta in (0.0, 0.25, 0.5):
+        a = oracle.bh(t, b, theta, 0.05, self_ids=np.arange(2)).out[0]
+        x = b.astype(np.float64)
+        r = x[1, :3] - x[0, :3]
+        e2 = float(np.float32(0.05)) ** 2
+        np.testing.assert_allclose(a[0], x[1, 3] * r / (r @ r + e2) ** 1.5, rtol=1e-14)
+        np.testing.assert_allclose(a[1], -x[0, 3] * r / (r @ r + e2) ** 1.5, rtol=1e-14)
+
+
+def test_bh_theta0_momentum_and_duplicates():
+    """Newton's third law: sum_i m_i a_i = 0 at theta = 0, incl. a depth-32 bucket."""
+    b = ttgen.plummer(600, seed=32)
+    b[10, :3] = b[11, :3] = b[12, :3]
+    t = oracle.build_oct(b)
+    a = oracle.bh(t, b, 0.0, 0.05, self_ids=np.arange(len(b))).out[0]
+    mom = (b[:, 3:4].astype(np.float64) * a).sum(0)
+    assert np.abs(mom).max() < 1e-12 * np.abs(b[:, 3:4] * a).sum()
+    want = brute.direct_sum(b, 0.05)
+    err = np.linalg.norm(a - want, axis=1) / np.linalg.norm(want, axis=1)
+    assert err.max() < 1e-11
+
+
+def test_bh_theta_half_approximation_is_small():
+    """theta = 0.5 monopole BH vs direct sum: characterises the approximation
+    (not parity): median error well below 1e-2."""
+    b = ttgen.plummer(4000, seed=33)
+    t = oracle.build_oct(b)
+    a = oracle.bh(t, b, 0.5, 0.05, self_ids=np.arange(len(b))).out[0]
+    want = brute.direct_sum(b, 0.05)
+    err = np.linalg.norm(a - want, axis=1) / np.linalg.norm(want, axis=1)
+    assert np.median(err) < 1e-2
+
+
+# ----------------------------------------------------------------------- kNN
+@pytest.mark.parametrize("k", [1, 8, 17])
+def test_knn_vs_bruteforce(k):
+    p = ttgen.gaussian_mixture(2048, 7, seed=41, components=6)
+    p[200:205] = p[3]  # ties broken by index (R4)
+    q = np.concatenate([ttgen.gaussian_mixture(400, 7, seed=42, components=6), p[:100]])
+    t = oracle.build_kd(p, 8)
+    idx, d2 = oracle.knn(t, q, k).out
+    bidx, bd2 = brute.knn(q, p, k)
+    assert np.array_equal(idx, bidx)
+    assert np.array_equal(d2, bd2)
+    assert np.all(np.diff(d2, axis=1) >= 0)  # sorted ascending
+    # pinned fp32 d2 is within D*u relative of the exact distance
+    exact = ((q[:, None, :].astype(np.float64) - p[idx].astype(np.float64)) ** 2).sum(-1)
+    assert np.all(np.abs(d2 - exact) <= 7 * 2.0 ** -23 * exact + 1e-30)
+
+
+def test_knn_k_exceeds_n_pads():
+    p = ttgen.uniform(5, 3, seed=43)
+    t = oracle.build_kd(p, 2)
+    idx, d2 = oracle.knn(t, p, 8).out
+    assert np.all(idx[:, 5:] == -1) and np.all(np.isinf(d2[:, 5:]))
+    assert np.array_equal(np.sort(idx[:, :5], 1), np.tile(np.arange(5), (5, 1)))
+
+
+def test_knn_cross_kernel_with_pc():
+    """With r2 := d2_k(q): PC count >= k; with the next float below: count < k."""
+    p = ttgen.gaussian_mixture(1500, 3, seed=44, components=4)
+    t1 = oracle.build_kd(p, 1)
+    t8 = oracle.build_kd(p, 8)
+    k = 8
+    idx, d2 = oracle.knn(t8, p[:200], k).out
+    for i in range(200):
+        rk = float(np.sqrt(np.float64(d2[i, -1])))
+        # radius whose fp32 square is >= d2_k ...
+        r = np.float32(rk)
+        while np.float32(r * r) < d2[i, -1]:
+            r = np.nextafter(r, np.float32(np.inf))
+        assert oracle.pc(t1, p[i:i + 1], float(r)).out[0][0] >= k
+        r = np.float32(rk)
+        while np.float32(r * r) >= d2[i, -1]:
+            r = np.nextafter(r, np.float32(0))
+        assert oracle.pc(t1, p[i:i + 1], float(r)).out[0][0] < k
+
+
+# ------------------------------------------------------------------------ VP
+def test_vp_vs_bruteforce_and_knn1():
+    p = ttgen.gaussian_mixture(2000, 16, seed=51, components=8)
+    p[300:303] = p[7]
+    q = np.concatenate([ttgen.gaussian_mixture(300, 16, seed=52, components=8), p[:50]])
+    t = oracle.build_vp(p)
+    idx, d2 = oracle.vp(t, q).out
+    bidx, bd2 = brute.nn(q, p)
+    assert np.array_equal(idx, bidx) and np.array_equal(d2, bd2)
+    kt = oracle.build_kd(p, 8)
+    kidx, kd2 = oracle.knn(kt, q, 1).out
+    assert np.array_equal(kidx[:, 0], idx) and np.array_equal(kd2[:, 0], d2)
+
+
+# ---------------------------------------------------------------- autoropes
+def test_visits_each_node_at_most_once_and_order_hash_stable():
+    """Each node tested at most once per traversal: visits <= n_nodes;
+    N-mode counts do not depend on the order points are processed (Table 1:
+    N rows identical sorted vs unsorted, e.g. P:L1154, L1166, L1178, L1202)."""
+    p = ttgen.uniform(3000, 3, seed=61)
+    t = oracle.build_kd(p, 1)
+    r = oracle.pc(t, p, 0.15, stats=True)
+    assert r.visits.max() <= t.n_nodes
+    perm = ttgen.permutation(len(p), 62)
+    r2 = oracle.pc(t, p[perm], 0.15, stats=True)
+    assert np.array_equal(r2.visits, r.visits[perm]) and np.array_equal(r2.hash, r.hash[perm])
+
+
+# --------------------------------------------------------------------- sort
+def test_sort_keys_kd_reproduce_tree_order():
+    p = ttgen.uniform(4096, 3, seed=71)
+    t = oracle.build_kd(p, 1)
+    perm = oracle.sort_perm(t, p)
+    assert np.array_equal(perm, t.tree_order())  # descent of a data point ends at its own leaf
+
+
+def test_sort_keys_oct_are_morton_and_tree_order():
+    b = ttgen.plummer(5000, seed=72)
+    t = oracle.build_oct(b)
+    c, side = t.root_cube()
+    keys = oracle.sort_keys(t, b)
+    assert np.array_equal(keys, brute.morton63(b, c, side))
+    perm = np.argsort(keys, kind="stable")
+    assert np.array_equal(perm, t.tree_order())  # Morton order == preorder of leaves
+
+
+def test_sort_keys_vp_are_a_stable_bijection():
+    p = ttgen.gaussian_mixture(3000, 16, seed=73, components=4)
+    t = oracle.build_vp(p)
+    keys = oracle.sort_keys(t, p)
+    perm = oracle.sort_perm(t, p)
+    assert np.array_equal(np.sort(perm), np.arange(len(p)))
+    ks = keys[perm]
+    assert np.all(ks[1:] >= ks[:-1])
+    # equal keys keep input order (stability)
+    same = ks[1:] == ks[:-1]
+    assert np.all(perm[1:][same] > perm[:-1][same])
+
+
+# ----------------------------------------------------------------- lockstep
+def test_unguided_lockstep_union_and_work_expansion():
+    """Work expansion = warp fetches / longest lane traversal >= 1;
+    sorting lowers it (Table 2)."""
+    b = ttgen.plummer(8192, seed=81)
+    t = oracle.build_oct(b)
+    r = oracle.bh(t, b, 0.5, 0.05, self_ids=np.arange(len(b)), stats=True)
+    perm = oracle.sort_perm(t, b)
+    for order in (perm, ttgen.permutation(len(b), 82)):
+        wf = oracle.unguided_warp_union(t, b[order], 0.5)
+        lv = r.visits[order].reshape(-1, 32)
+        assert np.all(wf >= lv.max(1)) and np.all(wf <= lv.sum(1))
+    ws = (oracle.unguided_warp_union(t, b[perm], 0.5) / r.visits[perm].reshape(-1, 32).max(1)).mean()
+    wu = (oracle.unguided_warp_union(t, b[ttgen.permutation(len(b), 82)], 0.5)
+          / r.visits[ttgen.permutation(len(b), 82)].reshape(-1, 32).max(1)).mean()
+    assert 1.0 <= ws < wu
+
+
+def test_guided_lockstep_results_equal_independent():
+    """Majority-vote call-set reduction does not change results."""
+    p = ttgen.gaussian_mixture(3000, 7, seed=91, components=6)
+    q = ttgen.gaussian_mixture(1000, 7, seed=92, components=6)
+    kt = oracle.build_kd(p, 8)
+    for qq in (q, q[oracle.sort_perm(kt, q)]):
+        idx, d2 = oracle.knn(kt, qq, 8).out
+        li, ld, lv, wf = oracle.knn_lockstep(kt, qq, 8)
+        assert np.array_equal(li, idx) and np.array_equal(ld, d2)
+        assert np.all(wf >= 1)
+    p16 = ttgen.gaussian_mixture(2000, 16, seed=93, components=6)
+    q16 = ttgen.gaussian_mixture(700, 16, seed=94, components=6)
+    vt = oracle.build_vp(p16)
+    idx, d2 = oracle.vp(vt, q16).out
+    li, ld, lv, wf = oracle.vp_lockstep(vt, q16)
+    assert np.array_equal(li, idx) and np.array_equal(ld, d2)
