@@ -1,0 +1,237 @@
+/*
+ * tt.h -- C ABI of the B200-native batched point-by-tree traversal library
+ * (libtt.so), after Goldfarb, Jo & Kulkarni, "General Transformations for GPU
+ * Execution of Tree Traversals", SC'13.  "P:Lx-y" cites /root/reference/PAPER.md.
+ *
+ * The method (Fig.1): many independent points each walk one shared
+ * tree; at every node a truncation test either stops the walk below that node
+ * or the point is updated and recurses into the children.  The library
+ * implements the paper's GPU form of it:
+ *   - autoropes (§3): the recursion becomes an iterative preorder
+ *     walk -- stackless via per-node ropes ("skip") for unguided traversals,
+ *     or an explicit rope stack (children pushed in reverse call order,
+ *     non-invariant arguments pushed with the node) for guided ones;
+ *   - lockstep traversal (§4.2, Fig.8): a warp walks the union of
+ *     its 32 points' traversals under an active mask (ballot), one node fetch
+ *     per warp; guided traversals reduce their call sets per warp by majority
+ *     vote (§4.3);
+ *   - point sorting (§4.4) and the choice between lockstep and
+ *     independent traversal, made here per warp.
+ *
+ * Conventions (all entry points):
+ *   - Every call returns tt_status; TT_OK == 0, errors are negative.  Calls
+ *     never abort or throw.  Argument errors are detected before any work.
+ *   - Traversal / sort calls are asynchronous on the caller's stream
+ *     (tt_stream = cudaStream_t; 0 = legacy default stream).  Device faults
+ *     surface at the caller's next synchronisation (and via tt_last_cuda_error).
+ *   - Point, order and result buffers are caller-owned DEVICE memory; the
+ *     library never frees them.  There is no CPU fallback: without a CUDA
+ *     device every traversal returns TT_ERR_CUDA.
+ *   - Results are written in the caller's original point order: result i
+ *     belongs to point i, whether or not an `order` permutation is used.
+ *   - n == 0 is valid and launches nothing.
+ *   - Inputs must be finite; NaN/Inf coordinates give unspecified results.
+ */
+#ifndef TT_H
+#define TT_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum tt_status {
+    TT_OK = 0,
+    TT_ERR_INVALID_ARG = -1,   /* null/misaligned pointer, bad size or parameter   */
+    TT_ERR_CUDA = -2,          /* CUDA runtime error (see tt_last_cuda_error)      */
+    TT_ERR_OOM = -3,           /* host or device allocation failed                 */
+    TT_ERR_TREE_TOO_DEEP = -4, /* tree height exceeds the compiled stack capacity  */
+    TT_ERR_KIND_MISMATCH = -5, /* e.g. tt_traverse_bh on a kd-tree                 */
+    TT_ERR_UNSUPPORTED = -6    /* parameter outside what the kernels implement     */
+} tt_status;
+
+typedef enum tt_kind {
+    TT_KIND_OCT = 1, /* Barnes-Hut oct-tree of bodies     */
+    TT_KIND_KD = 2,  /* kd-tree              */
+    TT_KIND_VP = 3   /* vantage-point tree [27]                    */
+} tt_kind;
+
+typedef enum tt_mode {
+    TT_MODE_AUTO = 0,        /* per-warp choice, see tt_traverse_opts.auto_min_depth */
+    TT_MODE_LOCKSTEP = 1,    /* "L" in Table 1                         */
+    TT_MODE_INDEPENDENT = 2  /* "N" in Table 1: non-lockstep autoropes                */
+} tt_mode;
+
+typedef enum tt_mem { TT_MEM_HOST = 0, TT_MEM_DEVICE = 1 } tt_mem;
+
+typedef void *tt_stream; /* cudaStream_t */
+
+#define TT_MAX_HEIGHT 48      /* rope-stack capacity bound (levels)            */
+#define TT_MAX_DIM 16         /* point dimensionality supported by the kernels */
+#define TT_MAX_K 32           /* kNN k supported by the kernels                */
+
+/* ------------------------------------------------------------------------ */
+/* Host-side tree construction (build rules: DESIGN.md R3, R8a, R9, R12).   */
+/* The paper takes the tree as given by the application; these
+ * builders produce the canonical left-biased linearisation (preorder, first
+ * child first, rope = preorder index after the subtree, Fig.2).
+ * Points are read from host memory (row-major, leading dimension `ld` floats)
+ * and copied; the host tree owns its arrays until tt_host_tree_free.        */
+typedef struct tt_host_tree tt_host_tree;
+
+tt_status tt_build_kd(const float *pts, int64_t n, int32_t dim, int32_t ld, int32_t leaf_size,
+                      tt_host_tree **out);
+/* bodies: n rows of (x, y, z, mass). */
+tt_status tt_build_oct(const float *bodies, int64_t n, tt_host_tree **out);
+tt_status tt_build_vp(const float *pts, int64_t n, int32_t dim, int32_t ld, tt_host_tree **out);
+void tt_host_tree_free(tt_host_tree *t);
+
+/* Canonical tree description, all arrays in preorder (host memory).  Node
+ * indices are preorder indices; -1 = absent.  Produced by tt_host_tree_desc,
+ * or filled by the caller with its own tree.                              */
+typedef struct tt_tree_desc {
+    int32_t kind;            /* tt_kind                                          */
+    int32_t dim;             /* point dimension (3 for OCT)                      */
+    int32_t height;          /* max node level (root = 0)                        */
+    int32_t leaf_size;       /* kd bucket size (informative)                     */
+    int64_t n_nodes;
+    int64_t n_points;
+    const int32_t *first_child; /* [n_nodes] first child (OCT/KD), -1 for a leaf  */
+    const int32_t *skip;        /* [n_nodes] rope: preorder index after subtree   */
+    const int32_t *level;       /* [n_nodes]                                      */
+    const int32_t *pbegin;      /* [n_nodes] first tree-order point of subtree    */
+    const int32_t *pcount;      /* [n_nodes] points in subtree                    */
+    /* KD */
+    const int32_t *split_dim;   /* [n_nodes] -1 for a leaf                        */
+    const float *split;         /* [n_nodes]                                      */
+    const float *lo, *hi;       /* [n_nodes * dim] tight bounding boxes           */
+    /* OCT */
+    const float *com;           /* [n_nodes * 4] centre of mass x,y,z and mass    */
+    const int32_t *body;        /* [n_nodes] body id of a leaf, -1 for a cell     */
+    double root_center[3];
+    double root_side;
+    /* VP */
+    const int32_t *in_child;    /* [n_nodes] inside child or -1                   */
+    const int32_t *out_child;   /* [n_nodes] outside child or -1                  */
+    const float *r_in_max;      /* [n_nodes] max distance vp -> inside points     */
+    const float *r_out_min;     /* [n_nodes] min distance vp -> outside points    */
+    /* points */
+    const int32_t *tree_order;  /* [n_points] original id of j-th tree-order point*/
+    const float *points;        /* [n_points * dim] by ORIGINAL id (OCT: 4 floats)*/
+} tt_tree_desc;
+
+tt_status tt_host_tree_desc(const tt_host_tree *t, tt_tree_desc *out);
+
+/* ------------------------------------------------------------------------ */
+/* a0: tree upload ("an identical linearized copy of the tree is
+ * constructed using a left-biased linearization, with the nodes structured
+ * according to [the field-split] layout ... and copied to the GPU's global
+ * memory").  Layout: one 32-byte record per node (two 128-bit
+ * field groups split by use), int32 node indices, the nodes of
+ * the top `top_levels` levels renumbered first so one bulk copy stages them
+ * in shared memory.  The packed blob is position-independent, so it can be
+ * NCCL-broadcast as bytes and adopted on another GPU.
+ * Errors: TT_ERR_INVALID_ARG (inconsistent desc), TT_ERR_TREE_TOO_DEEP
+ * (height > TT_MAX_HEIGHT), TT_ERR_UNSUPPORTED (dim > TT_MAX_DIM),
+ * TT_ERR_OOM, TT_ERR_CUDA.  The returned tree owns its device memory until
+ * tt_tree_free; it is read-only, so concurrent traversals are safe.      */
+typedef struct tt_tree tt_tree;
+
+tt_status tt_tree_pack_size(const tt_tree_desc *d, size_t *bytes);
+tt_status tt_tree_pack(const tt_tree_desc *d, void *host_blob, size_t bytes);
+/* mem = TT_MEM_HOST: blob in host memory (copied H2D on `s`);
+ * mem = TT_MEM_DEVICE: blob already in device memory (e.g. after an NCCL
+ * broadcast); it is copied device-to-device, the caller keeps ownership.
+ * The call synchronises `s` before returning.                             */
+tt_status tt_tree_from_blob(const void *blob, size_t bytes, int32_t mem, tt_stream s, tt_tree **out);
+tt_status tt_tree_upload(const tt_tree_desc *d, tt_stream s, tt_tree **out);
+tt_status tt_tree_free(tt_tree *t);
+
+typedef struct tt_tree_info {
+    int32_t kind, dim, dim_padded, height;
+    int64_t n_nodes, n_points;
+    int32_t top_levels;      /* levels staged in shared memory                   */
+    int32_t top_count;       /* nodes in those levels                           */
+    int64_t device_bytes;    /* bytes of the packed device layout               */
+    const void *device_blob; /* device pointer of the packed layout             */
+} tt_tree_info;
+tt_status tt_tree_get_info(const tt_tree *t, tt_tree_info *out);
+
+/* ------------------------------------------------------------------------ */
+/* a1: point sort (§4.4).  Key = where the point's descent of the
+ * tree by the build's split rule ends, in tree (preorder) order: kd -> the
+ * leaf's first tree-order point; oct -> 63-bit octant path (Morton order,
+ * equal to the preorder of leaves); vp -> 2-bit-per-level path code.  A
+ * stable radix sort of (key, index) gives perm: perm[j] = original index of
+ * the j-th point in tree order (ties by index).  pts: device, n rows of `ld`
+ * floats (OCT: ld >= 4 or 3).  keys_out (nullable): the keys, in input order.
+ * Temporary device memory is taken stream-ordered (cudaMallocAsync).      */
+tt_status tt_sort_points(const tt_tree *t, const float *pts, int64_t n, int32_t ld,
+                         uint32_t *perm_out, uint64_t *keys_out, tt_stream s);
+
+/* ------------------------------------------------------------------------ */
+/* a2-a6: traversal launch options (all optional; pass NULL for defaults).  */
+typedef struct tt_stats {
+    uint32_t *visits;        /* [n] per point: truncation tests it performed (the
+                                paper's per-point node count)      */
+    uint32_t *warp_fetches;  /* [ceil(n/32)] node records fetched by the warp
+                                (lockstep: one per step; independent: per lane) */
+    uint32_t *warp_steps;    /* [ceil(n/32)] loop iterations of the warp         */
+    uint8_t *warp_mode;      /* [ceil(n/32)] 1 = lockstep, 2 = independent      */
+} tt_stats;
+
+typedef struct tt_traverse_opts {
+    int32_t mode;            /* tt_mode                                          */
+    int32_t auto_min_depth;  /* AUTO: lockstep iff the warp's points share a tree
+                                path of at least this many levels; -1 = kernel
+                                default (BH, PC: 0 = always lockstep, P:L2235-2236;
+                                kNN: never; VP: tuned)            */
+    const uint32_t *order;   /* [n] device, nullable: lane j of the launch processes
+                                point order[j] (e.g. perm from tt_sort_points);
+                                results still go to the point's own slot        */
+    const tt_stats *stats;   /* host struct of device pointers, nullable         */
+    int32_t block_threads;   /* 0 = default (256)                               */
+    int32_t ctas_per_sm;     /* 0 = occupancy maximum                            */
+} tt_traverse_opts;
+
+/* Barnes-Hut force pass (Fig.9): bodies float4 (x,y,z,m) rows;
+ * self_ids[i] (nullable; default i) is the leaf body id whose interaction
+ * point i skips (R9).  A cell is opened iff it is a cell and
+ * |com - x|^2 < dsq_L, dsq_L = dsq_root * 0.25^L, dsq_root = (side/theta)^2
+ * (theta == 0 -> +inf: every cell opened).  acc_out: float4 (ax,ay,az,0),
+ * G = 1, softening eps.  Opening decisions use the pinned fp32 sequence R0. */
+tt_status tt_traverse_bh(const tt_tree *t, const float *bodies, const int32_t *self_ids, int64_t n,
+                         float theta, float eps, float *acc_out, const tt_traverse_opts *opts,
+                         tt_stream s);
+
+/* 2-point correlation (Fig.4/6/8):
+ * count_out[i] = #{data points p : d2(q_i, p) <= rn(radius^2)}.  q: n rows of
+ * `ld` floats, dim = tree dim.                                             */
+tt_status tt_traverse_pc(const tt_tree *t, const float *q, int64_t n, int32_t ld, float radius,
+                         uint32_t *count_out, const tt_traverse_opts *opts, tt_stream s);
+
+/* k-nearest neighbours (Fig.5/7): the k
+ * data points with the smallest (d2, id), ascending; idx_out/d2_out are n*k
+ * row-major; padded with (-1, +inf) when the tree holds fewer than k points.
+ * 1 <= k <= TT_MAX_K.                                                     */
+tt_status tt_traverse_knn(const tt_tree *t, const float *q, int64_t n, int32_t ld, int32_t k,
+                          int32_t *idx_out, float *d2_out, const tt_traverse_opts *opts,
+                          tt_stream s);
+
+/* Vantage-point-tree nearest neighbour ([27]): argmin (d2, id). */
+tt_status tt_traverse_vp(const tt_tree *t, const float *q, int64_t n, int32_t ld, int32_t *idx_out,
+                         float *d2_out, const tt_traverse_opts *opts, tt_stream s);
+
+/* ------------------------------------------------------------------------ */
+const char *tt_status_string(tt_status s);
+/* Last CUDA error code seen by the library (cudaError_t as int), 0 if none. */
+int32_t tt_last_cuda_error(void);
+/* Version / build identification string (compiled arch, flags). */
+const char *tt_build_info(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TT_H */
