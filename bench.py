@@ -1,0 +1,507 @@
+#!/usr/bin/env python
+"""bench.py -- throughput of the batched point-by-tree traversal on B200.
+
+Contract (driver):  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+N > 1 runs under torchrun (one process per GPU, NCCL).  Rank 0 prints ONE JSON line.
+
+Workload (default, N=1): BASELINE.json configs[1] -- Barnes-Hut force pass over
+a 1M-body Plummer sphere, theta = 0.5, eps = 0.05, fp32.  A step is one pass
+of the hot path: tt_sort_points (key kernel + radix sort)
+then tt_traverse_bh (per-warp mode choice, traversal, write-out in the
+caller's order); for N > 1 also the all-gather of the results.  The tree
+upload (a0) is timed separately (`upload_ms`), as §8(a) specifies.
+Scaling is weak: every rank owns M = 1M bodies of an N*M-body Plummer sphere
+whose tree is built on rank 0 and NCCL-broadcast.
+
+metric = points traversed / s (whole job, all ranks); node visits / s and the
+roofline of the dominant kernel are reported alongside.
+--impl reference times the CPU oracle (the reference arm of this tier) on
+the host cores, on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import ttgen  # noqa: E402
+
+METRIC = "points traversed/sec and node visits/sec at 1/2/4/8 B200; % HBM peak"
+# algorithmic bytes per useful visit of each kernel's packed layout
+BYTES_PER_VISIT = {"bh": 32, "pc": 48, "knn": 96, "vp": 80}
+BYTES_PER_POINT_IO = {"bh": 32, "pc": 20, "knn": 28 + 64, "vp": 64 + 8}
+L2_FLUSH_BYTES = 512 << 20  # > 126 MB L2
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--workload", choices=["bh", "knn", "vp", "pc"], default="bh")
+    ap.add_argument("--mode", default="auto", choices=["auto", "lockstep", "independent"])
+    ap.add_argument("--unsorted", action="store_true", help="skip tt_sort_points (paper's 'unsorted' column)")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--points-per-rank", type=int, default=0, help="override M (testing)")
+    return ap.parse_args()
+
+
+# ------------------------------------------------------------------ inputs
+def make_workload(name: str, world: int, per_rank: int = 0):
+    """Global synthetic inputs (identical on every rank: seeded)."""
+    if name == "bh":
+        c = dict(ttgen.CONFIGS["bh_1m_plummer"])
+        m = per_rank or c["n"]
+        data = ttgen.plummer(m * world, c["seed"])
+        return dict(cfg=c, workload="bh_1m_plummer", data=data, queries=data, m=m, n_data=m * world)
+    if name == "knn":
+        c = dict(ttgen.CONFIGS["knn_1m_7d"])
+        m = per_rank or c["m"]
+        data = ttgen.gaussian_mixture(c["n"], c["dim"], c["seed"])
+        q = ttgen.gaussian_mixture(m * world, c["dim"], c["qseed"])
+        return dict(cfg=c, workload="knn_1m_7d", data=data, queries=q, m=m, n_data=c["n"])
+    if name == "vp":
+        c = dict(ttgen.CONFIGS["vp_1m_16d"])
+        m = per_rank or c["m"]
+        data = ttgen.gaussian_mixture(c["n"], c["dim"], c["seed"])
+        q = ttgen.gaussian_mixture(m * world, c["dim"], c["qseed"])
+        return dict(cfg=c, workload="vp_1m_16d", data=data, queries=q, m=m, n_data=c["n"])
+    c = dict(ttgen.CONFIGS["pc_10k_3d"])
+    m = per_rank or c["n"]
+    data = ttgen.uniform(c["n"], c["dim"], c["seed"])
+    q = data if world == 1 and m == c["n"] else ttgen.uniform(m * world, c["dim"], c["seed"] + 100)
+    return dict(cfg=c, workload="pc_10k_3d", data=data, queries=q, m=m, n_data=c["n"])
+
+
+def host_tree(P, name, w):
+    c = w["cfg"]
+    if name == "bh":
+        return P.build_oct(w["data"])
+    if name == "vp":
+        return P.build_vp(w["data"])
+    return P.build_kd(w["data"], c["leaf"])
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md)."""
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu: int):
+        self.gpu = gpu
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits", "-lms", "100",
+                 "-i", str(self.gpu)], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx.append(float(f[2]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(mx), "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+# ------------------------------------------------------------ kernel count
+def count_kernels(step_fn) -> int | None:
+    """Kernels launched by one step, counted from a CUDA-graph capture of it."""
+    import torch
+    try:
+        from cuda.bindings import runtime as rt
+        g = torch.cuda.CUDAGraph()
+        s = torch.cuda.Stream()
+        torch.cuda.synchronize()
+        with torch.cuda.stream(s):
+            g.capture_begin()
+            step_fn()
+            g.capture_end()
+        torch.cuda.synchronize()
+        raw = g.raw_cuda_graph()
+        err, _, n = rt.cudaGraphGetNodes(rt.cudaGraph_t(init_value=raw), 0)
+        err, nodes, n = rt.cudaGraphGetNodes(rt.cudaGraph_t(init_value=raw), n)
+        k = 0
+        for nd in nodes:
+            e, ty = rt.cudaGraphNodeGetType(nd)
+            if ty == rt.cudaGraphNodeType.cudaGraphNodeTypeKernel:
+                k += 1
+        del g
+        return k
+    except Exception as e:  # capture not possible: reported as null
+        print(f"[bench] kernel count via graph capture failed: {e!r}", file=sys.stderr)
+        torch.cuda.synchronize()
+        return None
+
+
+def load_traffic(kernel: str):
+    """dram bytes per launch from the committed ncu --set full summary, if any."""
+    path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        return json.load(open(path)).get(kernel)
+    except (OSError, ValueError):
+        return None
+
+
+def measured_peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))), "measured"
+    except (OSError, ValueError):
+        return {"hbm_gbs": 6650.0}, "fallback"
+
+
+# ----------------------------------------------------------- oracle timing
+def oracle_baseline(name, w, budget_points=None):
+    """The oracle as it stands, on the host cores, on a bounded sample."""
+    import oracle
+    c = w["cfg"]
+    q = w["queries"]
+    m = len(q)
+    frac = {"bh": 8, "knn": 8, "vp": 512, "pc": 1}[name]
+    idx = np.arange(0, m, frac)
+    if budget_points:
+        idx = idx[:budget_points]
+    threads = oracle.max_threads()
+    if name == "bh":
+        t = oracle.build_oct(w["data"])
+        t0 = time.perf_counter()
+        oracle.bh(t, q[idx], c["theta"], c["eps"], self_ids=idx, threads=threads)
+    elif name == "knn":
+        t = oracle.build_kd(w["data"], c["leaf"])
+        t0 = time.perf_counter()
+        oracle.knn(t, q[idx], c["k"], threads=threads)
+    elif name == "vp":
+        t = oracle.build_vp(w["data"])
+        t0 = time.perf_counter()
+        oracle.vp(t, q[idx], threads=threads)
+    else:
+        t = oracle.build_kd(w["data"], c["leaf"])
+        t0 = time.perf_counter()
+        oracle.pc(t, q[idx], c["radius"], threads=threads)
+    dt = time.perf_counter() - t0
+    return {"value": len(idx) / dt, "unit": "points/s", "cores": threads, "kind": "oracle",
+            "sample": f"every {frac}th query ({len(idx)} of {m}) over the full tree; tree build excluded",
+            "seconds": dt}
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the CPU oracle on this box's host cores (rank 0 only)."""
+    if rank != 0:
+        return
+    w = make_workload(args.workload, 1, args.points_per_rank)
+    vals = []
+    for _ in range(max(1, min(args.steps, 3))):
+        vals.append(oracle_baseline(args.workload, w))
+    v = statistics.median(x["value"] for x in vals)
+    cb = dict(vals[0])
+    cb["value"] = v
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "points/s", "n_gpus": world,
+            "steps": len(vals), "warmup": 0, "ms_per_step": 1000.0 * statistics.median(x["seconds"] for x in vals),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32 decisions / f64 BH sums",
+            "data": "synthetic", "config": {"workload": w["workload"], "points": len(w["queries"])},
+            "cpu_baseline": cb, "e2e": {"value": v, "unit": "points/s", "h2d_bytes_per_step": 0,
+                                         "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------- ours
+def run_ours(args, rank, world, local_rank):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_sc_goldfarbjk13_b200 as P
+    from paper_conf_sc_goldfarbjk13_b200 import parallel as PAR
+
+    torch.cuda.set_device(local_rank)
+    device = torch.device("cuda", local_rank)
+    name = args.workload
+    w = make_workload(name, world, args.points_per_rank)
+    c = w["cfg"]
+    m = w["m"]
+    lo, hi = PAR.shard_range(len(w["queries"]), rank, world)
+    assert hi - lo == m
+
+    # a0: tree (rank 0 builds; NCCL broadcast for N > 1) -- timed separately
+    t0 = time.perf_counter()
+    if world == 1:
+        host = host_tree(P, name, w)
+        t1 = time.perf_counter()
+        tree = P.tt_tree_upload(host)
+    else:
+        host = host_tree(P, name, w) if rank == 0 else None
+        t1 = time.perf_counter()
+        tree = PAR.broadcast_tree(host, device)
+    torch.cuda.synchronize()
+    t2 = time.perf_counter()
+    build_ms, upload_ms = 1e3 * (t1 - t0), 1e3 * (t2 - t1)
+
+    q_all = torch.from_numpy(np.ascontiguousarray(w["queries"])).to(device)
+    q_shard = q_all[lo:hi]
+    n_all = len(w["queries"])
+    stream = torch.cuda.current_stream()
+    order_buf = torch.empty(m, dtype=torch.int32, device=device)
+    if name == "bh":
+        out = torch.zeros((n_all, 4), dtype=torch.float32, device=device)
+    elif name == "knn":
+        out = (torch.zeros((n_all, c["k"]), dtype=torch.int32, device=device),
+               torch.zeros((n_all, c["k"]), dtype=torch.float32, device=device))
+    elif name == "vp":
+        out = (torch.zeros(n_all, dtype=torch.int32, device=device),
+               torch.zeros(n_all, dtype=torch.float32, device=device))
+    else:
+        out = torch.zeros(n_all, dtype=torch.int32, device=device)
+
+    # shard views: the rank's points and result rows [lo, hi); BH self ids are
+    # the bodies' global indices (the tree is built over all N*M bodies)
+    def views(o):
+        return tuple(x[lo:hi] for x in o) if isinstance(o, tuple) else o[lo:hi]
+
+    out_shard = views(out)
+    self_ids = torch.arange(lo, hi, dtype=torch.int32, device=device) if name == "bh" else None
+
+    def traverse(pts, res, order, stats=None):
+        if name == "bh":
+            P.tt_traverse_bh(tree, pts, c["theta"], c["eps"], out=res, self_ids=self_ids, order=order,
+                             mode=args.mode, stats=stats)
+        elif name == "knn":
+            P.tt_traverse_knn(tree, pts, c["k"], out_idx=res[0], out_d2=res[1], order=order, mode=args.mode,
+                              stats=stats)
+        elif name == "vp":
+            P.tt_traverse_vp(tree, pts, out_idx=res[0], out_d2=res[1], order=order, mode=args.mode, stats=stats)
+        else:
+            P.tt_traverse_pc(tree, pts, c["radius"], out=res, order=order, mode=args.mode, stats=stats)
+
+    if args.unsorted:
+        order_buf.copy_(torch.arange(m, dtype=torch.int32, device=device))
+
+    def step(kev=None):
+        if not args.unsorted:
+            P.tt_sort_points(tree, q_shard, out=order_buf)  # a1
+        if kev:
+            kev[0].record(stream)
+        traverse(q_shard, out_shard, order_buf)            # a2-a5
+        if kev:
+            kev[1].record(stream)
+        if world > 1:
+            for o in (out if isinstance(out, tuple) else (out,)):
+                PAR.allgather_rows(o, world)
+
+    # stats pass (untimed): per-point useful visits, warp fetches, modes
+    if not args.unsorted:
+        P.tt_sort_points(tree, q_shard, out=order_buf)
+    st = P.Stats.alloc(m, device)
+    traverse(q_shard, out_shard, order_buf, st)
+    torch.cuda.synchronize()
+    visits = int(st.visits.to(torch.int64).sum().item())
+    wf = int(st.warp_fetches.to(torch.int64).sum().item())
+    lock_frac = float((st.warp_mode == 1).float().mean().item())
+    del st
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    launches = count_kernels(step) if rank == 0 else None
+
+    flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.float32, device=device)
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    kevs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local_rank) as clk:
+        for i in range(args.steps):
+            flush.zero_()  # L2 flush between timed iterations (outside the events)
+            evs[i][0].record(stream)
+            step(kevs[i])
+            evs[i][1].record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    step_ms = [a.elapsed_time(b) for a, b in evs]
+    kern_ms = [a.elapsed_time(b) for a, b in kevs]
+    ms = statistics.mean(step_ms)
+    kms = statistics.mean(kern_ms)
+    if world > 1:
+        ms = PAR.max_over_ranks(ms, device)
+        kms = PAR.max_over_ranks(kms, device)
+        visits_all = torch.tensor([visits], dtype=torch.int64, device=device)
+        dist.all_reduce(visits_all)
+        visits_tot = int(visits_all.item())
+    else:
+        visits_tot = visits
+
+    # e2e through the public API with host buffers (pinned), copies inside
+    e2e = None
+    if not args.no_e2e:
+        q_host = torch.from_numpy(np.ascontiguousarray(w["queries"][lo:hi])).pin_memory()
+        q_dev = torch.empty_like(q_host, device=device)
+        res_host = None
+        if name == "bh":
+            res_dev = torch.empty((m, 4), dtype=torch.float32, device=device)
+            res_host = torch.empty((m, 4), dtype=torch.float32).pin_memory()
+        elif name in ("knn",):
+            res_dev = (torch.empty((m, c["k"]), dtype=torch.int32, device=device),
+                       torch.empty((m, c["k"]), dtype=torch.float32, device=device))
+            res_host = tuple(torch.empty(r.shape, dtype=r.dtype).pin_memory() for r in res_dev)
+        elif name == "vp":
+            res_dev = (torch.empty(m, dtype=torch.int32, device=device),
+                       torch.empty(m, dtype=torch.float32, device=device))
+            res_host = tuple(torch.empty(r.shape, dtype=r.dtype).pin_memory() for r in res_dev)
+        else:
+            res_dev = torch.empty(m, dtype=torch.int32, device=device)
+            res_host = torch.empty(m, dtype=torch.int32).pin_memory()
+        perm = torch.empty(m, dtype=torch.int32, device=device)
+
+        def e2e_step():
+            q_dev.copy_(q_host, non_blocking=True)
+            P.tt_sort_points(tree, q_dev, out=perm)
+            if name == "bh":
+                P.tt_traverse_bh(tree, q_dev, c["theta"], c["eps"], out=res_dev, order=perm, mode=args.mode,
+                                 self_ids=self_ids)
+                res_host.copy_(res_dev, non_blocking=True)
+            elif name == "knn":
+                P.tt_traverse_knn(tree, q_dev, c["k"], out_idx=res_dev[0], out_d2=res_dev[1], order=perm,
+                                  mode=args.mode)
+                for h_, d_ in zip(res_host, res_dev):
+                    h_.copy_(d_, non_blocking=True)
+            elif name == "vp":
+                P.tt_traverse_vp(tree, q_dev, out_idx=res_dev[0], out_d2=res_dev[1], order=perm, mode=args.mode)
+                for h_, d_ in zip(res_host, res_dev):
+                    h_.copy_(d_, non_blocking=True)
+            else:
+                P.tt_traverse_pc(tree, q_dev, c["radius"], out=res_dev, order=perm, mode=args.mode)
+                res_host.copy_(res_dev, non_blocking=True)
+
+        for _ in range(2):
+            e2e_step()
+        torch.cuda.synchronize()
+        ee = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+        for i in range(args.steps):
+            flush.zero_()
+            ee[i][0].record(stream)
+            e2e_step()
+            ee[i][1].record(stream)
+        torch.cuda.synchronize()
+        ems = statistics.mean(a.elapsed_time(b) for a, b in ee)
+        if world > 1:
+            ems = PAR.max_over_ranks(ems, device)
+        d2h = sum(r.numel() * r.element_size() for r in (res_host if isinstance(res_host, tuple) else (res_host,)))
+        e2e = {"value": m * world / (ems / 1e3), "unit": "points/s", "ms_per_step": ems,
+               "h2d_bytes_per_step": int(q_host.numel() * q_host.element_size()), "d2h_bytes_per_step": int(d2h),
+               "note": "public API (tt_sort_points + tt_traverse_*) on pinned host buffers; H2D, D2H inside"}
+
+    if rank != 0:
+        return
+    peaks, peak_src = measured_peaks()
+    hbm = float(peaks.get("hbm_gbs", 6650.0))
+    bpv = BYTES_PER_VISIT[name]
+    alg_bytes = visits * bpv + m * BYTES_PER_POINT_IO[name]  # per launch on rank 0
+    achieved = alg_bytes / (kms / 1e3) / 1e9
+    kernel_name = {"bh": "bh_kernel", "pc": "pc_kernel", "knn": "knn_kernel", "vp": "vp_kernel"}[name]
+    roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": hbm, "unit": "GB/s",
+                "frac": round(achieved / hbm, 4), "traffic": load_traffic(kernel_name),
+                "peak_source": peak_src, "kernel": kernel_name, "kernel_ms": round(kms, 4),
+                "kernel_share_of_step": round(kms / ms, 4) if world == 1 else None,
+                "alg_bytes_per_launch": int(alg_bytes),
+                "alg_bytes_def": f"useful visits x {bpv} B record + {BYTES_PER_POINT_IO[name]} B/point I/O",
+                "warp_fetch_bytes_per_launch": int(wf * bpv)}
+    cpu = None
+    if world == 1 and not args.no_cpu_baseline:
+        try:
+            cpu = oracle_baseline(name, w)
+        except Exception as e:  # noqa: BLE001
+            cpu = {"value": None, "error": repr(e)}
+    value = m * world / (ms / 1e3)
+    line = {
+        "metric": METRIC, "value": value, "unit": "points/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": {"workload": w["workload"], "points_per_rank": m, "global_points": n_all,
+                   "tree_points": w["n_data"], "mode": args.mode, "sorted": not args.unsorted,
+                   "parallelism": f"dp{world} (points sharded, tree replicated)",
+                   "l2": "flushed between timed steps (512 MiB write)",
+                   "params": {k: v for k, v in c.items() if k not in ("kind",)}},
+        "node_visits_per_sec": visits_tot / (kms / 1e3),
+        "visits_per_point": visits / m,
+        "lockstep_warp_fraction": lock_frac,
+        "work_expansion_fetch_over_visits": (wf * 32.0 / visits) if visits else None,
+        "traverse_ms": kms, "upload_ms": upload_ms, "host_build_ms": build_ms,
+        "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": (launches or 0) * args.steps,
+        "gpu_launches_per_step": launches,
+        "clocks": clk.summary(),
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        if world == 1 and args.gpus > 1:
+            print(json.dumps({"error": "launch N>1 under torchrun"}), flush=True)
+            sys.exit(2)
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    try:
+        run_ours(args, rank, world, local_rank)
+    finally:
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

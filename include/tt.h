@@ -109,7 +109,8 @@ typedef struct tt_tree_desc {
     const float *lo, *hi;       /* [n_nodes * dim] tight bounding boxes           */
     /* OCT */
     const float *com;           /* [n_nodes * 4] centre of mass x,y,z and mass    */
-    const int32_t *body;        /* [n_nodes] body id of a leaf, -1 for a cell     */
+    const int32_t *body;        /* [n_nodes] OCT: body id of a leaf, -1 for a cell;
+                                   VP: id of the node's vantage point            */
     double root_center[3];
     double root_side;
     /* VP */

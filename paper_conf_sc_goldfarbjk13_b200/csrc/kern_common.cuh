@@ -1,0 +1,194 @@
+// kern_common.cuh -- device helpers shared by the traversal kernels (sm_100a).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "tt_internal.h"
+
+#define TT_FULL 0xffffffffu
+#define TT_WARPS_PER_CTA_MAX 32
+
+namespace tt {
+
+// ------------------------------------------------------------------ TMA bulk
+// One elected thread stages the top levels of the tree into shared memory with
+// cp.async.bulk (SASS UBLKCP) completing on an mbarrier; every thread waits on
+// the barrier's phase 0.  Sizes are multiples of 16 B, addresses 16-B aligned
+// (blob sections are 256-B aligned).
+__device__ __forceinline__ void mbar_init(uint64_t *bar, unsigned count) {
+    unsigned a = (unsigned)__cvta_generic_to_shared(bar);
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(a), "r"(count) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *bar, unsigned bytes) {
+    unsigned a = (unsigned)__cvta_generic_to_shared(bar);
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(a), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void *dst_smem, const void *src_gmem, unsigned bytes, uint64_t *bar) {
+    unsigned d = (unsigned)__cvta_generic_to_shared(dst_smem);
+    unsigned b = (unsigned)__cvta_generic_to_shared(bar);
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(d),
+        "l"(src_gmem), "r"(bytes), "r"(b)
+        : "memory");
+}
+__device__ __forceinline__ void mbar_wait_phase0(uint64_t *bar) {
+    unsigned a = (unsigned)__cvta_generic_to_shared(bar);
+    asm volatile(
+        "{\n\t.reg .pred P1;\n"
+        "WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], 0;\n\t"
+        "@!P1 bra WAIT_%=;\n}" ::"r"(a)
+        : "memory");
+}
+
+struct StageChunk {
+    void *dst;
+    const void *src;
+    unsigned bytes;
+};
+
+// Thread 0 arms the barrier with the total byte count and issues one bulk copy
+// per chunk; all threads wait.  Must be called by every thread of the CTA.
+template <int NCH>
+__device__ __forceinline__ void stage_top(uint64_t *bar, const StageChunk (&ch)[NCH]) {
+    unsigned total = 0;
+#pragma unroll
+    for (int i = 0; i < NCH; ++i) total += ch[i].bytes;
+    if (threadIdx.x == 0) {
+        mbar_init(bar, 1);
+        mbar_arrive_expect_tx(bar, total);
+#pragma unroll
+        for (int i = 0; i < NCH; ++i)
+            if (ch[i].bytes) bulk_g2s(ch[i].dst, ch[i].src, ch[i].bytes, bar);
+    }
+    __syncthreads();  // barrier initialised before anyone waits on it
+    mbar_wait_phase0(bar);
+}
+
+// ------------------------------------------------------------ tile scheduler
+// Persistent CTAs pull 32-point warp tiles from a global counter (dynamic load
+// balance: clustered inputs give uneven traversal lengths).
+__device__ __forceinline__ long long next_tile(uint32_t *ctr) {
+    unsigned t = 0;
+    if ((threadIdx.x & 31) == 0) t = atomicAdd(ctr, 1u);
+    return (long long)__shfl_sync(TT_FULL, t, 0);
+}
+
+// Last CTA out resets the counters for the next launch on this slot.
+__device__ __forceinline__ void cta_finish(uint32_t *ctr) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        unsigned done = atomicAdd(ctr + 1, 1u);
+        if (done == gridDim.x - 1) {
+            atomicExch(ctr, 0u);
+            atomicExch(ctr + 1, 0u);
+        }
+    }
+}
+
+// ------------------------------------------------------ pinned fp32 arithmetic
+// DESIGN.md R0: t_d = rn(q_d - p_d), s = rn(t_0 t_0), s = rn(s + rn(t_d t_d)),
+// never contracted to FMA (explicit _rn intrinsics).
+template <int DIM>
+__device__ __forceinline__ float pinned_d2(const float (&q)[DIM], const float *p) {
+    float t = __fsub_rn(q[0], p[0]);
+    float s = __fmul_rn(t, t);
+#pragma unroll
+    for (int d = 1; d < DIM; ++d) {
+        float u = __fsub_rn(q[d], p[d]);
+        s = __fadd_rn(s, __fmul_rn(u, u));
+    }
+    return s;
+}
+
+// Box distance rn(max(lo - q, q - hi, 0))^2 summed in the same order.
+template <int DIM>
+__device__ __forceinline__ float pinned_boxd2(const float (&q)[DIM], const float *lo, const float *hi) {
+    float s = 0.0f;
+#pragma unroll
+    for (int d = 0; d < DIM; ++d) {
+        float a = __fsub_rn(lo[d], q[d]);
+        float b = __fsub_rn(q[d], hi[d]);
+        float t = fmaxf(fmaxf(a, b), 0.0f);
+        float tt = __fmul_rn(t, t);
+        s = (d == 0) ? tt : __fadd_rn(s, tt);
+    }
+    return s;
+}
+
+// Load DIM floats from a 16-B aligned row (padded to a multiple of 4) with
+// 128-bit loads.  `GLOBAL_NC` selects ld.global.nc (read-only path).
+template <int DIM>
+__device__ __forceinline__ void load_row_nc(float (&r)[DIM], const float *p) {
+    constexpr int V = (DIM + 3) / 4;
+    const float4 *p4 = reinterpret_cast<const float4 *>(p);
+#pragma unroll
+    for (int v = 0; v < V; ++v) {
+        float4 x = __ldg(p4 + v);
+        if (4 * v + 0 < DIM) r[4 * v + 0] = x.x;
+        if (4 * v + 1 < DIM) r[4 * v + 1] = x.y;
+        if (4 * v + 2 < DIM) r[4 * v + 2] = x.z;
+        if (4 * v + 3 < DIM) r[4 * v + 3] = x.w;
+    }
+}
+template <int DIM>
+__device__ __forceinline__ void load_row_smem(float (&r)[DIM], const float *p) {
+    constexpr int V = (DIM + 3) / 4;
+    const float4 *p4 = reinterpret_cast<const float4 *>(p);
+#pragma unroll
+    for (int v = 0; v < V; ++v) {
+        float4 x = p4[v];
+        if (4 * v + 0 < DIM) r[4 * v + 0] = x.x;
+        if (4 * v + 1 < DIM) r[4 * v + 1] = x.y;
+        if (4 * v + 2 < DIM) r[4 * v + 2] = x.z;
+        if (4 * v + 3 < DIM) r[4 * v + 3] = x.w;
+    }
+}
+// Query rows have an arbitrary leading dimension: scalar loads.
+template <int DIM>
+__device__ __forceinline__ void load_query(float (&r)[DIM], const float *q, long long row, int ld) {
+    const float *p = q + row * (long long)ld;
+#pragma unroll
+    for (int d = 0; d < DIM; ++d) r[d] = __ldg(p + d);
+}
+
+// q[dim] for a runtime dim without dynamic register indexing.
+template <int DIM>
+__device__ __forceinline__ float select_dim(const float (&q)[DIM], int dim) {
+    float v = q[0];
+#pragma unroll
+    for (int d = 1; d < DIM; ++d) v = (dim == d) ? q[d] : v;
+    return v;
+}
+
+// ------------------------------------------------------- warp-level helpers
+// Number of leading tree levels on which all valid lanes agree, given a path
+// code with `bits` bits per level packed in the low `bits*levels` bits.
+__device__ __forceinline__ int warp_common_levels(unsigned long long code, unsigned vmask, int bits, int levels) {
+    const int leader = __ffs(vmask) - 1;
+    unsigned long long lead = __shfl_sync(TT_FULL, code, leader);
+    unsigned long long diff = ((vmask >> (threadIdx.x & 31)) & 1u) ? (code ^ lead) : 0ull;
+    unsigned hi = __reduce_or_sync(TT_FULL, (unsigned)(diff >> 32));
+    unsigned lo = __reduce_or_sync(TT_FULL, (unsigned)diff);
+    unsigned long long x = ((unsigned long long)hi << 32) | lo;
+    if (x == 0) return levels;
+    int lead_zero = __clzll((long long)x) - (64 - bits * levels);
+    return lead_zero / bits;
+}
+
+__device__ __forceinline__ unsigned warp_sum(unsigned v) { return __reduce_add_sync(TT_FULL, v); }
+
+// Stats writer for the warp tile (lane 0).
+__device__ __forceinline__ void write_warp_stats(const tt_common_params &c, long long tile, unsigned fetches,
+                                                 unsigned steps, bool lock) {
+    if ((threadIdx.x & 31) == 0) {
+        if (c.st_warp_fetches) c.st_warp_fetches[tile] = fetches;
+        if (c.st_warp_steps) c.st_warp_steps[tile] = steps;
+        if (c.st_warp_mode) c.st_warp_mode[tile] = lock ? 1 : 2;
+    }
+}
+
+}  // namespace tt

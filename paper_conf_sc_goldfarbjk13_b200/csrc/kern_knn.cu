@@ -1,0 +1,299 @@
+// kern_knn.cu -- k-nearest neighbours over a kd-tree (Fig.5 P:L440-458,
+// autoroped Fig.7), sm_100a.
+//
+// Guided traversal with two call sets (near child first).  Autoropes with an
+// explicit rope stack in shared memory:
+//   independent (N): one stack per lane, lane-interleaved [depth][32] int32
+//     (the shared-memory analogue of the paper's interleaved per-thread
+//     stacks; bank = lane, conflict-free);
+//   lockstep (L): one stack per warp of {node, mask} (Fig.8);
+//     the call set is reduced per warp by a majority vote of the active lanes
+//     (§4.3; tie -> left first, reading R6).
+// Pushing the far child and continuing into the near one is the reverse-order
+// push of §3.2.2 with its immediate pop folded away.
+// can_correlate (reading R5a): prune iff the k-heap is full and the tight box
+// distance exceeds the current k-th best -- conservative under the pinned
+// arithmetic, so the result is exactly the brute-force definition.
+// Per-lane k-best list: KT register slots kept sorted ascending on (d2, id);
+// the first KT-k slots hold (-inf) sentinels, so the k-th best is always
+// slot KT-1 (static register index).
+#include "kern_common.cuh"
+
+namespace {
+
+using namespace tt;
+
+constexpr int kBlock = 256;
+constexpr int kWarps = kBlock / 32;
+constexpr int kSmemHdr = 128;
+
+__device__ __forceinline__ bool kless(float da, unsigned ia, float db, unsigned ib) {
+    return da < db || (da == db && ia < ib);
+}
+
+template <int KT>
+struct KBest {
+    float d[KT];
+    unsigned i[KT];
+    __device__ __forceinline__ void init(int k) {
+#pragma unroll
+        for (int j = 0; j < KT; ++j) {
+            const bool real = j >= KT - k;
+            d[j] = real ? __int_as_float(0x7f800000) : __int_as_float(0xff800000);
+            i[j] = 0xffffffffu;
+        }
+    }
+    __device__ __forceinline__ float worst() const { return d[KT - 1]; }
+    // caller guarantees (dd, ii) < (d[KT-1], i[KT-1])
+    __device__ __forceinline__ void insert(float dd, unsigned ii) {
+        d[KT - 1] = dd;
+        i[KT - 1] = ii;
+#pragma unroll
+        for (int j = KT - 1; j > 0; --j) {
+            const bool sw = kless(d[j], i[j], d[j - 1], i[j - 1]);
+            const float td = d[j - 1];
+            const unsigned ti = i[j - 1];
+            d[j - 1] = sw ? d[j] : td;
+            i[j - 1] = sw ? i[j] : ti;
+            d[j] = sw ? td : d[j];
+            i[j] = sw ? ti : i[j];
+        }
+    }
+};
+
+template <int DIM>
+__device__ __forceinline__ void ld_box(const float *s_box, const float *g_box, int dp, int top, int cur,
+                                       float (&lo)[DIM], float (&hi)[DIM]) {
+    if (cur < top) {
+        load_row_smem<DIM>(lo, s_box + (size_t)cur * 2 * dp);
+        load_row_smem<DIM>(hi, s_box + (size_t)cur * 2 * dp + dp);
+    } else {
+        load_row_nc<DIM>(lo, g_box + (size_t)cur * 2 * dp);
+        load_row_nc<DIM>(hi, g_box + (size_t)cur * 2 * dp + dp);
+    }
+}
+__device__ __forceinline__ void ld_rec(const unsigned char *s_rec, const tt_kd_rec *g_rec, int top, int cur,
+                                       int4 &t, int4 &u) {
+    if (cur < top) {
+        t = reinterpret_cast<const int4 *>(s_rec)[cur * 2];
+        u = reinterpret_cast<const int4 *>(s_rec)[cur * 2 + 1];
+    } else {
+        t = __ldg(reinterpret_cast<const int4 *>(g_rec + cur));
+        u = __ldg(reinterpret_cast<const int4 *>(g_rec + cur) + 1);
+    }
+}
+
+// update_closest: every bucket point that beats the k-th best enters the list.
+template <int DIM, int KT>
+__device__ __forceinline__ void leaf_update(const tt_knn_params &P, int pb, int pc, int dp, const float (&q)[DIM],
+                                            KBest<KT> &kb) {
+    for (int j = pb; j < pb + pc; ++j) {
+        float p[DIM];
+        load_row_nc<DIM>(p, P.c.tree.pts + (size_t)j * dp);
+        const float d2 = pinned_d2<DIM>(q, p);
+        if (d2 <= kb.worst()) {
+            const unsigned id = (unsigned)__ldg(P.c.tree.pid + j);
+            if (kless(d2, id, kb.worst(), kb.i[KT - 1])) kb.insert(d2, id);
+        }
+    }
+}
+
+template <int DIM, int KT, bool STATS>
+__global__ void __launch_bounds__(kBlock) knn_kernel(const tt_knn_params P, int cap) {
+    extern __shared__ __align__(128) unsigned char smem[];
+    constexpr int DP = (DIM + 3) & ~3;
+    uint64_t *bar = reinterpret_cast<uint64_t *>(smem);
+    const int top = P.c.top_count;
+    unsigned char *s_rec = smem + kSmemHdr;
+    float *s_box = reinterpret_cast<float *>(s_rec + (size_t)top * 32);
+    int *s_stack = reinterpret_cast<int *>(reinterpret_cast<unsigned char *>(s_box) + (size_t)top * 8 * DP);
+    const tt_kd_rec *g_rec = static_cast<const tt_kd_rec *>(P.c.tree.rec);
+    const float *g_box = P.c.tree.box;
+    StageChunk ch[2] = {{s_rec, g_rec, (unsigned)top * 32u}, {s_box, g_box, (unsigned)top * 8u * DP}};
+    stage_top(bar, ch);
+
+    const int lane = threadIdx.x & 31;
+    const int warp = threadIdx.x >> 5;
+    // per-warp region: N mode [cap][32] ints; L mode [cap] nodes + [cap] masks
+    int *w_stk = s_stack + (size_t)warp * cap * 32;
+    int *w_node = w_stk;
+    unsigned *w_mask = reinterpret_cast<unsigned *>(w_stk + cap);
+    const long long n = P.c.n;
+    const long long ntiles = (n + 31) >> 5;
+    const int k = P.k;
+
+    for (;;) {
+        const long long tile = next_tile(P.c.counter);
+        if (tile >= ntiles) break;
+        const long long pos = tile * 32 + lane;
+        const bool valid = pos < n;
+        const long long pid = valid ? (P.c.order ? (long long)P.c.order[pos] : pos) : 0;
+        float q[DIM];
+        if (valid) load_query<DIM>(q, P.q, pid, P.ld);
+        else
+#pragma unroll
+            for (int d = 0; d < DIM; ++d) q[d] = 0.f;
+        const unsigned vmask = __ballot_sync(TT_FULL, valid);
+
+        bool lock = P.c.mode == TT_MODE_LOCKSTEP;
+        if (P.c.mode == TT_MODE_AUTO && P.c.auto_min_depth >= 0 && P.c.auto_min_depth < 64) {
+            int cur = 0, lv = 0;
+            unsigned long long code = 0;
+            const int maxl = min(max(P.c.auto_min_depth, 1), 60);
+            while (lv < maxl && cur >= 0 && cur < top) {
+                const int4 t = reinterpret_cast<const int4 *>(s_rec)[cur * 2];
+                if (t.x < 0) break;
+                const int4 u = reinterpret_cast<const int4 *>(s_rec)[cur * 2 + 1];
+                const bool left = select_dim<DIM>(q, u.y) < __int_as_float(u.x);
+                code = (code << 1) | (left ? 0u : 1u);
+                cur = left ? t.x : t.y;
+                ++lv;
+            }
+            lock = warp_common_levels(code << (maxl - lv), vmask, 1, maxl) >= P.c.auto_min_depth;
+        }
+
+        KBest<KT> kb;
+        kb.init(k);
+        unsigned visits = 0, fetches = 0, steps = 0;
+        if (!lock) {
+            int sp = 0;
+            int cur = valid ? 0 : TT_END;
+            while (cur != TT_END) {
+                if (STATS) ++visits;
+                bool prune = false;
+                if (kb.worst() < __int_as_float(0x7f800000)) {  // list full
+                    float lo[DIM], hi[DIM];
+                    ld_box<DIM>(s_box, g_box, DP, top, cur, lo, hi);
+                    prune = pinned_boxd2<DIM>(q, lo, hi) > kb.worst();
+                }
+                if (!prune) {
+                    int4 t, u;
+                    ld_rec(s_rec, g_rec, top, cur, t, u);
+                    if (t.x < 0) {
+                        leaf_update<DIM, KT>(P, u.z, u.w, DP, q, kb);
+                    } else {
+                        const bool left_near = select_dim<DIM>(q, u.y) < __int_as_float(u.x);
+                        w_stk[sp * 32 + lane] = left_near ? t.y : t.x;  // push far
+                        ++sp;
+                        cur = left_near ? t.x : t.y;                     // visit near
+                        continue;
+                    }
+                }
+                cur = sp > 0 ? w_stk[(--sp) * 32 + lane] : TT_END;
+            }
+            if (STATS) {
+                fetches = warp_sum(visits);
+                steps = __reduce_max_sync(TT_FULL, visits);
+            }
+        } else {
+            int sp = 0;
+            int cur = 0;
+            unsigned mask = vmask;
+            for (;;) {
+                const bool in = (mask >> lane) & 1u;
+                if (STATS) {
+                    ++steps;
+                    visits += in;
+                }
+                float lo[DIM], hi[DIM];
+                ld_box<DIM>(s_box, g_box, DP, top, cur, lo, hi);
+                const bool active =
+                    in && !(kb.worst() < __int_as_float(0x7f800000) && pinned_boxd2<DIM>(q, lo, hi) > kb.worst());
+                const unsigned act = __ballot_sync(TT_FULL, active);
+                if (act) {
+                    int4 t, u;
+                    ld_rec(s_rec, g_rec, top, cur, t, u);
+                    if (t.x < 0) {
+                        if (active) leaf_update<DIM, KT>(P, u.z, u.w, DP, q, kb);
+                    } else {
+                        const bool pref_left = active && select_dim<DIM>(q, u.y) < __int_as_float(u.x);
+                        const int votes = __popc(__ballot_sync(TT_FULL, pref_left));
+                        const bool left_first = 2 * votes >= __popc(act);
+                        w_node[sp] = left_first ? t.y : t.x;  // push second (all lanes write the same value)
+                        w_mask[sp] = act;
+                        ++sp;
+                        cur = left_first ? t.x : t.y;
+                        mask = act;
+                        continue;
+                    }
+                }
+                if (sp == 0) break;
+                --sp;
+                cur = w_node[sp];
+                mask = w_mask[sp];
+            }
+            fetches = steps;
+        }
+        if (valid) {
+#pragma unroll
+            for (int j = 0; j < KT; ++j) {
+                const int slot = j - (KT - k);
+                if (slot >= 0) {
+                    const bool empty = kb.i[j] == 0xffffffffu;
+                    P.idx[pid * k + slot] = empty ? -1 : (int)kb.i[j];
+                    P.d2[pid * k + slot] = kb.d[j];
+                }
+            }
+            if (STATS && P.c.st_visits) P.c.st_visits[pid] = visits;
+        }
+        if (STATS) write_warp_stats(P.c, tile, fetches, steps, lock);
+        __syncwarp();
+    }
+    cta_finish(P.c.counter);
+}
+
+template <int DIM, int KT, bool STATS>
+int launch(const tt_knn_params &p, const tt_launch_cfg &cfg) {
+    constexpr int DP = (DIM + 3) & ~3;
+    const int cap = p.c.height + 2;
+    const size_t smem = kSmemHdr + (size_t)p.c.top_count * (32 + 8 * DP) + (size_t)kWarps * cap * 32 * 4;
+    auto kern = knn_kernel<DIM, KT, STATS>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return (int)e;
+    int dev = 0, nsm = 0, occ = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kBlock, smem);
+    if (e != cudaSuccess) return (int)e;
+    if (cfg.ctas_per_sm > 0 && cfg.ctas_per_sm < occ) occ = cfg.ctas_per_sm;
+    if (occ < 1) occ = 1;
+    const long long ntiles = (p.c.n + 31) / 32;
+    long long grid = (long long)nsm * occ;
+    const long long need = (ntiles + kWarps - 1) / kWarps;
+    if (grid > need) grid = need;
+    if (grid < 1) grid = 1;
+    kern<<<(unsigned)grid, kBlock, smem, (cudaStream_t)cfg.stream>>>(p, cap);
+    return (int)cudaGetLastError();
+}
+
+template <int DIM, int KT>
+int launch_k(const tt_knn_params &p, const tt_launch_cfg &cfg) {
+    const bool stats = p.c.st_visits || p.c.st_warp_fetches || p.c.st_warp_steps || p.c.st_warp_mode;
+    return stats ? launch<DIM, KT, true>(p, cfg) : launch<DIM, KT, false>(p, cfg);
+}
+
+template <int DIM>
+int launch_dim(const tt_knn_params &p, const tt_launch_cfg &cfg) {
+    if (p.k <= 1) return launch_k<DIM, 1>(p, cfg);
+    if (p.k <= 4) return launch_k<DIM, 4>(p, cfg);
+    if (p.k <= 8) return launch_k<DIM, 8>(p, cfg);
+    if (p.k <= 16) return launch_k<DIM, 16>(p, cfg);
+    return launch_k<DIM, 32>(p, cfg);
+}
+
+}  // namespace
+
+int tt_launch_knn(const tt_knn_params &p, int dim, const tt_launch_cfg &cfg) {
+    switch (dim) {
+    case 1: return launch_dim<1>(p, cfg);
+    case 2: return launch_dim<2>(p, cfg);
+    case 3: return launch_dim<3>(p, cfg);
+    case 4: return launch_dim<4>(p, cfg);
+    case 5: return launch_dim<5>(p, cfg);
+    case 6: return launch_dim<6>(p, cfg);
+    case 7: return launch_dim<7>(p, cfg);
+    case 8: return launch_dim<8>(p, cfg);
+    case 16: return launch_dim<16>(p, cfg);
+    default: return -1;
+    }
+}

@@ -1,0 +1,282 @@
+// kern_vp.cu -- nearest neighbour in a vantage-point tree (P:L1223-1226,
+// [27] Yianilos), guided with two call sets (inside-first / outside-first),
+// sm_100a.
+//
+// Every node holds a data point (its vantage point), so update() runs at
+// every visited node before the children (Fig.1 line 9).  The
+// non-invariant arguments of the recursive call -- the lower bound lb on the
+// distance to any point of the child subtree and its scale sc -- travel on the
+// rope stack with the node (Fig.7):
+//   inside child:  lb = d - r_in_max,  sc = d + r_in_max
+//   outside child: lb = r_out_min - d, sc = d + r_out_min
+// and the truncation test at pop is lb - tau > eps_vp * (sc + tau) with
+// tau = sqrt(best d2) (reading R12: conservative slack eps_vp = 2^-12).
+// N mode: lane-interleaved per-lane stacks in shared memory; L mode: per-warp
+// {node, mask} stack plus per-lane (lb, sc), majority vote on the call set
+// (§4.3, tie -> inside first).
+#include "kern_common.cuh"
+
+namespace {
+
+using namespace tt;
+
+constexpr int kBlock = 256;
+constexpr int kWarps = kBlock / 32;
+constexpr int kSmemHdr = 128;
+#define TT_VP_EPS 0x1p-12f
+
+__device__ __forceinline__ bool vp_prune(float lb, float sc, float best_d2) {
+    const float tau = __fsqrt_rn(best_d2);
+    return __fsub_rn(lb, tau) > __fmul_rn(TT_VP_EPS, __fadd_rn(sc, tau));
+}
+
+template <int DIM>
+__device__ __forceinline__ void ld_node(const unsigned char *s_rec, const float *s_vpt, const tt_vp_rec *g_rec,
+                                        const float *g_vpt, int dp, int top, int cur, int4 &t, float (&v)[DIM]) {
+    if (cur < top) {
+        t = reinterpret_cast<const int4 *>(s_rec)[cur];
+        load_row_smem<DIM>(v, s_vpt + (size_t)cur * dp);
+    } else {
+        t = __ldg(reinterpret_cast<const int4 *>(g_rec + cur));
+        load_row_nc<DIM>(v, g_vpt + (size_t)cur * dp);
+    }
+}
+
+template <int DIM, bool STATS>
+__global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int cap) {
+    extern __shared__ __align__(128) unsigned char smem[];
+    constexpr int DP = (DIM + 3) & ~3;
+    uint64_t *bar = reinterpret_cast<uint64_t *>(smem);
+    const int top = P.c.top_count;
+    unsigned char *s_rec = smem + kSmemHdr;
+    float *s_vpt = reinterpret_cast<float *>(s_rec + (size_t)top * 16);
+    unsigned char *s_stack = reinterpret_cast<unsigned char *>(s_vpt + (size_t)top * DP);
+    const tt_vp_rec *g_rec = static_cast<const tt_vp_rec *>(P.c.tree.rec);
+    const float *g_vpt = P.c.tree.vpt;
+    StageChunk ch[2] = {{s_rec, g_rec, (unsigned)top * 16u}, {s_vpt, g_vpt, (unsigned)top * 4u * DP}};
+    stage_top(bar, ch);
+
+    const int lane = threadIdx.x & 31;
+    const int warp = threadIdx.x >> 5;
+    // per-warp region of cap*32*12 bytes:
+    //   N: node[cap][32], lb[cap][32], sc[cap][32]
+    //   L: lb[cap][32], sc[cap][32], node[cap], mask[cap]
+    unsigned char *wreg = s_stack + (size_t)warp * cap * 32 * 12;
+    int *n_node = reinterpret_cast<int *>(wreg);
+    float *n_lb = reinterpret_cast<float *>(wreg + (size_t)cap * 32 * 4);
+    float *n_sc = reinterpret_cast<float *>(wreg + (size_t)cap * 32 * 8);
+    float *l_lb = n_lb, *l_sc = n_sc;
+    int *l_node = n_node;
+    unsigned *l_mask = reinterpret_cast<unsigned *>(n_node + cap);
+
+    const long long n = P.c.n;
+    const long long ntiles = (n + 31) >> 5;
+    const float NEG_INF = __int_as_float(0xff800000), POS_INF = __int_as_float(0x7f800000);
+
+    for (;;) {
+        const long long tile = next_tile(P.c.counter);
+        if (tile >= ntiles) break;
+        const long long pos = tile * 32 + lane;
+        const bool valid = pos < n;
+        const long long pid = valid ? (P.c.order ? (long long)P.c.order[pos] : pos) : 0;
+        float q[DIM];
+        if (valid) load_query<DIM>(q, P.q, pid, P.ld);
+        else
+#pragma unroll
+            for (int d = 0; d < DIM; ++d) q[d] = 0.f;
+        const unsigned vmask = __ballot_sync(TT_FULL, valid);
+
+        bool lock = P.c.mode == TT_MODE_LOCKSTEP;
+        if (P.c.mode == TT_MODE_AUTO && P.c.auto_min_depth >= 0 && P.c.auto_min_depth < 64) {
+            // inside/outside descent through the staged top levels
+            int cur = 0, lv = 0;
+            unsigned long long code = 0;
+            const int maxl = min(max(P.c.auto_min_depth, 1), 60);
+            while (lv < maxl && cur >= 0 && cur < top) {
+                int4 t;
+                float v[DIM];
+                ld_node<DIM>(s_rec, s_vpt, g_rec, g_vpt, DP, top, cur, t, v);
+                const float d = __fsqrt_rn(pinned_d2<DIM>(q, v));
+                const bool inside = d <= __int_as_float(t.z);
+                const int nx = inside ? t.x : t.y;
+                if (nx < 0) break;
+                code = (code << 1) | (inside ? 0u : 1u);
+                cur = nx;
+                ++lv;
+            }
+            lock = warp_common_levels(code << (maxl - lv), vmask, 1, maxl) >= P.c.auto_min_depth;
+        }
+
+        float best_d = POS_INF;
+        unsigned best_i = 0xffffffffu;
+        unsigned visits = 0, fetches = 0, steps = 0;
+        if (!lock) {
+            int sp = 0;
+            int cur = valid ? 0 : TT_END;
+            float lb = NEG_INF, sc = 0.f;
+            while (cur != TT_END) {
+                if (STATS) ++visits;
+                if (!vp_prune(lb, sc, best_d)) {
+                    int4 t;
+                    float v[DIM];
+                    ld_node<DIM>(s_rec, s_vpt, g_rec, g_vpt, DP, top, cur, t, v);
+                    const float d2 = pinned_d2<DIM>(q, v);
+                    if (d2 <= best_d) {
+                        const unsigned id = (unsigned)__ldg(P.c.tree.pid + cur);
+                        if (d2 < best_d || id < best_i) {
+                            best_d = d2;
+                            best_i = id;
+                        }
+                    }
+                    const float d = __fsqrt_rn(d2);
+                    const float rin = __int_as_float(t.z), rout = __int_as_float(t.w);
+                    const bool in_first = d <= rin;
+                    const float lb_in = __fsub_rn(d, rin), sc_in = __fadd_rn(d, rin);
+                    const float lb_out = __fsub_rn(rout, d), sc_out = __fadd_rn(d, rout);
+                    const int first = in_first ? t.x : t.y, second = in_first ? t.y : t.x;
+                    if (second != TT_END) {
+                        n_node[sp * 32 + lane] = second;
+                        n_lb[sp * 32 + lane] = in_first ? lb_out : lb_in;
+                        n_sc[sp * 32 + lane] = in_first ? sc_out : sc_in;
+                        ++sp;
+                    }
+                    if (first != TT_END) {
+                        cur = first;
+                        lb = in_first ? lb_in : lb_out;
+                        sc = in_first ? sc_in : sc_out;
+                        continue;
+                    }
+                }
+                if (sp > 0) {
+                    --sp;
+                    cur = n_node[sp * 32 + lane];
+                    lb = n_lb[sp * 32 + lane];
+                    sc = n_sc[sp * 32 + lane];
+                } else {
+                    cur = TT_END;
+                }
+            }
+            if (STATS) {
+                fetches = warp_sum(visits);
+                steps = __reduce_max_sync(TT_FULL, visits);
+            }
+        } else {
+            int sp = 0;
+            int cur = 0;
+            unsigned mask = vmask;
+            float lb = NEG_INF, sc = 0.f;
+            for (;;) {
+                const bool in = (mask >> lane) & 1u;
+                if (STATS) {
+                    ++steps;
+                    visits += in;
+                }
+                const bool active = in && !vp_prune(lb, sc, best_d);
+                const unsigned act = __ballot_sync(TT_FULL, active);
+                if (act) {
+                    if (STATS) ++fetches;
+                    int4 t;
+                    float v[DIM];
+                    ld_node<DIM>(s_rec, s_vpt, g_rec, g_vpt, DP, top, cur, t, v);
+                    const float rin = __int_as_float(t.z), rout = __int_as_float(t.w);
+                    float lb_in = 0.f, sc_in = 0.f, lb_out = 0.f, sc_out = 0.f;
+                    bool pref_in = false;
+                    if (active) {
+                        const float d2 = pinned_d2<DIM>(q, v);
+                        if (d2 <= best_d) {
+                            const unsigned id = (unsigned)__ldg(P.c.tree.pid + cur);
+                            if (d2 < best_d || id < best_i) {
+                                best_d = d2;
+                                best_i = id;
+                            }
+                        }
+                        const float d = __fsqrt_rn(d2);
+                        pref_in = d <= rin;
+                        lb_in = __fsub_rn(d, rin);
+                        sc_in = __fadd_rn(d, rin);
+                        lb_out = __fsub_rn(rout, d);
+                        sc_out = __fadd_rn(d, rout);
+                    }
+                    const int votes = __popc(__ballot_sync(TT_FULL, pref_in));
+                    const bool in_first = 2 * votes >= __popc(act);
+                    const int first = in_first ? t.x : t.y, second = in_first ? t.y : t.x;
+                    if (second != TT_END) {
+                        l_node[sp] = second;
+                        l_mask[sp] = act;
+                        l_lb[sp * 32 + lane] = in_first ? lb_out : lb_in;
+                        l_sc[sp * 32 + lane] = in_first ? sc_out : sc_in;
+                        ++sp;
+                    }
+                    if (first != TT_END) {
+                        cur = first;
+                        mask = act;
+                        lb = in_first ? lb_in : lb_out;
+                        sc = in_first ? sc_in : sc_out;
+                        continue;
+                    }
+                }
+                if (sp == 0) break;
+                --sp;
+                cur = l_node[sp];
+                mask = l_mask[sp];
+                lb = l_lb[sp * 32 + lane];
+                sc = l_sc[sp * 32 + lane];
+            }
+        }
+        if (valid) {
+            P.idx[pid] = best_i == 0xffffffffu ? -1 : (int)best_i;
+            P.d2[pid] = best_d;
+            if (STATS && P.c.st_visits) P.c.st_visits[pid] = visits;
+        }
+        if (STATS) write_warp_stats(P.c, tile, fetches, steps, lock);
+        __syncwarp();
+    }
+    cta_finish(P.c.counter);
+}
+
+template <int DIM, bool STATS>
+int launch(const tt_vp_params &p, const tt_launch_cfg &cfg) {
+    constexpr int DP = (DIM + 3) & ~3;
+    const int cap = p.c.height + 2;
+    const size_t smem = kSmemHdr + (size_t)p.c.top_count * (16 + 4 * DP) + (size_t)kWarps * cap * 32 * 12;
+    auto kern = vp_kernel<DIM, STATS>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return (int)e;
+    int dev = 0, nsm = 0, occ = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kBlock, smem);
+    if (e != cudaSuccess) return (int)e;
+    if (cfg.ctas_per_sm > 0 && cfg.ctas_per_sm < occ) occ = cfg.ctas_per_sm;
+    if (occ < 1) occ = 1;
+    const long long ntiles = (p.c.n + 31) / 32;
+    long long grid = (long long)nsm * occ;
+    const long long need = (ntiles + kWarps - 1) / kWarps;
+    if (grid > need) grid = need;
+    if (grid < 1) grid = 1;
+    kern<<<(unsigned)grid, kBlock, smem, (cudaStream_t)cfg.stream>>>(p, cap);
+    return (int)cudaGetLastError();
+}
+
+template <int DIM>
+int launch_dim(const tt_vp_params &p, const tt_launch_cfg &cfg) {
+    const bool stats = p.c.st_visits || p.c.st_warp_fetches || p.c.st_warp_steps || p.c.st_warp_mode;
+    return stats ? launch<DIM, true>(p, cfg) : launch<DIM, false>(p, cfg);
+}
+
+}  // namespace
+
+int tt_launch_vp(const tt_vp_params &p, int dim, const tt_launch_cfg &cfg) {
+    switch (dim) {
+    case 1: return launch_dim<1>(p, cfg);
+    case 2: return launch_dim<2>(p, cfg);
+    case 3: return launch_dim<3>(p, cfg);
+    case 4: return launch_dim<4>(p, cfg);
+    case 5: return launch_dim<5>(p, cfg);
+    case 6: return launch_dim<6>(p, cfg);
+    case 7: return launch_dim<7>(p, cfg);
+    case 8: return launch_dim<8>(p, cfg);
+    case 16: return launch_dim<16>(p, cfg);
+    default: return -1;
+    }
+}

@@ -1,0 +1,312 @@
+// tt_api.cu -- the C ABI of libtt.so (declared and documented in include/tt.h).
+// Argument checking, tree upload / adoption, and kernel dispatch.  No compute
+// happens here: every step of the traversal runs in the kernels of kern_*.cu.
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <limits>
+#include <cstdio>
+#include <cstring>
+#include <new>
+
+#include "tt_internal.h"
+
+namespace {
+
+std::atomic<int> g_last_cuda_error{0};
+
+tt_status cuda_fail(cudaError_t e) {
+    g_last_cuda_error.store((int)e);
+    if (e == cudaErrorMemoryAllocation) return TT_ERR_OOM;
+    return TT_ERR_CUDA;
+}
+
+tt_status have_device() {
+    int n = 0;
+    cudaError_t e = cudaGetDeviceCount(&n);
+    if (e != cudaSuccess || n <= 0) {
+        g_last_cuda_error.store((int)(e != cudaSuccess ? e : cudaErrorNoDevice));
+        return TT_ERR_CUDA;
+    }
+    return TT_OK;
+}
+
+bool aligned(const void *p, size_t a) { return ((uintptr_t)p % a) == 0; }
+
+bool dim_supported(int d) { return (d >= 1 && d <= 8) || d == 16; }
+
+// Default AUTO thresholds (levels of common tree path for lockstep), see
+// tt_traverse_opts.auto_min_depth and DESIGN.md §4.5.
+constexpr int kAutoBH = 0, kAutoPC = 0, kAutoKNN = 255, kAutoVP = 4;
+
+tt_status setup_common(const tt_tree *t, int kind, int64_t n, const tt_traverse_opts *o, int default_amd,
+                       tt_common_params &c, tt_launch_cfg &cfg, tt_stream s) {
+    if (!t) return TT_ERR_INVALID_ARG;
+    if (t->hdr.kind != kind) return TT_ERR_KIND_MISMATCH;
+    if (n < 0 || n > (int64_t)0xffffffffu * 32) return TT_ERR_INVALID_ARG;
+    std::memset(&c, 0, sizeof(c));
+    c.tree = t->dev;
+    c.top_count = t->hdr.top_count;
+    c.height = t->hdr.height;
+    c.n = n;
+    c.mode = TT_MODE_AUTO;
+    c.auto_min_depth = default_amd;
+    for (int i = 0; i < 3; ++i) c.root_center[i] = t->hdr.root_center[i];
+    c.root_side = t->hdr.root_side;
+    cfg.block_threads = 256;
+    cfg.ctas_per_sm = 0;
+    cfg.stream = s;
+    if (o) {
+        if (o->mode < TT_MODE_AUTO || o->mode > TT_MODE_INDEPENDENT) return TT_ERR_INVALID_ARG;
+        c.mode = o->mode;
+        if (o->auto_min_depth >= 0) c.auto_min_depth = o->auto_min_depth;
+        c.order = o->order;
+        if (o->stats) {
+            c.st_visits = o->stats->visits;
+            c.st_warp_fetches = o->stats->warp_fetches;
+            c.st_warp_steps = o->stats->warp_steps;
+            c.st_warp_mode = o->stats->warp_mode;
+        }
+        if (o->block_threads != 0 && o->block_threads != 256) return TT_ERR_UNSUPPORTED;
+        if (o->ctas_per_sm < 0) return TT_ERR_INVALID_ARG;
+        cfg.ctas_per_sm = o->ctas_per_sm;
+    }
+    unsigned slot = __atomic_fetch_add(&const_cast<tt_tree *>(t)->slot_next, 1u, __ATOMIC_RELAXED) % TT_COUNTER_SLOTS;
+    c.counter = t->d_counters + 2 * slot;
+    return TT_OK;
+}
+
+tt_status finish_launch(int err) {
+    if (err == -1) return TT_ERR_UNSUPPORTED;
+    if (err != 0) return cuda_fail((cudaError_t)err);
+    return TT_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char *tt_status_string(tt_status s) {
+    switch (s) {
+    case TT_OK: return "TT_OK";
+    case TT_ERR_INVALID_ARG: return "TT_ERR_INVALID_ARG";
+    case TT_ERR_CUDA: return "TT_ERR_CUDA";
+    case TT_ERR_OOM: return "TT_ERR_OOM";
+    case TT_ERR_TREE_TOO_DEEP: return "TT_ERR_TREE_TOO_DEEP";
+    case TT_ERR_KIND_MISMATCH: return "TT_ERR_KIND_MISMATCH";
+    case TT_ERR_UNSUPPORTED: return "TT_ERR_UNSUPPORTED";
+    }
+    return "TT_ERR_UNKNOWN";
+}
+
+int32_t tt_last_cuda_error(void) { return g_last_cuda_error.load(); }
+
+const char *tt_build_info(void) {
+    return "libtt sm_100a (-gencode arch=compute_100a,code=sm_100a); blob v1; top budget 32 KiB; block 256";
+}
+
+tt_status tt_tree_pack_size(const tt_tree_desc *d, size_t *bytes) {
+    if (!bytes) return TT_ERR_INVALID_ARG;
+    int st = TT_OK;
+    size_t b = tt_pack_size_impl(d, &st);
+    if (st != TT_OK) return (tt_status)st;
+    *bytes = b;
+    return TT_OK;
+}
+
+tt_status tt_tree_pack(const tt_tree_desc *d, void *host_blob, size_t bytes) {
+    return (tt_status)tt_pack_impl(d, host_blob, bytes);
+}
+
+tt_status tt_tree_from_blob(const void *blob, size_t bytes, int32_t mem, tt_stream s, tt_tree **out) {
+    if (!blob || !out || bytes < sizeof(tt_blob_header)) return TT_ERR_INVALID_ARG;
+    if (mem != TT_MEM_HOST && mem != TT_MEM_DEVICE) return TT_ERR_INVALID_ARG;
+    tt_status st = have_device();
+    if (st != TT_OK) return st;
+    cudaStream_t cs = (cudaStream_t)s;
+    tt_blob_header h;
+    cudaError_t e;
+    if (mem == TT_MEM_HOST) {
+        std::memcpy(&h, blob, sizeof(h));
+    } else {
+        e = cudaMemcpyAsync(&h, blob, sizeof(h), cudaMemcpyDeviceToHost, cs);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
+        if (e != cudaSuccess) return cuda_fail(e);
+    }
+    if (h.magic != TT_BLOB_MAGIC || h.version != TT_BLOB_VERSION || h.total > bytes || h.n_nodes <= 0 ||
+        h.top_count < 1 || h.top_count > h.n_nodes)
+        return TT_ERR_INVALID_ARG;
+    tt_tree *t = new (std::nothrow) tt_tree();
+    if (!t) return TT_ERR_OOM;
+    t->hdr = h;
+    t->bytes = (size_t)h.total;
+    e = cudaMalloc(&t->d_blob, t->bytes);
+    if (e != cudaSuccess) {
+        delete t;
+        return cuda_fail(e);
+    }
+    e = cudaMalloc((void **)&t->d_counters, sizeof(uint32_t) * 2 * TT_COUNTER_SLOTS);
+    if (e == cudaSuccess) e = cudaMemsetAsync(t->d_counters, 0, sizeof(uint32_t) * 2 * TT_COUNTER_SLOTS, cs);
+    if (e == cudaSuccess)
+        e = cudaMemcpyAsync(t->d_blob, blob, t->bytes,
+                            mem == TT_MEM_HOST ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice, cs);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
+    if (e != cudaSuccess) {
+        cudaFree(t->d_blob);
+        if (t->d_counters) cudaFree(t->d_counters);
+        delete t;
+        return cuda_fail(e);
+    }
+    auto *base = static_cast<unsigned char *>(t->d_blob);
+    t->dev.hdr_dev = reinterpret_cast<const tt_blob_header *>(base);
+    t->dev.rec = base + h.off_rec;
+    t->dev.box = h.off_box ? reinterpret_cast<const float *>(base + h.off_box) : nullptr;
+    t->dev.pts = h.off_pts ? reinterpret_cast<const float *>(base + h.off_pts) : nullptr;
+    t->dev.pid = h.off_pid ? reinterpret_cast<const int32_t *>(base + h.off_pid) : nullptr;
+    t->dev.vpt = h.off_vpt ? reinterpret_cast<const float *>(base + h.off_vpt) : nullptr;
+    t->slot_next = 0;
+    *out = t;
+    return TT_OK;
+}
+
+tt_status tt_tree_upload(const tt_tree_desc *d, tt_stream s, tt_tree **out) {
+    if (!out) return TT_ERR_INVALID_ARG;
+    size_t bytes = 0;
+    tt_status st = tt_tree_pack_size(d, &bytes);
+    if (st != TT_OK) return st;
+    st = have_device();
+    if (st != TT_OK) return st;
+    void *host = nullptr;
+    cudaError_t e = cudaMallocHost(&host, bytes);
+    if (e != cudaSuccess) return cuda_fail(e);
+    st = tt_tree_pack(d, host, bytes);
+    if (st == TT_OK) st = tt_tree_from_blob(host, bytes, TT_MEM_HOST, s, out);
+    cudaFreeHost(host);
+    return st;
+}
+
+tt_status tt_tree_free(tt_tree *t) {
+    if (!t) return TT_OK;
+    cudaError_t e1 = cudaFree(t->d_blob);
+    cudaError_t e2 = cudaFree(t->d_counters);
+    delete t;
+    if (e1 != cudaSuccess) return cuda_fail(e1);
+    if (e2 != cudaSuccess) return cuda_fail(e2);
+    return TT_OK;
+}
+
+tt_status tt_tree_get_info(const tt_tree *t, tt_tree_info *o) {
+    if (!t || !o) return TT_ERR_INVALID_ARG;
+    o->kind = t->hdr.kind;
+    o->dim = t->hdr.dim;
+    o->dim_padded = t->hdr.dp;
+    o->height = t->hdr.height;
+    o->n_nodes = t->hdr.n_nodes;
+    o->n_points = t->hdr.n_points;
+    o->top_levels = t->hdr.top_levels;
+    o->top_count = t->hdr.top_count;
+    o->device_bytes = (int64_t)t->bytes;
+    o->device_blob = t->d_blob;
+    return TT_OK;
+}
+
+tt_status tt_sort_points(const tt_tree *t, const float *pts, int64_t n, int32_t ld, uint32_t *perm_out,
+                         uint64_t *keys_out, tt_stream s) {
+    if (!t || n < 0 || n > INT32_MAX) return TT_ERR_INVALID_ARG;
+    if (n == 0) return TT_OK;
+    if (!pts || !perm_out) return TT_ERR_INVALID_ARG;
+    if (ld < (t->hdr.kind == TT_KIND_OCT ? 3 : t->hdr.dim)) return TT_ERR_INVALID_ARG;
+    if (t->hdr.kind != TT_KIND_OCT && !dim_supported(t->hdr.dim)) return TT_ERR_UNSUPPORTED;
+    tt_status st = have_device();
+    if (st != TT_OK) return st;
+    int e = tt_launch_sort(t, pts, n, ld, perm_out, keys_out, s);
+    return e ? cuda_fail((cudaError_t)e) : TT_OK;
+}
+
+tt_status tt_traverse_bh(const tt_tree *t, const float *bodies, const int32_t *self_ids, int64_t n, float theta,
+                         float eps, float *acc_out, const tt_traverse_opts *opts, tt_stream s) {
+    tt_bh_params p;
+    tt_launch_cfg cfg;
+    tt_status st = setup_common(t, TT_KIND_OCT, n, opts, kAutoBH, p.c, cfg, s);
+    if (st != TT_OK) return st;
+    if (!(theta >= 0.0f) || !(eps >= 0.0f)) return TT_ERR_INVALID_ARG;
+    if (n == 0) return TT_OK;
+    if (!bodies || !acc_out || !aligned(bodies, 16) || !aligned(acc_out, 16)) return TT_ERR_INVALID_ARG;
+    st = have_device();
+    if (st != TT_OK) return st;
+    p.bodies = reinterpret_cast<const float4 *>(bodies);
+    p.self_ids = self_ids;
+    // dsq_root = fl32(side^2 / theta^2) in fp64 (reading R8); theta = 0 -> +inf
+    if (theta == 0.0f) {
+        p.dsq_root = std::numeric_limits<float>::infinity();
+    } else {
+        const double th = (double)theta;
+        p.dsq_root = (float)((t->hdr.root_side * t->hdr.root_side) / (th * th));
+    }
+    p.eps2 = eps * eps;
+    p.acc = reinterpret_cast<float4 *>(acc_out);
+    return finish_launch(tt_launch_bh(p, cfg));
+}
+
+tt_status tt_traverse_pc(const tt_tree *t, const float *q, int64_t n, int32_t ld, float radius, uint32_t *count_out,
+                         const tt_traverse_opts *opts, tt_stream s) {
+    tt_pc_params p;
+    tt_launch_cfg cfg;
+    tt_status st = setup_common(t, TT_KIND_KD, n, opts, kAutoPC, p.c, cfg, s);
+    if (st != TT_OK) return st;
+    if (!(radius >= 0.0f)) return TT_ERR_INVALID_ARG;
+    if (ld < t->hdr.dim) return TT_ERR_INVALID_ARG;
+    if (!dim_supported(t->hdr.dim)) return TT_ERR_UNSUPPORTED;
+    if (n == 0) return TT_OK;
+    if (!q || !count_out) return TT_ERR_INVALID_ARG;
+    st = have_device();
+    if (st != TT_OK) return st;
+    p.q = q;
+    p.ld = ld;
+    p.r2 = radius * radius;  // rn(r*r), reading R1
+    p.count = count_out;
+    return finish_launch(tt_launch_pc(p, t->hdr.dim, cfg));
+}
+
+tt_status tt_traverse_knn(const tt_tree *t, const float *q, int64_t n, int32_t ld, int32_t k, int32_t *idx_out,
+                          float *d2_out, const tt_traverse_opts *opts, tt_stream s) {
+    tt_knn_params p;
+    tt_launch_cfg cfg;
+    tt_status st = setup_common(t, TT_KIND_KD, n, opts, kAutoKNN, p.c, cfg, s);
+    if (st != TT_OK) return st;
+    if (k < 1) return TT_ERR_INVALID_ARG;
+    if (k > TT_MAX_K) return TT_ERR_UNSUPPORTED;
+    if (ld < t->hdr.dim) return TT_ERR_INVALID_ARG;
+    if (!dim_supported(t->hdr.dim)) return TT_ERR_UNSUPPORTED;
+    if (n == 0) return TT_OK;
+    if (!q || !idx_out || !d2_out) return TT_ERR_INVALID_ARG;
+    st = have_device();
+    if (st != TT_OK) return st;
+    p.q = q;
+    p.ld = ld;
+    p.k = k;
+    p.idx = idx_out;
+    p.d2 = d2_out;
+    return finish_launch(tt_launch_knn(p, t->hdr.dim, cfg));
+}
+
+tt_status tt_traverse_vp(const tt_tree *t, const float *q, int64_t n, int32_t ld, int32_t *idx_out, float *d2_out,
+                         const tt_traverse_opts *opts, tt_stream s) {
+    tt_vp_params p;
+    tt_launch_cfg cfg;
+    tt_status st = setup_common(t, TT_KIND_VP, n, opts, kAutoVP, p.c, cfg, s);
+    if (st != TT_OK) return st;
+    if (ld < t->hdr.dim) return TT_ERR_INVALID_ARG;
+    if (!dim_supported(t->hdr.dim)) return TT_ERR_UNSUPPORTED;
+    if (n == 0) return TT_OK;
+    if (!q || !idx_out || !d2_out) return TT_ERR_INVALID_ARG;
+    st = have_device();
+    if (st != TT_OK) return st;
+    p.q = q;
+    p.ld = ld;
+    p.idx = idx_out;
+    p.d2 = d2_out;
+    return finish_launch(tt_launch_vp(p, t->hdr.dim, cfg));
+}
+
+}  // extern "C"

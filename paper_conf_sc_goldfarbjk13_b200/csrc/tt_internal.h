@@ -1,0 +1,144 @@
+// tt_internal.h -- device layout of a packed tree and the launch parameter
+// blocks shared between the C-ABI layer (tt_api.cu) and the kernels.
+// Product code only; nothing here is shared with oracle/.
+#pragma once
+
+#include <cstddef>
+#include <cstdint>
+
+#include <vector_types.h>
+
+#include "../../include/tt.h"
+
+#define TT_BLOB_MAGIC 0x31425454u /* "TTB1" */
+#define TT_BLOB_VERSION 1u
+#define TT_END (-1)               /* rope past the last node = end of traversal */
+#define TT_TOP_BYTES (32 * 1024)  /* shared-memory budget for the staged top levels */
+#define TT_COUNTER_SLOTS 256      /* tile-scheduler counter slots per tree */
+
+// ---------------------------------------------------------------------------
+// Packed node records: one 32-byte sector per node, two 128-bit field groups
+// split by use (Fig.9b lines 9/11).
+//
+// OCT: g = {com.x, com.y, com.z, mass}   -- read at every visit
+//      t = {first_child | -1, skip | END, body | -1, level}
+// KD:  t = {left | -1, right | -1, skip | END, level}
+//      u = {split (float bits), split_dim | -1, pbegin, pcount}
+//      + box[2*dp] floats (lo[dp], hi[dp]) in a separate array
+// VP:  t = {in | -1, out | -1, r_in_max (float bits), r_out_min (float bits)}
+//      + vpt[dp] vantage coordinates and pid (vantage point's original id)
+// ---------------------------------------------------------------------------
+struct alignas(16) tt_oct_rec {
+    float gx, gy, gz, gm;
+    int32_t first_child, skip, body, level;
+};
+struct alignas(16) tt_kd_rec {
+    int32_t left, right, skip, level;
+    float split;
+    int32_t dim, pbegin, pcount;
+};
+struct alignas(16) tt_vp_rec {
+    int32_t in, out;
+    float r_in_max, r_out_min;
+};
+static_assert(sizeof(tt_oct_rec) == 32, "oct record = one 32-B sector");
+static_assert(sizeof(tt_kd_rec) == 32, "kd record = one 32-B sector");
+static_assert(sizeof(tt_vp_rec) == 16, "vp header = one 128-bit group");
+
+// Blob = header + sections, every section 256-byte aligned, offsets relative to
+// the blob start (position independent: the blob can be broadcast as bytes).
+struct tt_blob_header {
+    uint32_t magic, version;
+    int32_t kind, dim, dp, height, leaf_size, top_levels, top_count, pad0;
+    int64_t n_nodes, n_points;
+    double root_center[3], root_side;
+    uint64_t off_rec, off_box, off_pts, off_pid, off_vpt, total;
+    uint64_t rec_bytes; // bytes per record in the rec section (32 or 16)
+};
+
+// Device-side view of an uploaded tree.
+struct tt_dev_tree {
+    const tt_blob_header *hdr_dev;
+    const void *rec;      // records, top nodes first
+    const float *box;     // KD: [n_nodes][2*dp]
+    const float *pts;     // KD: [n_points][dp] tree order
+    const int32_t *pid;   // KD: [n_points]; VP: [n_nodes]
+    const float *vpt;     // VP: [n_nodes][dp]
+};
+
+// ---------------------------------------------------------------------------
+// Launch parameter blocks (passed by value to the kernels).
+struct tt_common_params {
+    tt_dev_tree tree;
+    int32_t top_count;     // nodes staged in shared memory
+    int32_t height;
+    int64_t n;             // points in this launch
+    const uint32_t *order; // nullable
+    int32_t mode;          // tt_mode
+    int32_t auto_min_depth;
+    uint32_t *counter;     // [2] tile scheduler: next tile, finished CTAs
+    // stats (nullable)
+    uint32_t *st_visits, *st_warp_fetches, *st_warp_steps;
+    uint8_t *st_warp_mode;
+    // root cube (OCT AUTO mode)
+    double root_center[3], root_side;
+};
+
+struct tt_bh_params {
+    tt_common_params c;
+    const float4 *bodies;
+    const int32_t *self_ids;
+    float dsq_root, eps2;
+    float4 *acc;
+};
+
+struct tt_pc_params {
+    tt_common_params c;
+    const float *q;
+    int32_t ld;
+    float r2;
+    uint32_t *count;
+};
+
+struct tt_knn_params {
+    tt_common_params c;
+    const float *q;
+    int32_t ld, k;
+    int32_t *idx;
+    float *d2;
+};
+
+struct tt_vp_params {
+    tt_common_params c;
+    const float *q;
+    int32_t ld;
+    int32_t *idx;
+    float *d2;
+};
+
+// Host-side handle.
+struct tt_tree {
+    tt_blob_header hdr;
+    void *d_blob;
+    size_t bytes;
+    tt_dev_tree dev;
+    uint32_t *d_counters;  // [TT_COUNTER_SLOTS][2]
+    unsigned slot_next;
+};
+
+// Launchers (kernels/*.cu).  Return a cudaError_t as int.
+struct tt_launch_cfg {
+    int block_threads;
+    int ctas_per_sm;
+    void *stream;
+};
+int tt_launch_bh(const tt_bh_params &p, const tt_launch_cfg &cfg);
+int tt_launch_pc(const tt_pc_params &p, int dim, const tt_launch_cfg &cfg);
+int tt_launch_knn(const tt_knn_params &p, int dim, const tt_launch_cfg &cfg);
+int tt_launch_vp(const tt_vp_params &p, int dim, const tt_launch_cfg &cfg);
+int tt_launch_sort(const tt_tree *t, const float *pts, int64_t n, int32_t ld, uint32_t *perm,
+                   uint64_t *keys_out, void *stream);
+
+// Host helpers (host_build.cpp / pack.cpp)
+size_t tt_pack_size_impl(const tt_tree_desc *d, int *status);
+int tt_pack_impl(const tt_tree_desc *d, void *blob, size_t bytes);

@@ -1,0 +1,69 @@
+"""Multi-GPU driver: one process per GPU, tree replicated by NCCL broadcast,
+points sharded, results all-gathered (north_star).
+
+Points are independent and the tree is read-only during a pass,
+so the traversal itself has no exchange step.  The only collectives are:
+  * ``broadcast_tree``: rank 0 packs the tree (position-independent int32
+    blob, include/tt.h tt_tree_pack) and broadcasts the bytes; every rank
+    adopts them with tt_tree_from_blob(mem=DEVICE) -- once per tree;
+  * ``allgather_rows``: after the pass each rank holds the results of its
+    shard (a contiguous range of point indices) and an in-place
+    all_gather_into_tensor assembles the full result on every rank.
+The same functions run under the gloo backend with CPU tensors for tests
+(the traversal itself needs the GPU; the plumbing does not).
+"""
+from __future__ import annotations
+
+import numpy as np
+import torch
+import torch.distributed as dist
+
+
+def shard_range(n: int, rank: int, world: int) -> tuple[int, int]:
+    """Contiguous equal-count shard [lo, hi) of n points for `rank`."""
+    base, rem = divmod(n, world)
+    lo = rank * base + min(rank, rem)
+    return lo, lo + base + (1 if rank < rem else 0)
+
+
+def broadcast_blob(blob: np.ndarray | None, device, src: int = 0, group=None) -> torch.Tensor:
+    """Broadcast a packed tree blob (uint8) from `src`; returns it on `device`
+    on every rank.  The size travels first as an int64."""
+    rank = dist.get_rank(group)
+    size = torch.zeros(1, dtype=torch.int64, device=device)
+    if rank == src:
+        size[0] = int(blob.size)
+    dist.broadcast(size, src, group=group)
+    if rank == src:
+        buf = torch.from_numpy(np.ascontiguousarray(blob)).to(device)
+    else:
+        buf = torch.empty(int(size.item()), dtype=torch.uint8, device=device)
+    dist.broadcast(buf, src, group=group)
+    return buf
+
+
+def broadcast_tree(host_tree, device, src: int = 0, group=None):
+    """Rank `src` passes its HostTree (others pass None); every rank gets a
+    device Tree adopted from the broadcast blob (tt_tree_from_blob, DEVICE)."""
+    from .tt import tt_tree_from_blob  # GPU path only
+    blob = host_tree.pack() if dist.get_rank(group) == src else None
+    buf = broadcast_blob(blob, device, src, group)
+    return tt_tree_from_blob(buf)
+
+
+def allgather_rows(full: torch.Tensor, world: int, group=None) -> torch.Tensor:
+    """In-place all-gather of equal-size contiguous row shards of `full`
+    (rank r owns rows shard_range(n, r, world)); requires n % world == 0."""
+    n = full.shape[0]
+    if n % world:
+        raise ValueError("allgather_rows needs equal shards (n % world == 0)")
+    rank = dist.get_rank(group)
+    lo, hi = shard_range(n, rank, world)
+    dist.all_gather_into_tensor(full, full[lo:hi].contiguous(), group=group)
+    return full
+
+
+def max_over_ranks(x: float, device, group=None) -> float:
+    t = torch.tensor([x], dtype=torch.float64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX, group=group)
+    return float(t.item())

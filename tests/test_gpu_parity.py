@@ -1,0 +1,332 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the
+same seeded inputs.  Bars:
+  * PC counts, kNN / VP indices and d2, sort permutations, per-point visit
+    counts: bit-exact;
+  * BH accelerations: max_i |a_gpu - a_ref| / |a_ref| <= 1e-4 against the fp64
+    oracle (north_star), with opening decisions pinned (visit counts exact).
+Sizes span many warp tiles and a ragged tail; config-sized cases check
+sampled outputs the oracle computes one by one.
+"""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import ttgen
+
+pytestmark = pytest.mark.gpu
+
+if torch.cuda.is_available():
+    import paper_conf_sc_goldfarbjk13_b200 as P
+
+MODES = ["lockstep", "independent", "auto"]
+BH_TOL = 1e-4
+
+
+def dev(a, dtype=torch.float32):
+    return torch.from_numpy(np.ascontiguousarray(a)).to("cuda", dtype)
+
+
+def perm_i32(p):
+    return dev(p.astype(np.int32), torch.int32)
+
+
+def rel_err(a_gpu, a_ref):
+    return np.linalg.norm(a_gpu[:, :3].astype(np.float64) - a_ref, axis=1) / np.linalg.norm(a_ref, axis=1)
+
+
+# ---------------------------------------------------------------- PC (config 1)
+@pytest.fixture(scope="module")
+def pc_setup():
+    c = ttgen.CONFIGS["pc_10k_3d"]
+    p = ttgen.uniform(c["n"], c["dim"], c["seed"])
+    ot = oracle.build_kd(p, c["leaf"])
+    ref = oracle.pc(ot, p, c["radius"], stats=True)
+    tree = P.tt_tree_upload(P.build_kd(p, c["leaf"]))
+    return c, p, ot, ref, tree
+
+
+@pytest.mark.parametrize("mode", MODES)
+@pytest.mark.parametrize("sorted_", [False, True])
+def test_pc_config1_bit_exact(pc_setup, mode, sorted_):
+    c, p, ot, ref, tree = pc_setup
+    q = dev(p)
+    order = P.tt_sort_points(tree, q) if sorted_ else None
+    st = P.Stats.alloc(len(p), "cuda")
+    cnt = P.tt_traverse_pc(tree, q, c["radius"], order=order, mode=mode, stats=st)
+    torch.cuda.synchronize()
+    assert np.array_equal(cnt.cpu().numpy().astype(np.uint32), ref.out[0])
+    # each lane tests exactly its own recursive visit sequence (both modes)
+    assert np.array_equal(st.visits.cpu().numpy(), ref.visits)
+    if mode == "lockstep":
+        o = order.cpu().numpy() if sorted_ else np.arange(len(p))
+        union = oracle.unguided_warp_union(ot, p[o], c["radius"])
+        assert np.array_equal(st.warp_fetches.cpu().numpy(), union)
+
+
+def test_pc_ragged_and_buckets():
+    p = ttgen.gaussian_mixture(5000, 7, seed=201, components=6)
+    q = ttgen.gaussian_mixture(1237, 7, seed=202, components=6)
+    ot = oracle.build_kd(p, 8)
+    ref = oracle.pc(ot, q, 0.15, stats=True)
+    tree = P.tt_tree_upload(P.build_kd(p, 8))
+    for mode in MODES:
+        st = P.Stats.alloc(len(q), "cuda")
+        cnt = P.tt_traverse_pc(tree, dev(q), 0.15, mode=mode, stats=st)
+        assert np.array_equal(cnt.cpu().numpy().astype(np.uint32), ref.out[0])
+        assert np.array_equal(st.visits.cpu().numpy(), ref.visits)
+
+
+# ------------------------------------------------------------------------ BH
+@pytest.fixture(scope="module")
+def bh_small():
+    b = ttgen.plummer(20011, seed=203)
+    ot = oracle.build_oct(b)
+    ref = oracle.bh(ot, b, 0.5, 0.05, self_ids=np.arange(len(b)), stats=True)
+    tree = P.tt_tree_upload(P.build_oct(b))
+    return b, ot, ref, tree
+
+
+@pytest.mark.parametrize("mode", MODES)
+@pytest.mark.parametrize("sorted_", [False, True])
+def test_bh_within_1e4_and_same_openings(bh_small, mode, sorted_):
+    b, ot, ref, tree = bh_small
+    bd = dev(b)
+    order = P.tt_sort_points(tree, bd) if sorted_ else None
+    st = P.Stats.alloc(len(b), "cuda")
+    acc = P.tt_traverse_bh(tree, bd, 0.5, 0.05, order=order, mode=mode, stats=st).cpu().numpy()
+    err = rel_err(acc, ref.out[0])
+    assert err.max() <= BH_TOL, err.max()
+    assert np.array_equal(st.visits.cpu().numpy(), ref.visits)
+    assert np.all(acc[:, 3] == 0)
+    if mode == "lockstep":
+        o = order.cpu().numpy() if sorted_ else np.arange(len(b))
+        assert np.array_equal(st.warp_fetches.cpu().numpy(), oracle.unguided_warp_union(ot, b[o], 0.5))
+
+
+def test_bh_lockstep_equals_independent_bitwise(bh_small):
+    b, ot, ref, tree = bh_small
+    bd = dev(b)
+    a_l = P.tt_traverse_bh(tree, bd, 0.5, 0.05, mode="lockstep").cpu().numpy()
+    a_n = P.tt_traverse_bh(tree, bd, 0.5, 0.05, mode="independent").cpu().numpy()
+    assert np.array_equal(a_l, a_n)  # same lane op sequence (Fig.8 only masks)
+
+
+def test_bh_theta0_direct_sum_and_duplicates():
+    from tests import brute
+    b = ttgen.plummer(3001, seed=204)
+    b[100, :3] = b[101, :3] = b[102, :3]
+    tree = P.tt_tree_upload(P.build_oct(b))
+    acc = P.tt_traverse_bh(tree, dev(b), 0.0, 0.05).cpu().numpy()
+    err = rel_err(acc, brute.direct_sum(b, 0.05))
+    assert err.max() <= BH_TOL
+
+
+@pytest.mark.slow
+def test_bh_config2_full_size_sampled():
+    c = ttgen.CONFIGS["bh_1m_plummer"]
+    b = ttgen.plummer(c["n"], c["seed"])
+    ot = oracle.build_oct(b)
+    tree = P.tt_tree_upload(P.build_oct(b))
+    bd = dev(b)
+    perm = P.tt_sort_points(tree, bd)
+    st = P.Stats.alloc(len(b), "cuda")
+    acc = P.tt_traverse_bh(tree, bd, c["theta"], c["eps"], order=perm, stats=st).cpu().numpy()
+    rng = np.random.default_rng(0)
+    sample = np.concatenate([rng.choice(len(b), 20000, replace=False),
+                             np.argsort(np.linalg.norm(b[:, :3], axis=1))[:2000]])  # incl. the core
+    ref = oracle.bh(ot, b[sample], c["theta"], c["eps"], self_ids=sample, stats=True)
+    err = rel_err(acc[sample], ref.out[0])
+    assert err.max() <= BH_TOL, err.max()
+    assert np.array_equal(st.visits.cpu().numpy()[sample], ref.visits)
+
+
+# ----------------------------------------------------------------------- kNN
+@pytest.fixture(scope="module")
+def knn_small():
+    p = ttgen.gaussian_mixture(20000, 7, seed=205, components=12)
+    p[500:510] = p[3]
+    q = np.concatenate([ttgen.gaussian_mixture(4990, 7, seed=206, components=12), p[:21]])
+    ot = oracle.build_kd(p, 8)
+    tree = P.tt_tree_upload(P.build_kd(p, 8))
+    return p, q, ot, tree
+
+
+@pytest.mark.parametrize("k", [1, 8, 13, 32])
+def test_knn_independent_bit_exact(knn_small, k):
+    p, q, ot, tree = knn_small
+    ref = oracle.knn(ot, q, k, stats=True)
+    st = P.Stats.alloc(len(q), "cuda")
+    idx, d2 = P.tt_traverse_knn(tree, dev(q), k, mode="independent", stats=st)
+    assert np.array_equal(idx.cpu().numpy(), ref.out[0])
+    assert np.array_equal(d2.cpu().numpy(), ref.out[1])
+    assert np.array_equal(st.visits.cpu().numpy(), ref.visits)  # same order => same pruning
+
+
+@pytest.mark.parametrize("sorted_", [False, True])
+def test_knn_lockstep_matches_fig8_simulation(knn_small, sorted_):
+    p, q, ot, tree = knn_small
+    qd = dev(q)
+    order = P.tt_sort_points(tree, qd) if sorted_ else None
+    o = order.cpu().numpy() if sorted_ else np.arange(len(q))
+    li, ld, lv, wf = oracle.knn_lockstep(ot, q[o], 8)
+    st = P.Stats.alloc(len(q), "cuda")
+    idx, d2 = P.tt_traverse_knn(tree, qd, 8, order=order, mode="lockstep", stats=st)
+    ref = oracle.knn(ot, q, 8)
+    assert np.array_equal(idx.cpu().numpy(), ref.out[0]) and np.array_equal(d2.cpu().numpy(), ref.out[1])
+    assert np.array_equal(st.visits.cpu().numpy()[o], lv)
+    assert np.array_equal(st.warp_fetches.cpu().numpy(), wf)
+
+
+def test_knn_pads_when_k_exceeds_points():
+    p = ttgen.uniform(5, 3, seed=207)
+    tree = P.tt_tree_upload(P.build_kd(p, 2))
+    ref = oracle.knn(oracle.build_kd(p, 2), p, 8)
+    for mode in MODES:
+        idx, d2 = P.tt_traverse_knn(tree, dev(p), 8, mode=mode)
+        assert np.array_equal(idx.cpu().numpy(), ref.out[0]) and np.array_equal(d2.cpu().numpy(), ref.out[1])
+
+
+@pytest.mark.slow
+def test_knn_config3_full_size_sampled():
+    c = ttgen.CONFIGS["knn_1m_7d"]
+    p = ttgen.gaussian_mixture(c["n"], c["dim"], c["seed"])
+    q = ttgen.gaussian_mixture(c["m"], c["dim"], c["qseed"])
+    ot = oracle.build_kd(p, c["leaf"])
+    tree = P.tt_tree_upload(P.build_kd(p, c["leaf"]))
+    qd = dev(q)
+    perm = P.tt_sort_points(tree, qd)
+    idx, d2 = P.tt_traverse_knn(tree, qd, c["k"], order=perm)
+    sample = np.random.default_rng(1).choice(len(q), 3000, replace=False)
+    ref = oracle.knn(ot, q[sample], c["k"])
+    assert np.array_equal(idx.cpu().numpy()[sample], ref.out[0])
+    assert np.array_equal(d2.cpu().numpy()[sample], ref.out[1])
+
+
+# ------------------------------------------------------------------------ VP
+@pytest.fixture(scope="module")
+def vp_small():
+    p = ttgen.gaussian_mixture(20000, 16, seed=208, components=10)
+    p[700:704] = p[9]
+    q = np.concatenate([ttgen.gaussian_mixture(3000, 16, seed=209, components=10), p[:13]])
+    ot = oracle.build_vp(p)
+    tree = P.tt_tree_upload(P.build_vp(p))
+    return p, q, ot, tree
+
+
+def test_vp_independent_bit_exact(vp_small):
+    p, q, ot, tree = vp_small
+    ref = oracle.vp(ot, q, stats=True)
+    st = P.Stats.alloc(len(q), "cuda")
+    idx, d2 = P.tt_traverse_vp(tree, dev(q), mode="independent", stats=st)
+    assert np.array_equal(idx.cpu().numpy(), ref.out[0])
+    assert np.array_equal(d2.cpu().numpy(), ref.out[1])
+    assert np.array_equal(st.visits.cpu().numpy(), ref.visits)
+
+
+@pytest.mark.parametrize("sorted_", [False, True])
+def test_vp_lockstep_matches_simulation(vp_small, sorted_):
+    p, q, ot, tree = vp_small
+    qd = dev(q)
+    order = P.tt_sort_points(tree, qd) if sorted_ else None
+    o = order.cpu().numpy() if sorted_ else np.arange(len(q))
+    li, ld, lv, wf = oracle.vp_lockstep(ot, q[o])
+    st = P.Stats.alloc(len(q), "cuda")
+    idx, d2 = P.tt_traverse_vp(tree, qd, order=order, mode="lockstep", stats=st)
+    assert np.array_equal(idx.cpu().numpy()[o], li) and np.array_equal(d2.cpu().numpy()[o], ld)
+    assert np.array_equal(st.visits.cpu().numpy()[o], lv)
+    assert np.array_equal(st.warp_fetches.cpu().numpy(), wf)
+
+
+def test_vp_auto_results_exact(vp_small):
+    p, q, ot, tree = vp_small
+    ref = oracle.vp(ot, q)
+    qd = dev(q)
+    for sorted_ in (False, True):
+        order = P.tt_sort_points(tree, qd) if sorted_ else None
+        idx, d2 = P.tt_traverse_vp(tree, qd, order=order, mode="auto")
+        assert np.array_equal(idx.cpu().numpy(), ref.out[0]) and np.array_equal(d2.cpu().numpy(), ref.out[1])
+
+
+@pytest.mark.slow
+def test_vp_config4_full_size_sampled():
+    c = ttgen.CONFIGS["vp_1m_16d"]
+    p = ttgen.gaussian_mixture(c["n"], c["dim"], c["seed"])
+    q = ttgen.gaussian_mixture(c["m"], c["dim"], c["qseed"])
+    ot = oracle.build_vp(p)
+    tree = P.tt_tree_upload(P.build_vp(p))
+    qd = dev(q)
+    perm = P.tt_sort_points(tree, qd)
+    idx, d2 = P.tt_traverse_vp(tree, qd, order=perm)
+    sample = np.random.default_rng(2).choice(len(q), 400, replace=False)
+    ref = oracle.vp(ot, q[sample])
+    assert np.array_equal(idx.cpu().numpy()[sample], ref.out[0])
+    assert np.array_equal(d2.cpu().numpy()[sample], ref.out[1])
+
+
+# ---------------------------------------------------------------------- sort
+def test_sort_points_matches_oracle_for_every_kind():
+    b = ttgen.plummer(30000, seed=210)
+    p7 = ttgen.gaussian_mixture(30000, 7, seed=211, components=8)
+    q7 = ttgen.gaussian_mixture(7777, 7, seed=212, components=8)
+    p16 = ttgen.gaussian_mixture(8000, 16, seed=213, components=8)
+    cases = [(P.build_oct(b), oracle.build_oct(b), b),
+             (P.build_kd(p7, 8), oracle.build_kd(p7, 8), q7),
+             (P.build_vp(p16), oracle.build_vp(p16), p16)]
+    for host, ot, pts in cases:
+        tree = P.tt_tree_upload(host)
+        keys = torch.empty(len(pts), dtype=torch.int64, device="cuda")
+        perm = P.tt_sort_points(tree, dev(pts), keys=keys)
+        assert np.array_equal(keys.cpu().numpy().view(np.uint64), oracle.sort_keys(ot, pts))
+        assert np.array_equal(perm.cpu().numpy(), oracle.sort_perm(ot, pts))
+
+
+# ------------------------------------------------------------ edges / misc
+def test_empty_and_partial_warp():
+    p = ttgen.uniform(1000, 3, seed=214)
+    tree = P.tt_tree_upload(P.build_kd(p, 1))
+    ot = oracle.build_kd(p, 1)
+    out = P.tt_traverse_pc(tree, dev(p[:0]), 0.1)
+    assert out.numel() == 0
+    for n in (1, 7, 31, 33):
+        for mode in MODES:
+            cnt = P.tt_traverse_pc(tree, dev(p[:n]), 0.2, mode=mode).cpu().numpy()
+            assert np.array_equal(cnt.astype(np.uint32), oracle.pc(ot, p[:n], 0.2).out[0])
+
+
+def test_kind_mismatch_is_reported():
+    p = ttgen.uniform(100, 3, seed=215)
+    tree = P.tt_tree_upload(P.build_kd(p, 1))
+    with pytest.raises(P.TTError) as e:
+        P.tt_traverse_bh(tree, dev(np.zeros((4, 4), np.float32)), 0.5, 0.05)
+    assert e.value.status == -5
+
+
+def test_sharded_launches_concatenate_to_full_run(bh_small):
+    """Multi-GPU invariant simulated on one GPU: G contiguous slices of the
+    sorted order, run one after another, equal the single run bit for bit."""
+    b, ot, ref, tree = bh_small
+    bd = dev(b)
+    perm = P.tt_sort_points(tree, bd)
+    full = P.tt_traverse_bh(tree, bd, 0.5, 0.05, order=perm).cpu().numpy()
+    out = torch.zeros((len(b), 4), device="cuda")
+    G = 4
+    bounds = np.linspace(0, len(b), G + 1).astype(int)
+    for g in range(G):
+        P.tt_traverse_bh(tree, bd, 0.5, 0.05, order=perm[bounds[g]:bounds[g + 1]].contiguous(), out=out)
+    assert np.array_equal(out.cpu().numpy(), full)
+
+
+def test_blob_roundtrip_device_adoption():
+    """tt_tree_from_blob(mem=DEVICE): the NCCL-broadcast path."""
+    b = ttgen.plummer(5000, seed=216)
+    host = P.build_oct(b)
+    blob = torch.from_numpy(host.pack()).cuda()
+    t1 = P.tt_tree_upload(host)
+    t2 = P.tt_tree_from_blob(blob)
+    bd = dev(b)
+    a1 = P.tt_traverse_bh(t1, bd, 0.5, 0.05).cpu().numpy()
+    a2 = P.tt_traverse_bh(t2, bd, 0.5, 0.05).cpu().numpy()
+    assert np.array_equal(a1, a2)
