@@ -92,7 +92,10 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
             lock = warp_common_levels(code, vmask, 3, lv) >= P.c.auto_min_depth;
         }
 
-        float ax = 0.f, ay = 0.f, az = 0.f;
+        // fp64 accumulation of fp32 terms: the tree-order partial sums of a body
+        // near the centre of mass cancel by 2-3 orders of magnitude, which fp32
+        // accumulation turns into >1e-4 relative error.
+        double ax = 0.0, ay = 0.0, az = 0.0;
         unsigned visits = 0, fetches = 0, steps = 0;
         if (lock) {
             int wait = valid ? INT_MAX : -1;
@@ -115,9 +118,9 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
                     if (!open && t.z != self) {
                         const float inv = rsqrtf(__fadd_rn(drsq, eps2));
                         const float f = g.w * inv * inv * inv;
-                        ax = fmaf(f, dx, ax);
-                        ay = fmaf(f, dy, ay);
-                        az = fmaf(f, dz, az);
+                        ax += (double)(f * dx);
+                        ay += (double)(f * dy);
+                        az += (double)(f * dz);
                     }
                 }
                 cur = __any_sync(TT_FULL, open) ? t.x : t.y;
@@ -138,9 +141,9 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
                 if (!open && t.z != self) {
                     const float inv = rsqrtf(__fadd_rn(drsq, eps2));
                     const float f = g.w * inv * inv * inv;
-                    ax = fmaf(f, dx, ax);
-                    ay = fmaf(f, dy, ay);
-                    az = fmaf(f, dz, az);
+                    ax += (double)(f * dx);
+                    ay += (double)(f * dy);
+                    az += (double)(f * dz);
                 }
                 cur = open ? t.x : t.y;
             }
@@ -150,7 +153,7 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
             }
         }
         if (valid) {
-            P.acc[pid] = make_float4(ax, ay, az, 0.f);
+            P.acc[pid] = make_float4((float)ax, (float)ay, (float)az, 0.f);
             if (STATS && P.c.st_visits) P.c.st_visits[pid] = visits;
         }
         if (STATS) write_warp_stats(P.c, tile, fetches, steps, lock);

@@ -139,6 +139,9 @@ def test_bh_config2_full_size_sampled():
                              np.argsort(np.linalg.norm(b[:, :3], axis=1))[:2000]])  # incl. the core
     ref = oracle.bh(ot, b[sample], c["theta"], c["eps"], self_ids=sample, stats=True)
     err = rel_err(acc[sample], ref.out[0])
+    w = int(np.argmax(err))
+    print(f"BH 1M sampled: max rel err {err.max():.3e} at body {sample[w]} "
+          f"(r={np.linalg.norm(b[sample[w], :3]):.4f}), p99.99 {np.quantile(err, 0.9999):.3e}")
     assert err.max() <= BH_TOL, err.max()
     assert np.array_equal(st.visits.cpu().numpy()[sample], ref.visits)
 
