@@ -11,8 +11,12 @@
 // rope target skip[m]) is not, so the lane re-activates exactly at the node
 // its own traversal visits next.  The warp descends iff any
 // active lane opens the cell (__any_sync = Fig.8's warp_and of masks).
-// Each lane therefore tests exactly its own recursive visit sequence: results
-// and per-point visit counts are bit-identical to the independent walk.
+// Each lane therefore tests exactly its own recursive visit sequence: opening
+// decisions and per-point visit counts are identical to the independent walk
+// (results differ only by the fp32->fp64 flush cadence of the accumulator).
+#include <cfloat>
+#include <cmath>
+
 #include "kern_common.cuh"
 
 namespace {
@@ -22,16 +26,46 @@ using namespace tt;
 constexpr int kBlock = 256;
 constexpr int kSmemHdr = 384;  // [0,16) mbarrier, [16,272) dsq table (64 floats)
 
-__device__ __forceinline__ void ld_rec(const tt_oct_rec *s_top, const tt_oct_rec *g, int top, int cur,
+// Record fetch through one generic pointer: the staged top levels live in
+// shared memory, the rest in global memory (L1/L2-cached); selecting the base
+// costs one SEL instead of two predicated load pairs.
+__device__ __forceinline__ void ld_rec(const unsigned char *s_base, const unsigned char *g_base, int top, int cur,
                                        float4 &gg, int4 &tt) {
-    if (cur < top) {
-        gg = *reinterpret_cast<const float4 *>(&s_top[cur].gx);
-        tt = *reinterpret_cast<const int4 *>(&s_top[cur].first_child);
-    } else {
-        gg = __ldg(reinterpret_cast<const float4 *>(&g[cur].gx));
-        tt = __ldg(reinterpret_cast<const int4 *>(&g[cur].first_child));
-    }
+    const unsigned char *p = (cur < top ? s_base : g_base) + (size_t)cur * 32u;
+    gg = *reinterpret_cast<const float4 *>(p);
+    tt = *reinterpret_cast<const int4 *>(p + 16);
 }
+
+// dsq_L = dsq_root * 0.25^L by exponent arithmetic: exact (a power-of-4
+// scaling of a normal float), bit-identical to repeated "dsq*0.25" (Fig.9a
+// line 4) -- the host checks dsq_root * 0.25^height stays normal, else the
+// table path is used.  theta = 0 (dsq_root = +inf) opens every cell.
+__device__ __forceinline__ float dsq_at(int dsq_bits, bool inf_root, int lvl) {
+    return inf_root ? __int_as_float(0x7f800000) : __int_as_float(dsq_bits - (lvl << 24));
+}
+
+// Interaction (update(), Fig.9a line 6): a += m (c - x) / (|c - x|^2 + eps^2)^{3/2}.
+// Terms go into fp32 partial sums that are flushed into fp64 every
+// kFlush steps: the fp32 partials stay small, so the
+// cancellation of a body near the centre of mass costs no accuracy.
+constexpr int kFlush = 16;
+struct Acc {
+    float x = 0.f, y = 0.f, z = 0.f;
+    double X = 0.0, Y = 0.0, Z = 0.0;
+    __device__ __forceinline__ void add(float m, float dx, float dy, float dz, float drsq, float eps2) {
+        const float inv = rsqrt_ftz(__fadd_rn(drsq, eps2));
+        const float f = m * (inv * inv) * inv;
+        x = fmaf(f, dx, x);
+        y = fmaf(f, dy, y);
+        z = fmaf(f, dz, z);
+    }
+    __device__ __forceinline__ void flush() {
+        X += (double)x;
+        Y += (double)y;
+        Z += (double)z;
+        x = y = z = 0.f;
+    }
+};
 
 // 63-bit octant path of a body through the root cube (fp64 comparisons, R8a).
 __device__ __forceinline__ unsigned long long oct_path(float4 b, const double c0[3], double side, int levels) {
@@ -49,7 +83,7 @@ __device__ __forceinline__ unsigned long long oct_path(float4 b, const double c0
     return code;
 }
 
-template <bool STATS>
+template <bool STATS, bool EXP_DSQ>
 __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
     extern __shared__ __align__(128) unsigned char smem[];
     uint64_t *bar = reinterpret_cast<uint64_t *>(smem);
@@ -74,6 +108,11 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
     const long long n = P.c.n;
     const long long ntiles = (n + 31) >> 5;
     const float eps2 = P.eps2;
+    const unsigned char *s_base = reinterpret_cast<const unsigned char *>(s_top);
+    const unsigned char *g_base = reinterpret_cast<const unsigned char *>(g_rec);
+    const int dsq_bits = __float_as_int(P.dsq_root);
+    const bool inf_root = !(P.dsq_root < __int_as_float(0x7f800000));
+    auto dsq = [&](int lvl) { return EXP_DSQ ? dsq_at(dsq_bits, inf_root, lvl) : s_dsq[lvl]; };
 
     for (;;) {
         const long long tile = next_tile(P.c.counter);
@@ -92,60 +131,57 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
             lock = warp_common_levels(code, vmask, 3, lv) >= P.c.auto_min_depth;
         }
 
-        // fp64 accumulation of fp32 terms: the tree-order partial sums of a body
-        // near the centre of mass cancel by 2-3 orders of magnitude, which fp32
-        // accumulation turns into >1e-4 relative error.
-        double ax = 0.0, ay = 0.0, az = 0.0;
+        Acc acc;
         unsigned visits = 0, fetches = 0, steps = 0;
         if (lock) {
             int wait = valid ? INT_MAX : -1;
             int cur = 0;
-            while (cur != TT_END) {
-                float4 g;
-                int4 t;
-                ld_rec(s_top, g_rec, top, cur, g, t);
-                if (STATS) ++steps;
-                const int lvl = t.w;
-                const bool active = lvl <= wait;
-                const float dx = __fsub_rn(g.x, b.x);
-                const float dy = __fsub_rn(g.y, b.y);
-                const float dz = __fsub_rn(g.z, b.z);
-                const float drsq = __fadd_rn(__fadd_rn(__fmul_rn(dx, dx), __fmul_rn(dy, dy)), __fmul_rn(dz, dz));
-                const bool open = active && t.x >= 0 && drsq < s_dsq[lvl];
-                if (active) {
-                    if (STATS) ++visits;
-                    wait = open ? INT_MAX : lvl;
-                    if (!open && t.z != self) {
-                        const float inv = rsqrtf(__fadd_rn(drsq, eps2));
-                        const float f = g.w * inv * inv * inv;
-                        ax += (double)(f * dx);
-                        ay += (double)(f * dy);
-                        az += (double)(f * dz);
-                    }
+            for (;;) {
+#pragma unroll 1
+                for (int k = 0; k < kFlush; ++k) {
+                    float4 g;
+                    int4 t;
+                    ld_rec(s_base, g_base, top, cur, g, t);
+                    if (STATS) ++steps;
+                    const int lvl = t.w;
+                    const bool active = lvl <= wait;
+                    const float dx = __fsub_rn(g.x, b.x);
+                    const float dy = __fsub_rn(g.y, b.y);
+                    const float dz = __fsub_rn(g.z, b.z);
+                    const float drsq =
+                        __fadd_rn(__fadd_rn(__fmul_rn(dx, dx), __fmul_rn(dy, dy)), __fmul_rn(dz, dz));
+                    const bool near = drsq < dsq(lvl);
+                    const bool open = active && t.x >= 0 && near;
+                    if (STATS) visits += active;
+                    wait = active ? (open ? INT_MAX : lvl) : wait;
+                    if (active && !open && t.z != self) acc.add(g.w, dx, dy, dz, drsq, eps2);
+                    cur = __any_sync(TT_FULL, open) ? t.x : t.y;
+                    if (cur == TT_END) break;
                 }
-                cur = __any_sync(TT_FULL, open) ? t.x : t.y;
+                acc.flush();  // warp-uniform
+                if (cur == TT_END) break;
             }
             fetches = steps;
         } else {
             int cur = valid ? 0 : TT_END;
             while (cur != TT_END) {
-                float4 g;
-                int4 t;
-                ld_rec(s_top, g_rec, top, cur, g, t);
-                if (STATS) ++visits;
-                const float dx = __fsub_rn(g.x, b.x);
-                const float dy = __fsub_rn(g.y, b.y);
-                const float dz = __fsub_rn(g.z, b.z);
-                const float drsq = __fadd_rn(__fadd_rn(__fmul_rn(dx, dx), __fmul_rn(dy, dy)), __fmul_rn(dz, dz));
-                const bool open = t.x >= 0 && drsq < s_dsq[t.w];
-                if (!open && t.z != self) {
-                    const float inv = rsqrtf(__fadd_rn(drsq, eps2));
-                    const float f = g.w * inv * inv * inv;
-                    ax += (double)(f * dx);
-                    ay += (double)(f * dy);
-                    az += (double)(f * dz);
+#pragma unroll 1
+                for (int k = 0; k < kFlush; ++k) {
+                    float4 g;
+                    int4 t;
+                    ld_rec(s_base, g_base, top, cur, g, t);
+                    if (STATS) ++visits;
+                    const float dx = __fsub_rn(g.x, b.x);
+                    const float dy = __fsub_rn(g.y, b.y);
+                    const float dz = __fsub_rn(g.z, b.z);
+                    const float drsq =
+                        __fadd_rn(__fadd_rn(__fmul_rn(dx, dx), __fmul_rn(dy, dy)), __fmul_rn(dz, dz));
+                    const bool open = t.x >= 0 && drsq < dsq(t.w);
+                    if (!open && t.z != self) acc.add(g.w, dx, dy, dz, drsq, eps2);
+                    cur = open ? t.x : t.y;
+                    if (cur == TT_END) break;
                 }
-                cur = open ? t.x : t.y;
+                acc.flush();
             }
             if (STATS) {
                 fetches = warp_sum(visits);
@@ -153,7 +189,7 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
             }
         }
         if (valid) {
-            P.acc[pid] = make_float4((float)ax, (float)ay, (float)az, 0.f);
+            P.acc[pid] = make_float4((float)acc.X, (float)acc.Y, (float)acc.Z, 0.f);
             if (STATS && P.c.st_visits) P.c.st_visits[pid] = visits;
         }
         if (STATS) write_warp_stats(P.c, tile, fetches, steps, lock);
@@ -161,10 +197,10 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
     cta_finish(P.c.counter);
 }
 
-template <bool STATS>
+template <bool STATS, bool EXP_DSQ>
 int launch(const tt_bh_params &p, const tt_launch_cfg &cfg) {
     const size_t smem = kSmemHdr + (size_t)p.c.top_count * 32;
-    auto kern = bh_kernel<STATS>;
+    auto kern = bh_kernel<STATS, EXP_DSQ>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return (int)e;
     int dev = 0, nsm = 0, occ = 0;
@@ -187,5 +223,10 @@ int launch(const tt_bh_params &p, const tt_launch_cfg &cfg) {
 
 int tt_launch_bh(const tt_bh_params &p, const tt_launch_cfg &cfg) {
     const bool stats = p.c.st_visits || p.c.st_warp_fetches || p.c.st_warp_steps || p.c.st_warp_mode;
-    return stats ? launch<true>(p, cfg) : launch<false>(p, cfg);
+    // exponent-arithmetic dsq is exact iff dsq_root * 0.25^height is a normal float
+    // (or dsq_root = +inf, theta = 0); otherwise use the shared-memory table
+    const float r = p.dsq_root;
+    const bool exp_ok = !(r < INFINITY) || (r > 0.f && std::ldexp((double)r, -2 * p.c.height) >= (double)FLT_MIN);
+    if (stats) return exp_ok ? launch<true, true>(p, cfg) : launch<true, false>(p, cfg);
+    return exp_ok ? launch<false, true>(p, cfg) : launch<false, false>(p, cfg);
 }

@@ -164,6 +164,34 @@ __device__ __forceinline__ float select_dim(const float (&q)[DIM], int dim) {
     return v;
 }
 
+// ------------------------------------------------ shared-space loads (LDS)
+// 32-bit shared-window addresses kept in registers: generic pointers into
+// dynamic shared memory make nvcc re-derive the window base (S2R CgaCtaId)
+// inside every loop iteration.
+__device__ __forceinline__ unsigned smem_addr(const void *p) { return (unsigned)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ float4 lds_f4(unsigned a) {
+    float4 v;
+    asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ int4 lds_i4(unsigned a) {
+    int4 v;
+    asm volatile("ld.shared.v4.s32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ float lds_f(unsigned a) {
+    float v;
+    asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(a));
+    return v;
+}
+// rsqrt without the denormal-input fixup (arguments are >= eps^2 > 0 or
+// normal); the result only feeds the force magnitude, not a decision.
+__device__ __forceinline__ float rsqrt_ftz(float x) {
+    float y;
+    asm("rsqrt.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
+}
+
 // ------------------------------------------------------- warp-level helpers
 // Number of leading tree levels on which all valid lanes agree, given a path
 // code with `bits` bits per level packed in the low `bits*levels` bits.

@@ -11,8 +11,12 @@
 //   outside child: lb = r_out_min - d, sc = d + r_out_min
 // and the truncation test at pop is lb - tau > eps_vp * (sc + tau) with
 // tau = sqrt(best d2) (reading R12: conservative slack eps_vp = 2^-12).
+// A stack entry stores (parent << 1 | side) and the lane's distance d to the
+// parent's vantage point; (lb, sc) and the child index are recomputed at pop
+// from the parent's 16-B header with the same fp32 operations as at push, so
+// the arguments are bit-identical while an entry costs 8 B instead of 12.
 // N mode: lane-interleaved per-lane stacks in shared memory; L mode: per-warp
-// {node, mask} stack plus per-lane (lb, sc), majority vote on the call set
+// {parent|side, mask} stack plus per-lane d, majority vote on the call set
 // (§4.3, tie -> inside first).
 #include "kern_common.cuh"
 
@@ -42,6 +46,14 @@ __device__ __forceinline__ void ld_node(const unsigned char *s_rec, const float 
     }
 }
 
+// Child of `parent` on `side` (0 = inside, 1 = outside) and its (lb, sc).
+__device__ __forceinline__ int child_args(int4 t, int side, float d, float &lb, float &sc) {
+    const float rin = __int_as_float(t.z), rout = __int_as_float(t.w);
+    lb = side ? __fsub_rn(rout, d) : __fsub_rn(d, rin);
+    sc = side ? __fadd_rn(d, rout) : __fadd_rn(d, rin);
+    return side ? t.y : t.x;
+}
+
 template <int DIM, bool STATS>
 __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int cap) {
     extern __shared__ __align__(128) unsigned char smem[];
@@ -58,16 +70,21 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
 
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
-    // per-warp region of cap*32*12 bytes:
-    //   N: node[cap][32], lb[cap][32], sc[cap][32]
-    //   L: lb[cap][32], sc[cap][32], node[cap], mask[cap]
-    unsigned char *wreg = s_stack + (size_t)warp * cap * 32 * 12;
-    int *n_node = reinterpret_cast<int *>(wreg);
-    float *n_lb = reinterpret_cast<float *>(wreg + (size_t)cap * 32 * 4);
-    float *n_sc = reinterpret_cast<float *>(wreg + (size_t)cap * 32 * 8);
-    float *l_lb = n_lb, *l_sc = n_sc;
-    int *l_node = n_node;
-    unsigned *l_mask = reinterpret_cast<unsigned *>(n_node + cap);
+    // per-warp region of cap*32*8 bytes:
+    //   N: ent[cap][32] (parent<<1|side), d[cap][32]
+    //   L: d[cap][32], ent[cap], mask[cap]
+    unsigned char *wreg = s_stack + (size_t)warp * cap * 32 * 8;
+    int *n_ent = reinterpret_cast<int *>(wreg);
+    float *n_d = reinterpret_cast<float *>(wreg + (size_t)cap * 32 * 4);
+    float *l_d = reinterpret_cast<float *>(wreg);
+    int *l_ent = reinterpret_cast<int *>(wreg + (size_t)cap * 32 * 4);
+    unsigned *l_mask = reinterpret_cast<unsigned *>(l_ent + cap);
+    const unsigned char *s_hdr_base = s_rec;
+    const unsigned char *g_hdr_base = reinterpret_cast<const unsigned char *>(g_rec);
+    auto hdr = [&](int node) -> int4 {
+        const unsigned char *p = (node < top ? s_hdr_base : g_hdr_base) + (size_t)node * 16;
+        return *reinterpret_cast<const int4 *>(p);
+    };
 
     const long long n = P.c.n;
     const long long ntiles = (n + 31) >> 5;
@@ -129,29 +146,23 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
                         }
                     }
                     const float d = __fsqrt_rn(d2);
-                    const float rin = __int_as_float(t.z), rout = __int_as_float(t.w);
-                    const bool in_first = d <= rin;
-                    const float lb_in = __fsub_rn(d, rin), sc_in = __fadd_rn(d, rin);
-                    const float lb_out = __fsub_rn(rout, d), sc_out = __fadd_rn(d, rout);
-                    const int first = in_first ? t.x : t.y, second = in_first ? t.y : t.x;
+                    const int first_side = d <= __int_as_float(t.z) ? 0 : 1;
+                    const int second = first_side ? t.x : t.y;
                     if (second != TT_END) {
-                        n_node[sp * 32 + lane] = second;
-                        n_lb[sp * 32 + lane] = in_first ? lb_out : lb_in;
-                        n_sc[sp * 32 + lane] = in_first ? sc_out : sc_in;
+                        n_ent[sp * 32 + lane] = (cur << 1) | (first_side ^ 1);
+                        n_d[sp * 32 + lane] = d;
                         ++sp;
                     }
+                    const int first = child_args(t, first_side, d, lb, sc);
                     if (first != TT_END) {
                         cur = first;
-                        lb = in_first ? lb_in : lb_out;
-                        sc = in_first ? sc_in : sc_out;
                         continue;
                     }
                 }
                 if (sp > 0) {
                     --sp;
-                    cur = n_node[sp * 32 + lane];
-                    lb = n_lb[sp * 32 + lane];
-                    sc = n_sc[sp * 32 + lane];
+                    const int e = n_ent[sp * 32 + lane];
+                    cur = child_args(hdr(e >> 1), e & 1, n_d[sp * 32 + lane], lb, sc);
                 } else {
                     cur = TT_END;
                 }
@@ -178,8 +189,7 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
                     int4 t;
                     float v[DIM];
                     ld_node<DIM>(s_rec, s_vpt, g_rec, g_vpt, DP, top, cur, t, v);
-                    const float rin = __int_as_float(t.z), rout = __int_as_float(t.w);
-                    float lb_in = 0.f, sc_in = 0.f, lb_out = 0.f, sc_out = 0.f;
+                    float d = 0.f;
                     bool pref_in = false;
                     if (active) {
                         const float d2 = pinned_d2<DIM>(q, v);
@@ -190,37 +200,30 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
                                 best_i = id;
                             }
                         }
-                        const float d = __fsqrt_rn(d2);
-                        pref_in = d <= rin;
-                        lb_in = __fsub_rn(d, rin);
-                        sc_in = __fadd_rn(d, rin);
-                        lb_out = __fsub_rn(rout, d);
-                        sc_out = __fadd_rn(d, rout);
+                        d = __fsqrt_rn(d2);
+                        pref_in = d <= __int_as_float(t.z);
                     }
                     const int votes = __popc(__ballot_sync(TT_FULL, pref_in));
-                    const bool in_first = 2 * votes >= __popc(act);
-                    const int first = in_first ? t.x : t.y, second = in_first ? t.y : t.x;
+                    const int first_side = 2 * votes >= __popc(act) ? 0 : 1;
+                    const int second = first_side ? t.x : t.y;
                     if (second != TT_END) {
-                        l_node[sp] = second;
+                        l_ent[sp] = (cur << 1) | (first_side ^ 1);  // all lanes write the same value
                         l_mask[sp] = act;
-                        l_lb[sp * 32 + lane] = in_first ? lb_out : lb_in;
-                        l_sc[sp * 32 + lane] = in_first ? sc_out : sc_in;
+                        l_d[sp * 32 + lane] = d;
                         ++sp;
                     }
+                    const int first = child_args(t, first_side, d, lb, sc);
                     if (first != TT_END) {
                         cur = first;
                         mask = act;
-                        lb = in_first ? lb_in : lb_out;
-                        sc = in_first ? sc_in : sc_out;
                         continue;
                     }
                 }
                 if (sp == 0) break;
                 --sp;
-                cur = l_node[sp];
+                const int e = l_ent[sp];
                 mask = l_mask[sp];
-                lb = l_lb[sp * 32 + lane];
-                sc = l_sc[sp * 32 + lane];
+                cur = child_args(hdr(e >> 1), e & 1, l_d[sp * 32 + lane], lb, sc);
             }
         }
         if (valid) {
@@ -238,7 +241,7 @@ template <int DIM, bool STATS>
 int launch(const tt_vp_params &p, const tt_launch_cfg &cfg) {
     constexpr int DP = (DIM + 3) & ~3;
     const int cap = p.c.height + 2;
-    const size_t smem = kSmemHdr + (size_t)p.c.top_count * (16 + 4 * DP) + (size_t)kWarps * cap * 32 * 12;
+    const size_t smem = kSmemHdr + (size_t)p.c.top_count * (16 + 4 * DP) + (size_t)kWarps * cap * 32 * 8;
     auto kern = vp_kernel<DIM, STATS>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return (int)e;

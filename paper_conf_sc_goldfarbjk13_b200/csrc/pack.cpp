@@ -7,11 +7,12 @@
 //   * one 32-byte record per node = one DRAM/L2 sector, read as two 128-bit
 //     loads (the use-split groups of Fig.9b lines 9 and 11);
 //   * int32 node indices, rope (skip) stored on every node (Fig.2 ropes);
-//   * the nodes of the top `top_levels` levels are renumbered first (in
-//     preorder among themselves), the rest follow in preorder, so a single
-//     bulk copy stages the top of the tree in shared memory.  The walk only
-//     follows explicit child / rope indices and node levels, so it is
-//     independent of the numbering.
+//   * the nodes of the top `top_levels` levels are renumbered first, level by
+//     level (preorder within a level), the rest follow in preorder, so one
+//     bulk copy of a prefix stages the top L levels in shared memory (each
+//     kernel picks the L that fits its budget).  The walk only follows
+//     explicit child / rope indices and node levels, so it is independent of
+//     the numbering.
 #include <cstring>
 #include <new>
 #include <vector>
@@ -23,10 +24,6 @@ namespace {
 inline uint64_t align256(uint64_t x) { return (x + 255) & ~uint64_t(255); }
 
 int dim_padded(int dim) { return (dim + 3) & ~3; }
-
-struct Layout {
-    tt_blob_header h;
-};
 
 int stage_bytes_per_node(int kind, int dp) {
     if (kind == TT_KIND_OCT) return 32;
@@ -95,9 +92,11 @@ void plan(const tt_tree_desc *d, tt_blob_header &h, std::vector<int32_t> *newidx
     const int sb = stage_bytes_per_node(d->kind, h.dp);
     int64_t acc = 0;
     int L = 0;
-    while (L <= d->height && (acc + per_level[(size_t)L]) * sb <= TT_TOP_BYTES) {
+    h.level_prefix[0] = 0;
+    while (L <= d->height && L < TT_TOP_LEVELS_MAX && (acc + per_level[(size_t)L]) * sb <= TT_TOP_BYTES) {
         acc += per_level[(size_t)L];
         ++L;
+        h.level_prefix[L] = (int32_t)acc;
     }
     h.top_levels = L;
     h.top_count = (int32_t)acc;
@@ -120,10 +119,15 @@ void plan(const tt_tree_desc *d, tt_blob_header &h, std::vector<int32_t> *newidx
     }
     h.total = off;
     if (newidx) {
+        // top region level by level (preorder within a level), then the rest
+        // of the tree in preorder
         newidx->assign((size_t)d->n_nodes, -1);
-        int32_t a = 0, b = h.top_count;
-        for (int64_t v = 0; v < d->n_nodes; ++v)
-            (*newidx)[(size_t)v] = d->level[v] < h.top_levels ? a++ : b++;
+        std::vector<int32_t> next(h.level_prefix, h.level_prefix + h.top_levels + 1);
+        int32_t b = h.top_count;
+        for (int64_t v = 0; v < d->n_nodes; ++v) {
+            const int l = d->level[v];
+            (*newidx)[(size_t)v] = l < h.top_levels ? next[(size_t)l]++ : b++;
+        }
     }
 }
 

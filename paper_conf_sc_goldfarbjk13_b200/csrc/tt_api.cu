@@ -37,16 +37,21 @@ bool dim_supported(int d) { return (d >= 1 && d <= 8) || d == 16; }
 
 // Default AUTO thresholds (levels of common tree path for lockstep), see
 // tt_traverse_opts.auto_min_depth and DESIGN.md §4.5.
-constexpr int kAutoBH = 0, kAutoPC = 0, kAutoKNN = 255, kAutoVP = 4;
+constexpr int kAutoBH = 0, kAutoPC = 0, kAutoKNN = 4, kAutoVP = 4;
+
+// Shared-memory budgets for the staged top levels, per kernel (bytes/node):
+// the budget trades staged levels against occupancy.
+constexpr int kTopBH = 32 * 1024, kTopPC = 32 * 1024, kTopKNN = 16 * 1024, kTopVP = 4 * 1024;
 
 tt_status setup_common(const tt_tree *t, int kind, int64_t n, const tt_traverse_opts *o, int default_amd,
-                       tt_common_params &c, tt_launch_cfg &cfg, tt_stream s) {
+                       int stage_bytes_per_node, int stage_budget, tt_common_params &c, tt_launch_cfg &cfg,
+                       tt_stream s) {
     if (!t) return TT_ERR_INVALID_ARG;
     if (t->hdr.kind != kind) return TT_ERR_KIND_MISMATCH;
     if (n < 0 || n > (int64_t)0xffffffffu * 32) return TT_ERR_INVALID_ARG;
     std::memset(&c, 0, sizeof(c));
     c.tree = t->dev;
-    c.top_count = t->hdr.top_count;
+    c.top_count = tt_stage_count(t->hdr, stage_bytes_per_node, stage_budget);
     c.height = t->hdr.height;
     c.n = n;
     c.mode = TT_MODE_AUTO;
@@ -227,7 +232,7 @@ tt_status tt_traverse_bh(const tt_tree *t, const float *bodies, const int32_t *s
                          float eps, float *acc_out, const tt_traverse_opts *opts, tt_stream s) {
     tt_bh_params p;
     tt_launch_cfg cfg;
-    tt_status st = setup_common(t, TT_KIND_OCT, n, opts, kAutoBH, p.c, cfg, s);
+    tt_status st = setup_common(t, TT_KIND_OCT, n, opts, kAutoBH, 32, kTopBH, p.c, cfg, s);
     if (st != TT_OK) return st;
     if (!(theta >= 0.0f) || !(eps >= 0.0f)) return TT_ERR_INVALID_ARG;
     if (n == 0) return TT_OK;
@@ -252,7 +257,7 @@ tt_status tt_traverse_pc(const tt_tree *t, const float *q, int64_t n, int32_t ld
                          const tt_traverse_opts *opts, tt_stream s) {
     tt_pc_params p;
     tt_launch_cfg cfg;
-    tt_status st = setup_common(t, TT_KIND_KD, n, opts, kAutoPC, p.c, cfg, s);
+    tt_status st = setup_common(t, TT_KIND_KD, n, opts, kAutoPC, 32 + 8 * t->hdr.dp, kTopPC, p.c, cfg, s);
     if (st != TT_OK) return st;
     if (!(radius >= 0.0f)) return TT_ERR_INVALID_ARG;
     if (ld < t->hdr.dim) return TT_ERR_INVALID_ARG;
@@ -272,7 +277,7 @@ tt_status tt_traverse_knn(const tt_tree *t, const float *q, int64_t n, int32_t l
                           float *d2_out, const tt_traverse_opts *opts, tt_stream s) {
     tt_knn_params p;
     tt_launch_cfg cfg;
-    tt_status st = setup_common(t, TT_KIND_KD, n, opts, kAutoKNN, p.c, cfg, s);
+    tt_status st = setup_common(t, TT_KIND_KD, n, opts, kAutoKNN, 32 + 8 * t->hdr.dp, kTopKNN, p.c, cfg, s);
     if (st != TT_OK) return st;
     if (k < 1) return TT_ERR_INVALID_ARG;
     if (k > TT_MAX_K) return TT_ERR_UNSUPPORTED;
@@ -294,7 +299,7 @@ tt_status tt_traverse_vp(const tt_tree *t, const float *q, int64_t n, int32_t ld
                          const tt_traverse_opts *opts, tt_stream s) {
     tt_vp_params p;
     tt_launch_cfg cfg;
-    tt_status st = setup_common(t, TT_KIND_VP, n, opts, kAutoVP, p.c, cfg, s);
+    tt_status st = setup_common(t, TT_KIND_VP, n, opts, kAutoVP, 16 + 4 * t->hdr.dp, kTopVP, p.c, cfg, s);
     if (st != TT_OK) return st;
     if (ld < t->hdr.dim) return TT_ERR_INVALID_ARG;
     if (!dim_supported(t->hdr.dim)) return TT_ERR_UNSUPPORTED;

@@ -15,6 +15,7 @@
 #define TT_END (-1)               /* rope past the last node = end of traversal */
 #define TT_TOP_BYTES (32 * 1024)  /* shared-memory budget for the staged top levels */
 #define TT_COUNTER_SLOTS 256      /* tile-scheduler counter slots per tree */
+#define TT_TOP_LEVELS_MAX 32      /* levels tracked in the header's level_prefix */
 
 // ---------------------------------------------------------------------------
 // Packed node records: one 32-byte sector per node, two 128-bit field groups
@@ -50,6 +51,10 @@ static_assert(sizeof(tt_vp_rec) == 16, "vp header = one 128-bit group");
 struct tt_blob_header {
     uint32_t magic, version;
     int32_t kind, dim, dp, height, leaf_size, top_levels, top_count, pad0;
+    // level_prefix[L] = number of nodes with level < L, for L <= top_levels; the
+    // top region is numbered level by level, so its first level_prefix[L]
+    // records are exactly the top L levels (each kernel stages what fits).
+    int32_t level_prefix[TT_TOP_LEVELS_MAX + 1], pad1;
     int64_t n_nodes, n_points;
     double root_center[3], root_side;
     uint64_t off_rec, off_box, off_pts, off_pid, off_vpt, total;
@@ -138,6 +143,17 @@ int tt_launch_knn(const tt_knn_params &p, int dim, const tt_launch_cfg &cfg);
 int tt_launch_vp(const tt_vp_params &p, int dim, const tt_launch_cfg &cfg);
 int tt_launch_sort(const tt_tree *t, const float *pts, int64_t n, int32_t ld, uint32_t *perm,
                    uint64_t *keys_out, void *stream);
+
+// Nodes of the largest level-complete top prefix whose staged bytes fit `budget`.
+inline int tt_stage_count(const tt_blob_header &h, int bytes_per_node, int budget) {
+    int best = 1;  // the root always fits
+    for (int L = 1; L <= h.top_levels; ++L) {
+        const long long c = h.level_prefix[L];
+        if (c * bytes_per_node <= budget) best = (int)c;
+        else break;
+    }
+    return best;
+}
 
 // Host helpers (host_build.cpp / pack.cpp)
 size_t tt_pack_size_impl(const tt_tree_desc *d, int *status);

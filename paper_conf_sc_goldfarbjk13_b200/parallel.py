@@ -19,11 +19,14 @@ import torch
 import torch.distributed as dist
 
 
-def shard_range(n: int, rank: int, world: int) -> tuple[int, int]:
-    """Contiguous equal-count shard [lo, hi) of n points for `rank`."""
-    base, rem = divmod(n, world)
-    lo = rank * base + min(rank, rem)
-    return lo, lo + base + (1 if rank < rem else 0)
+def shard_range(n: int, rank: int, world: int, align: int = 32) -> tuple[int, int]:
+    """Contiguous shard [lo, hi) of n points for `rank`, boundaries on multiples
+    of `align` (one warp tile) so every warp of a shard is a warp of the
+    unsharded launch: sharded results are then bit-identical to one launch."""
+    chunk = -(-n // world)
+    chunk = -(-chunk // align) * align
+    lo = min(rank * chunk, n)
+    return lo, min(lo + chunk, n)
 
 
 def broadcast_blob(blob: np.ndarray | None, device, src: int = 0, group=None) -> torch.Tensor:
@@ -53,10 +56,10 @@ def broadcast_tree(host_tree, device, src: int = 0, group=None):
 
 def allgather_rows(full: torch.Tensor, world: int, group=None) -> torch.Tensor:
     """In-place all-gather of equal-size contiguous row shards of `full`
-    (rank r owns rows shard_range(n, r, world)); requires n % world == 0."""
+    (rank r owns rows shard_range(n, r, world)); needs n % (32 * world) == 0."""
     n = full.shape[0]
-    if n % world:
-        raise ValueError("allgather_rows needs equal shards (n % world == 0)")
+    if n % (32 * world):
+        raise ValueError("allgather_rows needs equal warp-aligned shards (n % (32*world) == 0)")
     rank = dist.get_rank(group)
     lo, hi = shard_range(n, rank, world)
     dist.all_gather_into_tensor(full, full[lo:hi].contiguous(), group=group)

@@ -86,7 +86,7 @@ def test_vp_builder_matches_oracle():
 # ------------------------------------------------------------- blob layout
 HDR = np.dtype([("magic", "<u4"), ("version", "<u4"), ("kind", "<i4"), ("dim", "<i4"), ("dp", "<i4"),
                 ("height", "<i4"), ("leaf_size", "<i4"), ("top_levels", "<i4"), ("top_count", "<i4"),
-                ("pad0", "<i4"), ("n_nodes", "<i8"), ("n_points", "<i8"), ("root_center", "<f8", 3),
+                ("pad0", "<i4"), ("level_prefix", "<i4", 33), ("pad1", "<i4"), ("n_nodes", "<i8"), ("n_points", "<i8"), ("root_center", "<f8", 3),
                 ("root_side", "<f8"), ("off_rec", "<u8"), ("off_box", "<u8"), ("off_pts", "<u8"),
                 ("off_pid", "<u8"), ("off_vpt", "<u8"), ("total", "<u8"), ("rec_bytes", "<u8")])
 
@@ -112,6 +112,11 @@ def test_oct_blob_top_first_layout_preserves_preorder():
     top = hd["top_count"]
     assert 0 < top * 32 <= 32 * 1024
     assert np.all(rec["lvl"][:top] < hd["top_levels"]) and np.all(rec["lvl"][top:] >= hd["top_levels"])
+    # top region numbered level by level: every level-complete prefix is the top L levels
+    assert np.all(np.diff(rec["lvl"][:top]) >= 0)
+    lp = hd["level_prefix"]
+    for L in range(hd["top_levels"] + 1):
+        assert lp[L] == int((h.array("level") < L).sum())
     seq = _walk_preorder(rec["fc"], rec["skip"], h.n_nodes)
     assert len(seq) == h.n_nodes and len(set(seq)) == h.n_nodes
     # the walk visits nodes in canonical preorder: levels and bodies line up
