@@ -145,11 +145,11 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
                     if (STATS) ++steps;
                     const int lvl = t.w;
                     const bool active = lvl <= wait;
-                    const float dx = __fsub_rn(g.x, b.x);
-                    const float dy = __fsub_rn(g.y, b.y);
+                    float dx, dy, sx, sy;
+                    sub2_rn(g.x, g.y, b.x, b.y, dx, dy);
+                    sqr2_rn(dx, dy, sx, sy);
                     const float dz = __fsub_rn(g.z, b.z);
-                    const float drsq =
-                        __fadd_rn(__fadd_rn(__fmul_rn(dx, dx), __fmul_rn(dy, dy)), __fmul_rn(dz, dz));
+                    const float drsq = __fadd_rn(__fadd_rn(sx, sy), __fmul_rn(dz, dz));
                     const bool near = drsq < dsq(lvl);
                     const bool open = active && t.x >= 0 && near;
                     if (STATS) visits += active;
@@ -171,11 +171,11 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
                     int4 t;
                     ld_rec(s_base, g_base, top, cur, g, t);
                     if (STATS) ++visits;
-                    const float dx = __fsub_rn(g.x, b.x);
-                    const float dy = __fsub_rn(g.y, b.y);
+                    float dx, dy, sx, sy;
+                    sub2_rn(g.x, g.y, b.x, b.y, dx, dy);
+                    sqr2_rn(dx, dy, sx, sy);
                     const float dz = __fsub_rn(g.z, b.z);
-                    const float drsq =
-                        __fadd_rn(__fadd_rn(__fmul_rn(dx, dx), __fmul_rn(dy, dy)), __fmul_rn(dz, dz));
+                    const float drsq = __fadd_rn(__fadd_rn(sx, sy), __fmul_rn(dz, dz));
                     const bool open = t.x >= 0 && drsq < dsq(t.w);
                     if (!open && t.z != self) acc.add(g.w, dx, dy, dz, drsq, eps2);
                     cur = open ? t.x : t.y;

@@ -91,31 +91,67 @@ __device__ __forceinline__ void cta_finish(uint32_t *ctr) {
 
 // ------------------------------------------------------ pinned fp32 arithmetic
 // DESIGN.md R0: t_d = rn(q_d - p_d), s = rn(t_0 t_0), s = rn(s + rn(t_d t_d)),
-// never contracted to FMA (explicit _rn intrinsics).
+// never contracted to FMA.  The independent per-dimension subtractions and
+// squares run two at a time on Blackwell's packed FP32x2 pipe (FADD2 / FMUL2:
+// sub.rn.f32x2 / mul.rn.f32x2, each lane rounded exactly like the scalar op);
+// the sum stays sequential in dimension order.
+__device__ __forceinline__ void sub2_rn(float a0, float a1, float b0, float b1, float &r0, float &r1) {
+    asm("{\n\t.reg .b64 x, y, z;\n\tmov.b64 x, {%2, %3};\n\tmov.b64 y, {%4, %5};\n\t"
+        "sub.rn.f32x2 z, x, y;\n\tmov.b64 {%0, %1}, z;\n\t}"
+        : "=f"(r0), "=f"(r1)
+        : "f"(a0), "f"(a1), "f"(b0), "f"(b1));
+}
+__device__ __forceinline__ void sqr2_rn(float a0, float a1, float &r0, float &r1) {
+    asm("{\n\t.reg .b64 x, z;\n\tmov.b64 x, {%2, %3};\n\t"
+        "mul.rn.f32x2 z, x, x;\n\tmov.b64 {%0, %1}, z;\n\t}"
+        : "=f"(r0), "=f"(r1)
+        : "f"(a0), "f"(a1));
+}
+
+// per-dimension squared differences rn(rn(q_d - p_d)^2) into sq[]
+template <int DIM>
+__device__ __forceinline__ void sq_diffs(const float (&q)[DIM], const float *p, float (&sq)[DIM]) {
+#pragma unroll
+    for (int d = 0; d + 1 < DIM; d += 2) {
+        float t0, t1;
+        sub2_rn(q[d], q[d + 1], p[d], p[d + 1], t0, t1);
+        sqr2_rn(t0, t1, sq[d], sq[d + 1]);
+    }
+    if (DIM & 1) {
+        const float t = __fsub_rn(q[DIM - 1], p[DIM - 1]);
+        sq[DIM - 1] = __fmul_rn(t, t);
+    }
+}
+
 template <int DIM>
 __device__ __forceinline__ float pinned_d2(const float (&q)[DIM], const float *p) {
-    float t = __fsub_rn(q[0], p[0]);
-    float s = __fmul_rn(t, t);
+    float sq[DIM];
+    sq_diffs<DIM>(q, p, sq);
+    float s = sq[0];
 #pragma unroll
-    for (int d = 1; d < DIM; ++d) {
-        float u = __fsub_rn(q[d], p[d]);
-        s = __fadd_rn(s, __fmul_rn(u, u));
-    }
+    for (int d = 1; d < DIM; ++d) s = __fadd_rn(s, sq[d]);
     return s;
 }
 
 // Box distance rn(max(lo - q, q - hi, 0))^2 summed in the same order.
 template <int DIM>
 __device__ __forceinline__ float pinned_boxd2(const float (&q)[DIM], const float *lo, const float *hi) {
-    float s = 0.0f;
+    float sq[DIM];
 #pragma unroll
-    for (int d = 0; d < DIM; ++d) {
-        float a = __fsub_rn(lo[d], q[d]);
-        float b = __fsub_rn(q[d], hi[d]);
-        float t = fmaxf(fmaxf(a, b), 0.0f);
-        float tt = __fmul_rn(t, t);
-        s = (d == 0) ? tt : __fadd_rn(s, tt);
+    for (int d = 0; d + 1 < DIM; d += 2) {
+        float a0, a1, b0, b1;
+        sub2_rn(lo[d], lo[d + 1], q[d], q[d + 1], a0, a1);
+        sub2_rn(q[d], q[d + 1], hi[d], hi[d + 1], b0, b1);
+        sqr2_rn(fmaxf(fmaxf(a0, b0), 0.0f), fmaxf(fmaxf(a1, b1), 0.0f), sq[d], sq[d + 1]);
     }
+    if (DIM & 1) {
+        const int d = DIM - 1;
+        const float t = fmaxf(fmaxf(__fsub_rn(lo[d], q[d]), __fsub_rn(q[d], hi[d])), 0.0f);
+        sq[d] = __fmul_rn(t, t);
+    }
+    float s = sq[0];
+#pragma unroll
+    for (int d = 1; d < DIM; ++d) s = __fadd_rn(s, sq[d]);
     return s;
 }
 
@@ -190,6 +226,12 @@ __device__ __forceinline__ float rsqrt_ftz(float x) {
     float y;
     asm("rsqrt.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
     return y;
+}
+
+// L1 prefetch of a global line (the next nodes of a walk are known one step
+// ahead: both children are in the current record).
+__device__ __forceinline__ void prefetch_l1(const void *p) {
+    asm volatile("prefetch.global.L1 [%0];" ::"l"(p));
 }
 
 // ------------------------------------------------------- warp-level helpers

@@ -83,10 +83,24 @@ __device__ __forceinline__ void ld_rec(const unsigned char *s_rec, const tt_kd_r
     }
 }
 
+// Bring both children's box row and record towards L1 (one is the next node).
+template <int DP>
+__device__ __forceinline__ void prefetch_children(int4 t, int top, const tt_kd_rec *g_rec, const float *g_box) {
+    if (t.x >= top) {
+        prefetch_l1(g_rec + t.x);
+        prefetch_l1(g_box + (size_t)t.x * 2 * DP);
+    }
+    if (t.y >= top) {
+        prefetch_l1(g_rec + t.y);
+        prefetch_l1(g_box + (size_t)t.y * 2 * DP);
+    }
+}
+
 // update_closest: every bucket point that beats the k-th best enters the list.
 template <int DIM, int KT>
 __device__ __forceinline__ void leaf_update(const tt_knn_params &P, int pb, int pc, int dp, const float (&q)[DIM],
                                             KBest<KT> &kb) {
+#pragma unroll 2
     for (int j = pb; j < pb + pc; ++j) {
         float p[DIM];
         load_row_nc<DIM>(p, P.c.tree.pts + (size_t)j * dp);
@@ -172,6 +186,7 @@ __global__ void __launch_bounds__(kBlock) knn_kernel(const tt_knn_params P, int 
                     if (t.x < 0) {
                         leaf_update<DIM, KT>(P, u.z, u.w, DP, q, kb);
                     } else {
+                        prefetch_children<DP>(t, top, g_rec, g_box);
                         const bool left_near = select_dim<DIM>(q, u.y) < __int_as_float(u.x);
                         w_stk[sp * 32 + lane] = left_near ? t.y : t.x;  // push far
                         ++sp;

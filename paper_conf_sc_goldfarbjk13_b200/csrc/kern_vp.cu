@@ -29,8 +29,9 @@ constexpr int kWarps = kBlock / 32;
 constexpr int kSmemHdr = 128;
 #define TT_VP_EPS 0x1p-12f
 
-__device__ __forceinline__ bool vp_prune(float lb, float sc, float best_d2) {
-    const float tau = __fsqrt_rn(best_d2);
+// tau = sqrt_rn(best d2) is kept in a register, recomputed only when the
+// best improves (same value as recomputing it at every pop).
+__device__ __forceinline__ bool vp_prune(float lb, float sc, float tau) {
     return __fsub_rn(lb, tau) > __fmul_rn(TT_VP_EPS, __fadd_rn(sc, tau));
 }
 
@@ -124,7 +125,7 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
             lock = warp_common_levels(code << (maxl - lv), vmask, 1, maxl) >= P.c.auto_min_depth;
         }
 
-        float best_d = POS_INF;
+        float best_d = POS_INF, tau = POS_INF;
         unsigned best_i = 0xffffffffu;
         unsigned visits = 0, fetches = 0, steps = 0;
         if (!lock) {
@@ -133,7 +134,7 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
             float lb = NEG_INF, sc = 0.f;
             while (cur != TT_END) {
                 if (STATS) ++visits;
-                if (!vp_prune(lb, sc, best_d)) {
+                if (!vp_prune(lb, sc, tau)) {
                     int4 t;
                     float v[DIM];
                     ld_node<DIM>(s_rec, s_vpt, g_rec, g_vpt, DP, top, cur, t, v);
@@ -143,6 +144,7 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
                         if (d2 < best_d || id < best_i) {
                             best_d = d2;
                             best_i = id;
+                            tau = __fsqrt_rn(d2);
                         }
                     }
                     const float d = __fsqrt_rn(d2);
@@ -182,7 +184,7 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
                     ++steps;
                     visits += in;
                 }
-                const bool active = in && !vp_prune(lb, sc, best_d);
+                const bool active = in && !vp_prune(lb, sc, tau);
                 const unsigned act = __ballot_sync(TT_FULL, active);
                 if (act) {
                     if (STATS) ++fetches;
@@ -198,6 +200,7 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
                             if (d2 < best_d || id < best_i) {
                                 best_d = d2;
                                 best_i = id;
+                                tau = __fsqrt_rn(d2);
                             }
                         }
                         d = __fsqrt_rn(d2);
