@@ -181,11 +181,13 @@ def count_kernels(step_fn) -> int | None:
         return None
 
 
-def load_traffic(kernel: str):
-    """dram bytes per launch from the committed ncu --set full summary, if any."""
-    path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+def load_counts(workload: str, mode: str):
+    """Per-point DRAM bytes and executed warp instructions of the traversal
+    kernel from the committed `ncu --set full` capture (profiles/ncu_counts.json,
+    written by tools/make_profiles.py), if any."""
+    path = os.path.join(ROOT, "profiles", "ncu_counts.json")
     try:
-        return json.load(open(path)).get(kernel)
+        return json.load(open(path)).get(f"{workload}/{mode}")
     except (OSError, ValueError):
         return None
 
@@ -204,7 +206,7 @@ def oracle_baseline(name, w, budget_points=None):
     c = w["cfg"]
     q = w["queries"]
     m = len(q)
-    frac = {"bh": 8, "knn": 8, "vp": 512, "pc": 1}[name]
+    frac = {"bh": 2, "knn": 8, "vp": 512, "pc": 1}[name]  # ~10-30 s of CPU work per sample
     idx = np.arange(0, m, frac)
     if budget_points:
         idx = idx[:budget_points]
@@ -452,8 +454,22 @@ def run_ours(args, rank, world, local_rank):
     alg_bytes = visits * bpv + m * BYTES_PER_POINT_IO[name]  # per launch on rank 0
     achieved = alg_bytes / (kms / 1e3) / 1e9
     kernel_name = {"bh": "bh_kernel", "pc": "pc_kernel", "knn": "knn_kernel", "vp": "vp_kernel"}[name]
+    cnt = load_counts(name, args.mode) if not args.unsorted else None
+    clocks = clk.summary()
+    sm_mhz = clocks.get("sm_mhz") or float(peaks.get("sm_max_mhz", 1965.0))
+    nsm = torch.cuda.get_device_properties(device).multi_processor_count
+    issue = None
+    if cnt:
+        inst = cnt["warp_inst_per_point"] * m
+        issue_peak = nsm * 4 * sm_mhz * 1e6 / 1e9  # warp instructions / ns -> G/s
+        issue = {"bound": "issue", "achieved": round(inst / (kms / 1e3) / 1e9, 1), "peak": round(issue_peak, 1),
+                 "unit": "Gwarp-inst/s", "frac": round(inst / (kms / 1e3) / 1e9 / issue_peak, 4),
+                 "inst_per_launch": int(inst), "source": f"ncu smsp__inst_executed ({cnt['round']}) x live time",
+                 "peak_def": f"{nsm} SMs x 4 schedulers x 1 warp-inst/clk x {sm_mhz:.0f} MHz"}
     roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": hbm, "unit": "GB/s",
-                "frac": round(achieved / hbm, 4), "traffic": load_traffic(kernel_name),
+                "frac": round(achieved / hbm, 4),
+                "traffic": int(cnt["dram_bytes_per_point"] * m) if cnt else None,
+                "issue": issue,
                 "peak_source": peak_src, "kernel": kernel_name, "kernel_ms": round(kms, 4),
                 "kernel_share_of_step": round(kms / ms, 4) if world == 1 else None,
                 "alg_bytes_per_launch": int(alg_bytes),
@@ -483,7 +499,7 @@ def run_ours(args, rank, world, local_rank):
         "traverse_ms": kms, "upload_ms": upload_ms, "host_build_ms": build_ms,
         "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": (launches or 0) * args.steps,
         "gpu_launches_per_step": launches,
-        "clocks": clk.summary(),
+        "clocks": clocks,
     }
     print(json.dumps(line), flush=True)
 

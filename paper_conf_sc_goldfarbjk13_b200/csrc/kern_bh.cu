@@ -67,6 +67,17 @@ struct Acc {
     }
 };
 
+constexpr int kBPL = 1;  // bodies per lane (2 measured: no gain, 64 regs -> 32 warps/SM)
+
+struct Body {
+    float4 b;
+    long long pid;
+    int self, wait;
+    unsigned visits;
+    bool valid;
+    Acc acc;
+};
+
 // 63-bit octant path of a body through the root cube (fp64 comparisons, R8a).
 __device__ __forceinline__ unsigned long long oct_path(float4 b, const double c0[3], double side, int levels) {
     double c[3] = {c0[0], c0[1], c0[2]};
@@ -106,7 +117,6 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
 
     const int lane = threadIdx.x & 31;
     const long long n = P.c.n;
-    const long long ntiles = (n + 31) >> 5;
     const float eps2 = P.eps2;
     const unsigned char *s_base = reinterpret_cast<const unsigned char *>(s_top);
     const unsigned char *g_base = reinterpret_cast<const unsigned char *>(g_rec);
@@ -114,27 +124,48 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
     const bool inf_root = !(P.dsq_root < __int_as_float(0x7f800000));
     auto dsq = [&](int lvl) { return EXP_DSQ ? dsq_at(dsq_bits, inf_root, lvl) : s_dsq[lvl]; };
 
+    // A warp tile is kBPL*32 consecutive points of the (sorted) order: lane l
+    // owns points tile*64 + l and tile*64 + 32 + l.  In lockstep the warp walks
+    // the union of all 64 traversals; the per-node fetch / vote / loop cost is
+    // shared by two bodies per lane.
+    const long long ntiles = (n + 32 * kBPL - 1) / (32 * kBPL);
     for (;;) {
         const long long tile = next_tile(P.c.counter);
         if (tile >= ntiles) break;
-        const long long pos = tile * 32 + lane;
-        const bool valid = pos < n;
-        const long long pid = valid ? (P.c.order ? (long long)P.c.order[pos] : pos) : 0;
-        const float4 b = valid ? __ldg(P.bodies + pid) : make_float4(0.f, 0.f, 0.f, 0.f);
-        const int self = valid ? (P.self_ids ? __ldg(P.self_ids + pid) : (int)pid) : -2;
-        const unsigned vmask = __ballot_sync(TT_FULL, valid);
+        Body bd[kBPL];
+#pragma unroll
+        for (int j = 0; j < kBPL; ++j) {
+            const long long pos = tile * 32 * kBPL + 32 * j + lane;
+            bd[j].valid = pos < n;
+            bd[j].pid = bd[j].valid ? (P.c.order ? (long long)P.c.order[pos] : pos) : 0;
+            bd[j].b = bd[j].valid ? __ldg(P.bodies + bd[j].pid) : make_float4(0.f, 0.f, 0.f, 0.f);
+            bd[j].self = bd[j].valid ? (P.self_ids ? __ldg(P.self_ids + bd[j].pid) : (int)bd[j].pid) : -2;
+            bd[j].wait = bd[j].valid ? INT_MAX : -1;
+            bd[j].visits = 0;
+        }
 
         bool lock = P.c.mode != TT_MODE_INDEPENDENT;
         if (P.c.mode == TT_MODE_AUTO && P.c.auto_min_depth > 0) {
             const int lv = min(P.c.auto_min_depth, 21);
-            unsigned long long code = oct_path(b, P.c.root_center, P.c.root_side, lv);
-            lock = warp_common_levels(code, vmask, 3, lv) >= P.c.auto_min_depth;
+            // common octant-path prefix over all kBPL*32 bodies of the tile
+            const unsigned long long c0 = oct_path(bd[0].b, P.c.root_center, P.c.root_side, lv);
+            const int leader = __ffs(__ballot_sync(TT_FULL, bd[0].valid)) - 1;
+            const unsigned long long lead = __shfl_sync(TT_FULL, c0, leader);
+            unsigned long long acc_or = 0;
+#pragma unroll
+            for (int j = 0; j < kBPL; ++j) {
+                const unsigned long long cj = j == 0 ? c0 : oct_path(bd[j].b, P.c.root_center, P.c.root_side, lv);
+                if (bd[j].valid) acc_or |= cj ^ lead;
+            }
+            const unsigned hi = __reduce_or_sync(TT_FULL, (unsigned)(acc_or >> 32));
+            const unsigned lo = __reduce_or_sync(TT_FULL, (unsigned)acc_or);
+            const unsigned long long x = ((unsigned long long)hi << 32) | lo;
+            const int common = x == 0 ? lv : (__clzll((long long)x) - (64 - 3 * lv)) / 3;
+            lock = common >= P.c.auto_min_depth;
         }
 
-        Acc acc;
-        unsigned visits = 0, fetches = 0, steps = 0;
+        unsigned fetches = 0, steps = 0;
         if (lock) {
-            int wait = valid ? INT_MAX : -1;
             int cur = 0;
             for (;;) {
 #pragma unroll 1
@@ -144,53 +175,71 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
                     ld_rec(s_base, g_base, top, cur, g, t);
                     if (STATS) ++steps;
                     const int lvl = t.w;
-                    const bool active = lvl <= wait;
-                    float dx, dy, sx, sy;
-                    sub2_rn(g.x, g.y, b.x, b.y, dx, dy);
-                    sqr2_rn(dx, dy, sx, sy);
-                    const float dz = __fsub_rn(g.z, b.z);
-                    const float drsq = __fadd_rn(__fadd_rn(sx, sy), __fmul_rn(dz, dz));
-                    const bool near = drsq < dsq(lvl);
-                    const bool open = active && t.x >= 0 && near;
-                    if (STATS) visits += active;
-                    wait = active ? (open ? INT_MAX : lvl) : wait;
-                    if (active && !open && t.z != self) acc.add(g.w, dx, dy, dz, drsq, eps2);
-                    cur = __any_sync(TT_FULL, open) ? t.x : t.y;
+                    const float dl = dsq(lvl);
+                    bool any_open = false;
+#pragma unroll
+                    for (int j = 0; j < kBPL; ++j) {
+                        const bool active = lvl <= bd[j].wait;
+                        float dx, dy, sx, sy;
+                        sub2_rn(g.x, g.y, bd[j].b.x, bd[j].b.y, dx, dy);
+                        sqr2_rn(dx, dy, sx, sy);
+                        const float dz = __fsub_rn(g.z, bd[j].b.z);
+                        const float drsq = __fadd_rn(__fadd_rn(sx, sy), __fmul_rn(dz, dz));
+                        const bool open = active && t.x >= 0 && drsq < dl;
+                        if (STATS) bd[j].visits += active;
+                        bd[j].wait = active ? (open ? INT_MAX : lvl) : bd[j].wait;
+                        if (active && !open && t.z != bd[j].self) bd[j].acc.add(g.w, dx, dy, dz, drsq, eps2);
+                        any_open |= open;
+                    }
+                    cur = __any_sync(TT_FULL, any_open) ? t.x : t.y;
                     if (cur == TT_END) break;
                 }
-                acc.flush();  // warp-uniform
+#pragma unroll
+                for (int j = 0; j < kBPL; ++j) bd[j].acc.flush();  // warp-uniform
                 if (cur == TT_END) break;
             }
             fetches = steps;
         } else {
-            int cur = valid ? 0 : TT_END;
-            while (cur != TT_END) {
+#pragma unroll
+            for (int j = 0; j < kBPL; ++j) {
+                int cur = bd[j].valid ? 0 : TT_END;
+                while (cur != TT_END) {
 #pragma unroll 1
-                for (int k = 0; k < kFlush; ++k) {
-                    float4 g;
-                    int4 t;
-                    ld_rec(s_base, g_base, top, cur, g, t);
-                    if (STATS) ++visits;
-                    float dx, dy, sx, sy;
-                    sub2_rn(g.x, g.y, b.x, b.y, dx, dy);
-                    sqr2_rn(dx, dy, sx, sy);
-                    const float dz = __fsub_rn(g.z, b.z);
-                    const float drsq = __fadd_rn(__fadd_rn(sx, sy), __fmul_rn(dz, dz));
-                    const bool open = t.x >= 0 && drsq < dsq(t.w);
-                    if (!open && t.z != self) acc.add(g.w, dx, dy, dz, drsq, eps2);
-                    cur = open ? t.x : t.y;
-                    if (cur == TT_END) break;
+                    for (int k = 0; k < kFlush; ++k) {
+                        float4 g;
+                        int4 t;
+                        ld_rec(s_base, g_base, top, cur, g, t);
+                        if (STATS) ++bd[j].visits;
+                        float dx, dy, sx, sy;
+                        sub2_rn(g.x, g.y, bd[j].b.x, bd[j].b.y, dx, dy);
+                        sqr2_rn(dx, dy, sx, sy);
+                        const float dz = __fsub_rn(g.z, bd[j].b.z);
+                        const float drsq = __fadd_rn(__fadd_rn(sx, sy), __fmul_rn(dz, dz));
+                        const bool open = t.x >= 0 && drsq < dsq(t.w);
+                        if (!open && t.z != bd[j].self) bd[j].acc.add(g.w, dx, dy, dz, drsq, eps2);
+                        cur = open ? t.x : t.y;
+                        if (cur == TT_END) break;
+                    }
+                    bd[j].acc.flush();
                 }
-                acc.flush();
             }
             if (STATS) {
-                fetches = warp_sum(visits);
-                steps = __reduce_max_sync(TT_FULL, visits);
+                unsigned v = 0, mx = 0;
+#pragma unroll
+                for (int j = 0; j < kBPL; ++j) {
+                    v += bd[j].visits;
+                    mx = max(mx, bd[j].visits);
+                }
+                fetches = warp_sum(v);
+                steps = __reduce_max_sync(TT_FULL, mx);
             }
         }
-        if (valid) {
-            P.acc[pid] = make_float4((float)acc.X, (float)acc.Y, (float)acc.Z, 0.f);
-            if (STATS && P.c.st_visits) P.c.st_visits[pid] = visits;
+#pragma unroll
+        for (int j = 0; j < kBPL; ++j) {
+            if (bd[j].valid) {
+                P.acc[bd[j].pid] = make_float4((float)bd[j].acc.X, (float)bd[j].acc.Y, (float)bd[j].acc.Z, 0.f);
+                if (STATS && P.c.st_visits) P.c.st_visits[bd[j].pid] = bd[j].visits;
+            }
         }
         if (STATS) write_warp_stats(P.c, tile, fetches, steps, lock);
     }
@@ -210,7 +259,7 @@ int launch(const tt_bh_params &p, const tt_launch_cfg &cfg) {
     if (e != cudaSuccess) return (int)e;
     if (cfg.ctas_per_sm > 0 && cfg.ctas_per_sm < occ) occ = cfg.ctas_per_sm;
     if (occ < 1) occ = 1;
-    const long long ntiles = (p.c.n + 31) / 32;
+    const long long ntiles = (p.c.n + 32 * kBPL - 1) / (32 * kBPL);
     long long grid = (long long)nsm * occ;
     const long long need = (ntiles + kBlock / 32 - 1) / (kBlock / 32);
     if (grid > need) grid = need;
