@@ -260,8 +260,9 @@ def run_ours(args, rank, world, local_rank):
     import paper_conf_sc_goldfarbjk13_b200 as P
     from paper_conf_sc_goldfarbjk13_b200 import parallel as PAR
 
-    torch.cuda.set_device(local_rank)
-    device = torch.device("cuda", local_rank)
+    gpu = local_rank % torch.cuda.device_count()  # test mode may put ranks on one GPU
+    torch.cuda.set_device(gpu)
+    device = torch.device("cuda", gpu)
     name = args.workload
     w = make_workload(name, world, args.points_per_rank)
     c = w["cfg"]
@@ -324,7 +325,7 @@ def run_ours(args, rank, world, local_rank):
     if args.unsorted:
         order_buf.copy_(torch.arange(m, dtype=torch.int32, device=device))
 
-    def step(kev=None):
+    def step(kev=None, collective=True):
         if not args.unsorted:
             P.tt_sort_points(tree, q_shard, out=order_buf)  # a1
         if kev:
@@ -332,11 +333,11 @@ def run_ours(args, rank, world, local_rank):
         traverse(q_shard, out_shard, order_buf)            # a2-a5
         if kev:
             kev[1].record(stream)
-        if world > 1:
+        if world > 1 and collective:
             for o in (out if isinstance(out, tuple) else (out,)):
                 PAR.allgather_rows(o, world)
 
-    clk = ClockSampler(local_rank).__enter__()
+    clk = ClockSampler(gpu).__enter__()
     # stats pass (untimed): per-point useful visits, warp fetches, modes
     if not args.unsorted:
         P.tt_sort_points(tree, q_shard, out=order_buf)
@@ -351,7 +352,8 @@ def run_ours(args, rank, world, local_rank):
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
-    launches = count_kernels(step) if rank == 0 else None
+    # our kernels per step (the NCCL all-gather of N > 1 is not ours: excluded)
+    launches = count_kernels(lambda: step(collective=False)) if rank == 0 else None
 
     flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.float32, device=device)
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
@@ -374,7 +376,7 @@ def run_ours(args, rank, world, local_rank):
     if world > 1:
         ms = PAR.max_over_ranks(ms, device)
         kms = PAR.max_over_ranks(kms, device)
-        visits_all = torch.tensor([visits], dtype=torch.int64, device=device)
+        visits_all = torch.tensor([visits], dtype=torch.int64, device=PAR._wire(device))
         dist.all_reduce(visits_all)
         visits_tot = int(visits_all.item())
     else:
@@ -519,8 +521,13 @@ def main():
     if world > 1:
         import torch
         import torch.distributed as dist
-        torch.cuda.set_device(local_rank)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        backend = os.environ.get("TT_DIST_BACKEND", "nccl")  # gloo: multi-rank flow test on one GPU
+        gpu = local_rank % torch.cuda.device_count()
+        torch.cuda.set_device(gpu)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", gpu))
+        else:
+            dist.init_process_group(backend)
     try:
         run_ours(args, rank, world, local_rank)
     finally:

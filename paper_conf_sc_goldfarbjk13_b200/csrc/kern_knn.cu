@@ -224,8 +224,10 @@ __global__ void __launch_bounds__(kBlock) knn_kernel(const tt_knn_params P, int 
                         const bool pref_left = active && select_dim<DIM>(q, u.y) < __int_as_float(u.x);
                         const int votes = __popc(__ballot_sync(TT_FULL, pref_left));
                         const bool left_first = 2 * votes >= __popc(act);
-                        w_node[sp] = left_first ? t.y : t.x;  // push second (all lanes write the same value)
-                        w_mask[sp] = act;
+                        if (lane == 0) {  // push second (warp-uniform entry)
+                            w_node[sp] = left_first ? t.y : t.x;
+                            w_mask[sp] = act;
+                        }
                         ++sp;
                         cur = left_first ? t.x : t.y;
                         mask = act;
@@ -234,8 +236,15 @@ __global__ void __launch_bounds__(kBlock) knn_kernel(const tt_knn_params P, int 
                 }
                 if (sp == 0) break;
                 --sp;
-                cur = w_node[sp];
-                mask = w_mask[sp];
+                // lane 0 owns the warp-uniform stack; its pop is broadcast
+                int e_node = 0;
+                unsigned e_mask = 0;
+                if (lane == 0) {
+                    e_node = w_node[sp];
+                    e_mask = w_mask[sp];
+                }
+                cur = __shfl_sync(TT_FULL, e_node, 0);
+                mask = __shfl_sync(TT_FULL, e_mask, 0);
             }
             fetches = steps;
         }

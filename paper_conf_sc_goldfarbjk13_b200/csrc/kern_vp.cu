@@ -210,8 +210,10 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
                     const int first_side = 2 * votes >= __popc(act) ? 0 : 1;
                     const int second = first_side ? t.x : t.y;
                     if (second != TT_END) {
-                        l_ent[sp] = (cur << 1) | (first_side ^ 1);  // all lanes write the same value
-                        l_mask[sp] = act;
+                        if (lane == 0) {  // warp-uniform part of the entry
+                            l_ent[sp] = (cur << 1) | (first_side ^ 1);
+                            l_mask[sp] = act;
+                        }
                         l_d[sp * 32 + lane] = d;
                         ++sp;
                     }
@@ -224,8 +226,15 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
                 }
                 if (sp == 0) break;
                 --sp;
-                const int e = l_ent[sp];
-                mask = l_mask[sp];
+                // lane 0 owns the warp-uniform part of the stack; broadcast its pop
+                int e0 = 0;
+                unsigned m0 = 0;
+                if (lane == 0) {
+                    e0 = l_ent[sp];
+                    m0 = l_mask[sp];
+                }
+                const int e = __shfl_sync(TT_FULL, e0, 0);
+                mask = __shfl_sync(TT_FULL, m0, 0);
                 cur = child_args(hdr(e >> 1), e & 1, l_d[sp * 32 + lane], lb, sc);
             }
         }

@@ -29,20 +29,28 @@ def shard_range(n: int, rank: int, world: int, align: int = 32) -> tuple[int, in
     return lo, min(lo + chunk, n)
 
 
+def _wire(device, group=None):
+    """Device the collectives run on: the tensors' own device under NCCL;
+    host memory under gloo (used to exercise the multi-rank flow without
+    NVLink, e.g. several ranks on one GPU in tests)."""
+    return torch.device("cpu") if dist.get_backend(group) == "gloo" else torch.device(device)
+
+
 def broadcast_blob(blob: np.ndarray | None, device, src: int = 0, group=None) -> torch.Tensor:
     """Broadcast a packed tree blob (uint8) from `src`; returns it on `device`
     on every rank.  The size travels first as an int64."""
     rank = dist.get_rank(group)
-    size = torch.zeros(1, dtype=torch.int64, device=device)
+    wire = _wire(device, group)
+    size = torch.zeros(1, dtype=torch.int64, device=wire)
     if rank == src:
         size[0] = int(blob.size)
     dist.broadcast(size, src, group=group)
     if rank == src:
-        buf = torch.from_numpy(np.ascontiguousarray(blob)).to(device)
+        buf = torch.from_numpy(np.ascontiguousarray(blob)).to(wire)
     else:
-        buf = torch.empty(int(size.item()), dtype=torch.uint8, device=device)
+        buf = torch.empty(int(size.item()), dtype=torch.uint8, device=wire)
     dist.broadcast(buf, src, group=group)
-    return buf
+    return buf.to(device)
 
 
 def broadcast_tree(host_tree, device, src: int = 0, group=None):
@@ -62,11 +70,17 @@ def allgather_rows(full: torch.Tensor, world: int, group=None) -> torch.Tensor:
         raise ValueError("allgather_rows needs equal warp-aligned shards (n % (32*world) == 0)")
     rank = dist.get_rank(group)
     lo, hi = shard_range(n, rank, world)
-    dist.all_gather_into_tensor(full, full[lo:hi].contiguous(), group=group)
+    wire = _wire(full.device, group)
+    if wire == full.device:
+        dist.all_gather_into_tensor(full, full[lo:hi], group=group)  # in place
+    else:
+        staged = full.to(wire)
+        dist.all_gather_into_tensor(staged, staged[lo:hi].clone(), group=group)
+        full.copy_(staged)
     return full
 
 
 def max_over_ranks(x: float, device, group=None) -> float:
-    t = torch.tensor([x], dtype=torch.float64, device=device)
+    t = torch.tensor([x], dtype=torch.float64, device=_wire(device, group))
     dist.all_reduce(t, op=dist.ReduceOp.MAX, group=group)
     return float(t.item())
