@@ -186,9 +186,10 @@ typedef struct tt_stats {
 typedef struct tt_traverse_opts {
     int32_t mode;            /* tt_mode                                          */
     int32_t auto_min_depth;  /* AUTO: lockstep iff the warp's points share a tree
-                                path of at least this many levels; -1 = kernel
-                                default (BH, PC: 0 = always lockstep, P:L2235-2236;
-                                kNN: never; VP: tuned)            */
+                                path of at least this many levels (0 = always,
+                                >= 64 = never); -1 = kernel default, measured on
+                                B200: BH 6, kNN 4, VP 4, PC never
+                                (10k-point PC is latency-bound: independent wins) */
     const uint32_t *order;   /* [n] device, nullable: lane j of the launch processes
                                 point order[j] (e.g. perm from tt_sort_points);
                                 results still go to the point's own slot        */
