@@ -49,7 +49,9 @@ def parse():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--workload", choices=["bh", "knn", "vp", "pc"], default="bh")
+    ap.add_argument("--workload", choices=["bh", "knn", "vp", "pc", "bh16m", "knn16m"], default="bh",
+                    help="bh/knn/vp/pc: configs[0..3] (weak scaling, M points per rank); "
+                         "bh16m/knn16m: configs[4] (16M points split over the ranks, strong scaling)")
     ap.add_argument("--mode", default="auto", choices=["auto", "lockstep", "independent"])
     ap.add_argument("--unsorted", action="store_true", help="skip tt_sort_points (paper's 'unsorted' column)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -62,6 +64,18 @@ def parse():
 # ------------------------------------------------------------------ inputs
 def make_workload(name: str, world: int, per_rank: int = 0):
     """Global synthetic inputs (identical on every rank: seeded)."""
+    if name == "bh16m":
+        c = dict(ttgen.CONFIGS["bh_16m_plummer"])
+        n = per_rank * world if per_rank else c["n"]
+        data = ttgen.plummer(n, c["seed"])
+        return dict(cfg=c, workload="bh_16m_plummer", data=data, queries=data, m=n // world, n_data=n,
+                    strong=True)
+    if name == "knn16m":
+        c = dict(ttgen.CONFIGS["knn_16m_7d"])
+        n = per_rank * world if per_rank else c["m"]
+        data = ttgen.gaussian_mixture(c["n"], c["dim"], c["seed"])
+        q = ttgen.gaussian_mixture(n, c["dim"], c["qseed"])
+        return dict(cfg=c, workload="knn_16m_7d", data=data, queries=q, m=n // world, n_data=c["n"], strong=True)
     if name == "bh":
         c = dict(ttgen.CONFIGS["bh_1m_plummer"])
         m = per_rank or c["n"]
@@ -206,7 +220,9 @@ def oracle_baseline(name, w, budget_points=None):
     c = w["cfg"]
     q = w["queries"]
     m = len(q)
-    frac = {"bh": 2, "knn": 8, "vp": 512, "pc": 1}[name]  # ~10-30 s of CPU work per sample
+    # sample sized for ~10-30 s of CPU work: every frac-th query
+    target = {"bh": 500_000, "knn": 125_000, "vp": 2_000, "pc": 10_000}[name]
+    frac = max(1, m // target)
     idx = np.arange(0, m, frac)
     if budget_points:
         idx = idx[:budget_points]
@@ -238,9 +254,10 @@ def run_reference(args, rank, world):
     if rank != 0:
         return
     w = make_workload(args.workload, 1, args.points_per_rank)
+    name = {"bh16m": "bh", "knn16m": "knn"}.get(args.workload, args.workload)
     vals = []
     for _ in range(max(1, min(args.steps, 3))):
-        vals.append(oracle_baseline(args.workload, w))
+        vals.append(oracle_baseline(name, w))
     v = statistics.median(x["value"] for x in vals)
     cb = dict(vals[0])
     cb["value"] = v
@@ -263,12 +280,12 @@ def run_ours(args, rank, world, local_rank):
     gpu = local_rank % torch.cuda.device_count()  # test mode may put ranks on one GPU
     torch.cuda.set_device(gpu)
     device = torch.device("cuda", gpu)
-    name = args.workload
-    w = make_workload(name, world, args.points_per_rank)
+    w = make_workload(args.workload, world, args.points_per_rank)
+    name = {"bh16m": "bh", "knn16m": "knn"}.get(args.workload, args.workload)
     c = w["cfg"]
     m = w["m"]
     lo, hi = PAR.shard_range(len(w["queries"]), rank, world)
-    assert hi - lo == m
+    m = hi - lo  # warp-aligned shard (strong-scaling workloads: the last may be shorter)
 
     # a0: tree (rank 0 builds; NCCL broadcast for N > 1) -- timed separately
     t0 = time.perf_counter()
@@ -438,7 +455,7 @@ def run_ours(args, rank, world, local_rank):
         if world > 1:
             ems = PAR.max_over_ranks(ems, device)
         d2h = sum(r.numel() * r.element_size() for r in (res_host if isinstance(res_host, tuple) else (res_host,)))
-        e2e = {"value": m * world / (ems / 1e3), "unit": "points/s", "ms_per_step": ems,
+        e2e = {"value": n_all / (ems / 1e3), "unit": "points/s", "ms_per_step": ems,
                "h2d_bytes_per_step": int(q_host.numel() * q_host.element_size()), "d2h_bytes_per_step": int(d2h),
                "note": "public API (tt_sort_points + tt_traverse_*) on pinned host buffers; H2D, D2H inside"}
 
@@ -483,10 +500,11 @@ def run_ours(args, rank, world, local_rank):
             cpu = oracle_baseline(name, w)
         except Exception as e:  # noqa: BLE001
             cpu = {"value": None, "error": repr(e)}
-    value = m * world / (ms / 1e3)
+    value = n_all / (ms / 1e3)  # all points of all ranks per second
     line = {
         "metric": METRIC, "value": value, "unit": "points/s", "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+        "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+        "scaling": "strong" if w.get("strong") else "weak",
         "vs_baseline": None, "dtype": "f32", "data": "synthetic",
         "config": {"workload": w["workload"], "points_per_rank": m, "global_points": n_all,
                    "tree_points": w["n_data"], "mode": args.mode, "sorted": not args.unsorted,

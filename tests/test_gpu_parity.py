@@ -343,3 +343,22 @@ def test_blob_roundtrip_device_adoption():
     a1 = P.tt_traverse_bh(t1, bd, 0.5, 0.05).cpu().numpy()
     a2 = P.tt_traverse_bh(t2, bd, 0.5, 0.05).cpu().numpy()
     assert np.array_equal(a1, a2)
+
+
+@pytest.mark.slow
+def test_bh_config5_16m_sampled():
+    """configs[4]: 16,777,216-body Plummer sphere (the multi-GPU config) on one
+    GPU, sampled bodies against the oracle."""
+    c = ttgen.CONFIGS["bh_16m_plummer"]
+    b = ttgen.plummer(c["n"], c["seed"])
+    tree = P.tt_tree_upload(P.build_oct(b))
+    bd = dev(b)
+    perm = P.tt_sort_points(tree, bd)
+    acc = P.tt_traverse_bh(tree, bd, c["theta"], c["eps"], order=perm).cpu().numpy()
+    ot = oracle.build_oct(b)
+    sample = np.concatenate([np.random.default_rng(3).choice(len(b), 4000, replace=False),
+                             np.argsort(np.linalg.norm(b[:, :3], axis=1))[:500]])
+    ref = oracle.bh(ot, b[sample], c["theta"], c["eps"], self_ids=sample)
+    err = rel_err(acc[sample], ref.out[0])
+    print(f"BH 16M sampled: max rel err {err.max():.3e}")
+    assert err.max() <= BH_TOL
