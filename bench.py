@@ -58,6 +58,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--points-per-rank", type=int, default=0, help="override M (testing)")
     ap.add_argument("--auto-min-depth", type=int, default=None, help="AUTO-mode threshold (default: kernel's)")
+    ap.add_argument("--variant", default="autoropes", choices=["autoropes", "recursive"],
+                    help="recursive = the paper's naive recursive GPU baseline (ablation, N mode)")
     return ap.parse_args()
 
 
@@ -328,16 +330,17 @@ def run_ours(args, rank, world, local_rank):
     def traverse(pts, res, order, stats=None):
         if name == "bh":
             P.tt_traverse_bh(tree, pts, c["theta"], c["eps"], out=res, self_ids=self_ids, order=order,
-                             mode=args.mode, auto_min_depth=args.auto_min_depth, stats=stats)
+                             mode=args.mode, auto_min_depth=args.auto_min_depth, stats=stats,
+                             variant=args.variant)
         elif name == "knn":
             P.tt_traverse_knn(tree, pts, c["k"], out_idx=res[0], out_d2=res[1], order=order, mode=args.mode,
-                              auto_min_depth=args.auto_min_depth, stats=stats)
+                              auto_min_depth=args.auto_min_depth, stats=stats, variant=args.variant)
         elif name == "vp":
             P.tt_traverse_vp(tree, pts, out_idx=res[0], out_d2=res[1], order=order, mode=args.mode,
-                             auto_min_depth=args.auto_min_depth, stats=stats)
+                             auto_min_depth=args.auto_min_depth, stats=stats, variant=args.variant)
         else:
             P.tt_traverse_pc(tree, pts, c["radius"], out=res, order=order, mode=args.mode,
-                             auto_min_depth=args.auto_min_depth, stats=stats)
+                             auto_min_depth=args.auto_min_depth, stats=stats, variant=args.variant)
 
     if args.unsorted:
         order_buf.copy_(torch.arange(m, dtype=torch.int32, device=device))
@@ -508,7 +511,7 @@ def run_ours(args, rank, world, local_rank):
         "vs_baseline": None, "dtype": "f32", "data": "synthetic",
         "config": {"workload": w["workload"], "points_per_rank": m, "global_points": n_all,
                    "tree_points": w["n_data"], "mode": args.mode, "sorted": not args.unsorted,
-                   "auto_min_depth": args.auto_min_depth,
+                   "auto_min_depth": args.auto_min_depth, "variant": args.variant,
                    "parallelism": f"dp{world} (points sharded, tree replicated)",
                    "l2": "flushed between timed steps (512 MiB write)",
                    "params": {k: v for k, v in c.items() if k not in ("kind",)}},

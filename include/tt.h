@@ -196,7 +196,17 @@ typedef struct tt_traverse_opts {
     const tt_stats *stats;   /* host struct of device pointers, nullable         */
     int32_t block_threads;   /* 0 = default (256)                               */
     int32_t ctas_per_sm;     /* 0 = occupancy maximum                            */
+    int32_t variant;         /* tt_variant: 0 = autoropes (the method);
+                                1 = naive recursive baseline (P:L1084-1090,
+                                independent mode only -- LOCKSTEP is
+                                TT_ERR_UNSUPPORTED; it fills stats->visits only,
+                                the warp_* arrays are left untouched)           */
 } tt_traverse_opts;
+
+typedef enum tt_variant {
+    TT_VARIANT_AUTOROPES = 0,
+    TT_VARIANT_RECURSIVE = 1
+} tt_variant;
 
 /* Barnes-Hut force pass (Fig.9): bodies float4 (x,y,z,m) rows;
  * self_ids[i] (nullable; default i) is the leaf body id whose interaction

@@ -18,6 +18,7 @@ STATUS = {0: "TT_OK", -1: "TT_ERR_INVALID_ARG", -2: "TT_ERR_CUDA", -3: "TT_ERR_O
 KIND_OCT, KIND_KD, KIND_VP = 1, 2, 3
 MODE = {"auto": 0, "lockstep": 1, "L": 1, "independent": 2, "N": 2}
 MEM_HOST, MEM_DEVICE = 0, 1
+VARIANT = {"autoropes": 0, "recursive": 1}
 MAX_HEIGHT, MAX_DIM, MAX_K = 48, 16, 32
 
 
@@ -61,7 +62,8 @@ class tt_stats(C.Structure):
 
 class tt_traverse_opts(C.Structure):
     _fields_ = [("mode", C.c_int32), ("auto_min_depth", C.c_int32), ("order", C.c_void_p),
-                ("stats", C.c_void_p), ("block_threads", C.c_int32), ("ctas_per_sm", C.c_int32)]
+                ("stats", C.c_void_p), ("block_threads", C.c_int32), ("ctas_per_sm", C.c_int32),
+                ("variant", C.c_int32)]
 
 
 # name -> (restype, argtypes); every function declared in include/tt.h

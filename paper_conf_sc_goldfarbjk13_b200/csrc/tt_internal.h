@@ -136,11 +136,17 @@ struct tt_launch_cfg {
     int block_threads;
     int ctas_per_sm;
     void *stream;
+    int variant;  // tt_variant
 };
 int tt_launch_bh(const tt_bh_params &p, const tt_launch_cfg &cfg);
 int tt_launch_pc(const tt_pc_params &p, int dim, const tt_launch_cfg &cfg);
 int tt_launch_knn(const tt_knn_params &p, int dim, const tt_launch_cfg &cfg);
 int tt_launch_vp(const tt_vp_params &p, int dim, const tt_launch_cfg &cfg);
+// naive recursive baseline (kern_recursive.cu)
+int tt_launch_bh_recursive(const tt_bh_params &p, const tt_launch_cfg &cfg);
+int tt_launch_pc_recursive(const tt_pc_params &p, int dim, const tt_launch_cfg &cfg);
+int tt_launch_knn_recursive(const tt_knn_params &p, int dim, const tt_launch_cfg &cfg);
+int tt_launch_vp_recursive(const tt_vp_params &p, int dim, const tt_launch_cfg &cfg);
 int tt_launch_sort(const tt_tree *t, const float *pts, int64_t n, int32_t ld, uint32_t *perm,
                    uint64_t *keys_out, void *stream);
 

@@ -222,8 +222,9 @@ def _lanes(order, n):
     return n if order is None else order.numel()
 
 
-def _opts(mode, auto_min_depth, order, stats, n):
+def _opts(mode, auto_min_depth, order, stats, n, variant="autoropes"):
     o = L.tt_traverse_opts()
+    o.variant = L.VARIANT[variant]
     o.mode = L.MODE[mode] if isinstance(mode, str) else int(mode)
     o.auto_min_depth = -1 if auto_min_depth is None else int(auto_min_depth)
     keep = []
@@ -258,7 +259,8 @@ def tt_sort_points(tree: Tree, pts: torch.Tensor, out: torch.Tensor | None = Non
 
 def tt_traverse_bh(tree: Tree, bodies: torch.Tensor, theta: float, eps: float, out: torch.Tensor | None = None,
                    self_ids: torch.Tensor | None = None, order: torch.Tensor | None = None, mode="auto",
-                   auto_min_depth: int | None = None, stats: Stats | None = None, stream=None) -> torch.Tensor:
+                   auto_min_depth: int | None = None, stats: Stats | None = None, stream=None,
+                   variant: str = "autoropes") -> torch.Tensor:
     _dev(bodies, torch.float32, "bodies", 4)
     if bodies.shape[1] != 4 or not bodies.is_contiguous():
         raise ValueError("bodies must be a contiguous (n, 4) float32 tensor")
@@ -269,7 +271,7 @@ def tt_traverse_bh(tree: Tree, bodies: torch.Tensor, theta: float, eps: float, o
     if self_ids is not None:
         _dev(self_ids, torch.int32, "self_ids")
         sp = self_ids.data_ptr()
-    o, keep = _opts(mode, auto_min_depth, order, stats, n)
+    o, keep = _opts(mode, auto_min_depth, order, stats, n, variant)
     check(L.load().tt_traverse_bh(tree._h, bodies.data_ptr(), sp, _lanes(order, n), float(theta), float(eps), out.data_ptr(),
                                   C.byref(o), C.c_void_p(_stream_handle(stream))), "tt_traverse_bh")
     del keep
@@ -278,12 +280,12 @@ def tt_traverse_bh(tree: Tree, bodies: torch.Tensor, theta: float, eps: float, o
 
 def tt_traverse_pc(tree: Tree, q: torch.Tensor, radius: float, out: torch.Tensor | None = None,
                    order: torch.Tensor | None = None, mode="auto", auto_min_depth: int | None = None,
-                   stats: Stats | None = None, stream=None) -> torch.Tensor:
+                   stats: Stats | None = None, stream=None, variant: str = "autoropes") -> torch.Tensor:
     _dev(q, torch.float32, "q", tree.dim)
     n = q.shape[0]
     if out is None:
         out = torch.empty(n, dtype=torch.int32, device=q.device)
-    o, keep = _opts(mode, auto_min_depth, order, stats, n)
+    o, keep = _opts(mode, auto_min_depth, order, stats, n, variant)
     check(L.load().tt_traverse_pc(tree._h, q.data_ptr(), _lanes(order, n), q.stride(0), float(radius), out.data_ptr(), C.byref(o),
                                   C.c_void_p(_stream_handle(stream))), "tt_traverse_pc")
     del keep
@@ -292,14 +294,15 @@ def tt_traverse_pc(tree: Tree, q: torch.Tensor, radius: float, out: torch.Tensor
 
 def tt_traverse_knn(tree: Tree, q: torch.Tensor, k: int, out_idx: torch.Tensor | None = None,
                     out_d2: torch.Tensor | None = None, order: torch.Tensor | None = None, mode="auto",
-                    auto_min_depth: int | None = None, stats: Stats | None = None, stream=None):
+                    auto_min_depth: int | None = None, stats: Stats | None = None, stream=None,
+                    variant: str = "autoropes"):
     _dev(q, torch.float32, "q", tree.dim)
     n = q.shape[0]
     if out_idx is None:
         out_idx = torch.empty((n, k), dtype=torch.int32, device=q.device)
     if out_d2 is None:
         out_d2 = torch.empty((n, k), dtype=torch.float32, device=q.device)
-    o, keep = _opts(mode, auto_min_depth, order, stats, n)
+    o, keep = _opts(mode, auto_min_depth, order, stats, n, variant)
     check(L.load().tt_traverse_knn(tree._h, q.data_ptr(), _lanes(order, n), q.stride(0), int(k), out_idx.data_ptr(),
                                    out_d2.data_ptr(), C.byref(o), C.c_void_p(_stream_handle(stream))),
           "tt_traverse_knn")
@@ -309,14 +312,15 @@ def tt_traverse_knn(tree: Tree, q: torch.Tensor, k: int, out_idx: torch.Tensor |
 
 def tt_traverse_vp(tree: Tree, q: torch.Tensor, out_idx: torch.Tensor | None = None,
                    out_d2: torch.Tensor | None = None, order: torch.Tensor | None = None, mode="auto",
-                   auto_min_depth: int | None = None, stats: Stats | None = None, stream=None):
+                   auto_min_depth: int | None = None, stats: Stats | None = None, stream=None,
+                   variant: str = "autoropes"):
     _dev(q, torch.float32, "q", tree.dim)
     n = q.shape[0]
     if out_idx is None:
         out_idx = torch.empty(n, dtype=torch.int32, device=q.device)
     if out_d2 is None:
         out_d2 = torch.empty(n, dtype=torch.float32, device=q.device)
-    o, keep = _opts(mode, auto_min_depth, order, stats, n)
+    o, keep = _opts(mode, auto_min_depth, order, stats, n, variant)
     check(L.load().tt_traverse_vp(tree._h, q.data_ptr(), _lanes(order, n), q.stride(0), out_idx.data_ptr(), out_d2.data_ptr(),
                                   C.byref(o), C.c_void_p(_stream_handle(stream))), "tt_traverse_vp")
     del keep

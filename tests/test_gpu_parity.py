@@ -362,3 +362,24 @@ def test_bh_config5_16m_sampled():
     err = rel_err(acc[sample], ref.out[0])
     print(f"BH 16M sampled: max rel err {err.max():.3e}")
     assert err.max() <= BH_TOL
+
+
+# ------------------------------------------------ recursive baseline (NEXT-2)
+def test_recursive_baseline_matches_oracle(bh_small, knn_small, vp_small, pc_setup):
+    """The naive recursive GPU baseline computes the same results
+    and visits the same nodes as the oracle -- it differs from the autoroped
+    kernels only in using device recursion."""
+    b, ot, ref, tree = bh_small
+    acc = P.tt_traverse_bh(tree, dev(b), 0.5, 0.05, mode="independent", variant="recursive").cpu().numpy()
+    assert rel_err(acc, ref.out[0]).max() <= BH_TOL
+    c, p, otp, refp, treep = pc_setup
+    cnt = P.tt_traverse_pc(treep, dev(p), c["radius"], mode="independent", variant="recursive")
+    assert np.array_equal(cnt.cpu().numpy().astype(np.uint32), refp.out[0])
+    p, q, otk, treek = knn_small
+    refk = oracle.knn(otk, q, 8)
+    idx, d2 = P.tt_traverse_knn(treek, dev(q), 8, mode="independent", variant="recursive")
+    assert np.array_equal(idx.cpu().numpy(), refk.out[0]) and np.array_equal(d2.cpu().numpy(), refk.out[1])
+    p, q, otv, treev = vp_small
+    refv = oracle.vp(otv, q, stats=True)
+    idx, d2 = P.tt_traverse_vp(treev, dev(q), mode="independent", variant="recursive")
+    assert np.array_equal(idx.cpu().numpy(), refv.out[0]) and np.array_equal(d2.cpu().numpy(), refv.out[1])
