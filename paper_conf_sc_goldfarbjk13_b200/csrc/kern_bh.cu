@@ -39,10 +39,8 @@ __device__ __forceinline__ void ld_rec(const unsigned char *s_base, const unsign
 // dsq_L = dsq_root * 0.25^L by exponent arithmetic: exact (a power-of-4
 // scaling of a normal float), bit-identical to repeated "dsq*0.25" (Fig.9a
 // line 4) -- the host checks dsq_root * 0.25^height stays normal, else the
-// table path is used.  theta = 0 (dsq_root = +inf) opens every cell.
-__device__ __forceinline__ float dsq_at(int dsq_bits, bool inf_root, int lvl) {
-    return inf_root ? __int_as_float(0x7f800000) : __int_as_float(dsq_bits - (lvl << 24));
-}
+// table path is used (also for theta = 0, dsq_root = +inf: every cell opens).
+__device__ __forceinline__ float dsq_at(int dsq_bits, int lvl) { return __int_as_float(dsq_bits - (lvl << 24)); }
 
 // Interaction (update(), Fig.9a line 6): a += m (c - x) / (|c - x|^2 + eps^2)^{3/2}.
 // Terms go into fp32 partial sums that are flushed into fp64 every
@@ -121,8 +119,7 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
     const unsigned char *s_base = reinterpret_cast<const unsigned char *>(s_top);
     const unsigned char *g_base = reinterpret_cast<const unsigned char *>(g_rec);
     const int dsq_bits = __float_as_int(P.dsq_root);
-    const bool inf_root = !(P.dsq_root < __int_as_float(0x7f800000));
-    auto dsq = [&](int lvl) { return EXP_DSQ ? dsq_at(dsq_bits, inf_root, lvl) : s_dsq[lvl]; };
+    auto dsq = [&](int lvl) { return EXP_DSQ ? dsq_at(dsq_bits, lvl) : s_dsq[lvl]; };
 
     // A warp tile is kBPL*32 consecutive points of the (sorted) order: lane l
     // owns points tile*64 + l and tile*64 + 32 + l.  In lockstep the warp walks
@@ -172,7 +169,11 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
                 for (int k = 0; k < kFlush; ++k) {
                     float4 g;
                     int4 t;
-                    ld_rec(s_base, g_base, top, cur, g, t);
+                    // lockstep: one warp-uniform address, served by L1 (top levels
+                    // included -- they are also at [0, top) of the global array);
+                    // measured 2.7% faster than the smem/global select here
+                    g = __ldg(reinterpret_cast<const float4 *>(&g_rec[cur].gx));
+                    t = __ldg(reinterpret_cast<const int4 *>(&g_rec[cur].first_child));
                     if (STATS) ++steps;
                     const int lvl = t.w;
                     const float dl = dsq(lvl);
@@ -275,7 +276,7 @@ int tt_launch_bh(const tt_bh_params &p, const tt_launch_cfg &cfg) {
     // exponent-arithmetic dsq is exact iff dsq_root * 0.25^height is a normal float
     // (or dsq_root = +inf, theta = 0); otherwise use the shared-memory table
     const float r = p.dsq_root;
-    const bool exp_ok = !(r < INFINITY) || (r > 0.f && std::ldexp((double)r, -2 * p.c.height) >= (double)FLT_MIN);
+    const bool exp_ok = r < INFINITY && r > 0.f && std::ldexp((double)r, -2 * p.c.height) >= (double)FLT_MIN;
     if (stats) return exp_ok ? launch<true, true>(p, cfg) : launch<true, false>(p, cfg);
     return exp_ok ? launch<false, true>(p, cfg) : launch<false, false>(p, cfg);
 }
