@@ -58,6 +58,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--points-per-rank", type=int, default=0, help="override M (testing)")
     ap.add_argument("--auto-min-depth", type=int, default=None, help="AUTO-mode threshold (default: kernel's)")
+    ap.add_argument("--device-build", action="store_true",
+                    help="BH: build the oct-tree on the GPU (tt_build_oct_device) instead of host build + upload")
     ap.add_argument("--variant", default="autoropes", choices=["autoropes", "recursive"],
                     help="recursive = the paper's naive recursive GPU baseline (ablation, N mode)")
     return ap.parse_args()
@@ -291,7 +293,15 @@ def run_ours(args, rank, world, local_rank):
 
     # a0: tree (rank 0 builds; NCCL broadcast for N > 1) -- timed separately
     t0 = time.perf_counter()
-    if world == 1:
+    if args.device_build and name == "bh":
+        # every rank builds the identical tree from the identical bodies (NEXT-1)
+        bodies_dev = torch.from_numpy(np.ascontiguousarray(w["data"])).to(device)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        tree = P.tt_build_oct_device(bodies_dev)
+        t1 = time.perf_counter()
+        del bodies_dev
+    elif world == 1:
         host = host_tree(P, name, w)
         t1 = time.perf_counter()
         tree = P.tt_tree_upload(host)
@@ -302,6 +312,7 @@ def run_ours(args, rank, world, local_rank):
     torch.cuda.synchronize()
     t2 = time.perf_counter()
     build_ms, upload_ms = 1e3 * (t1 - t0), 1e3 * (t2 - t1)
+    build_where = "device (tt_build_oct_device)" if (args.device_build and name == "bh") else "host (tt_build_*)"
 
     q_all = torch.from_numpy(np.ascontiguousarray(w["queries"])).to(device)
     q_shard = q_all[lo:hi]
@@ -519,7 +530,7 @@ def run_ours(args, rank, world, local_rank):
         "visits_per_point": visits / m,
         "lockstep_warp_fraction": lock_frac,
         "work_expansion_fetch_over_visits": (wf * 32.0 / visits) if visits else None,
-        "traverse_ms": kms, "upload_ms": upload_ms, "host_build_ms": build_ms,
+        "traverse_ms": kms, "upload_ms": upload_ms, "tree_build_ms": build_ms, "tree_build": build_where,
         "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": (launches or 0) * args.steps,
         "gpu_launches_per_step": launches,
         "clocks": clocks,

@@ -148,6 +148,15 @@ tt_status tt_tree_pack(const tt_tree_desc *d, void *host_blob, size_t bytes);
  * The call synchronises `s` before returning.                             */
 tt_status tt_tree_from_blob(const void *blob, size_t bytes, int32_t mem, tt_stream s, tt_tree **out);
 tt_status tt_tree_upload(const tt_tree_desc *d, tt_stream s, tt_tree **out);
+/* NEXT-1: build a Barnes-Hut oct-tree on the GPU from device bodies (n rows
+ * of x, y, z, mass; 16-B aligned) straight into the packed device layout --
+ * the same bytes tt_tree_pack produces for tt_build_oct of the same bodies
+ * (build rules R8a/R9).  Synchronises `s`.  Errors: TT_ERR_INVALID_ARG,
+ * TT_ERR_TREE_TOO_DEEP (never for R9 trees: height <= 33), TT_ERR_CUDA/OOM. */
+tt_status tt_build_oct_device(const float *bodies, int64_t n, tt_stream s, tt_tree **out);
+/* Copy the packed device blob back to host memory (bytes >= device_bytes of
+ * tt_tree_get_info); synchronous.  E.g. to checkpoint a tree.              */
+tt_status tt_tree_download(const tt_tree *t, void *host_blob, size_t bytes);
 tt_status tt_tree_free(tt_tree *t);
 
 typedef struct tt_tree_info {

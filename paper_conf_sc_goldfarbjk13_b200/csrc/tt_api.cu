@@ -85,6 +85,33 @@ tt_status setup_common(const tt_tree *t, int kind, int64_t n, const tt_traverse_
     return TT_OK;
 }
 
+// Wrap a device blob (already in device memory, owned) into a tree handle.
+tt_status adopt_blob(const tt_blob_header &h, void *d_blob, cudaStream_t cs, tt_tree **out) {
+    tt_tree *t = new (std::nothrow) tt_tree();
+    if (!t) return TT_ERR_OOM;
+    t->hdr = h;
+    t->bytes = (size_t)h.total;
+    t->d_blob = d_blob;
+    cudaError_t e = cudaMalloc((void **)&t->d_counters, sizeof(uint32_t) * 2 * TT_COUNTER_SLOTS);
+    if (e == cudaSuccess) e = cudaMemsetAsync(t->d_counters, 0, sizeof(uint32_t) * 2 * TT_COUNTER_SLOTS, cs);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
+    if (e != cudaSuccess) {
+        if (t->d_counters) cudaFree(t->d_counters);
+        delete t;
+        return cuda_fail(e);
+    }
+    auto *base = static_cast<unsigned char *>(t->d_blob);
+    t->dev.hdr_dev = reinterpret_cast<const tt_blob_header *>(base);
+    t->dev.rec = base + h.off_rec;
+    t->dev.box = h.off_box ? reinterpret_cast<const float *>(base + h.off_box) : nullptr;
+    t->dev.pts = h.off_pts ? reinterpret_cast<const float *>(base + h.off_pts) : nullptr;
+    t->dev.pid = h.off_pid ? reinterpret_cast<const int32_t *>(base + h.off_pid) : nullptr;
+    t->dev.vpt = h.off_vpt ? reinterpret_cast<const float *>(base + h.off_vpt) : nullptr;
+    t->slot_next = 0;
+    *out = t;
+    return TT_OK;
+}
+
 tt_status finish_launch(int err) {
     if (err == -1) return TT_ERR_UNSUPPORTED;
     if (err != 0) return cuda_fail((cudaError_t)err);
@@ -145,37 +172,41 @@ tt_status tt_tree_from_blob(const void *blob, size_t bytes, int32_t mem, tt_stre
     if (h.magic != TT_BLOB_MAGIC || h.version != TT_BLOB_VERSION || h.total > bytes || h.n_nodes <= 0 ||
         h.top_count < 1 || h.top_count > h.n_nodes)
         return TT_ERR_INVALID_ARG;
-    tt_tree *t = new (std::nothrow) tt_tree();
-    if (!t) return TT_ERR_OOM;
-    t->hdr = h;
-    t->bytes = (size_t)h.total;
-    e = cudaMalloc(&t->d_blob, t->bytes);
+    void *d_blob = nullptr;
+    e = cudaMalloc(&d_blob, (size_t)h.total);
+    if (e != cudaSuccess) return cuda_fail(e);
+    e = cudaMemcpyAsync(d_blob, blob, (size_t)h.total,
+                        mem == TT_MEM_HOST ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice, cs);
     if (e != cudaSuccess) {
-        delete t;
+        cudaFree(d_blob);
         return cuda_fail(e);
     }
-    e = cudaMalloc((void **)&t->d_counters, sizeof(uint32_t) * 2 * TT_COUNTER_SLOTS);
-    if (e == cudaSuccess) e = cudaMemsetAsync(t->d_counters, 0, sizeof(uint32_t) * 2 * TT_COUNTER_SLOTS, cs);
-    if (e == cudaSuccess)
-        e = cudaMemcpyAsync(t->d_blob, blob, t->bytes,
-                            mem == TT_MEM_HOST ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice, cs);
-    if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
-    if (e != cudaSuccess) {
-        cudaFree(t->d_blob);
-        if (t->d_counters) cudaFree(t->d_counters);
-        delete t;
-        return cuda_fail(e);
+    st = adopt_blob(h, d_blob, cs, out);
+    if (st != TT_OK) cudaFree(d_blob);
+    return st;
+}
+
+tt_status tt_build_oct_device(const float *bodies, int64_t n, tt_stream s, tt_tree **out) {
+    if (!bodies || !out || n <= 0 || n > INT32_MAX / 3 || !aligned(bodies, 16)) return TT_ERR_INVALID_ARG;
+    tt_status st = have_device();
+    if (st != TT_OK) return st;
+    tt_blob_header h;
+    void *d_blob = nullptr;
+    const int e = tt_build_oct_gpu_impl(bodies, n, s, &h, &d_blob);
+    if (e) return cuda_fail((cudaError_t)e);
+    if (h.height > TT_MAX_HEIGHT) {
+        cudaFree(d_blob);
+        return TT_ERR_TREE_TOO_DEEP;
     }
-    auto *base = static_cast<unsigned char *>(t->d_blob);
-    t->dev.hdr_dev = reinterpret_cast<const tt_blob_header *>(base);
-    t->dev.rec = base + h.off_rec;
-    t->dev.box = h.off_box ? reinterpret_cast<const float *>(base + h.off_box) : nullptr;
-    t->dev.pts = h.off_pts ? reinterpret_cast<const float *>(base + h.off_pts) : nullptr;
-    t->dev.pid = h.off_pid ? reinterpret_cast<const int32_t *>(base + h.off_pid) : nullptr;
-    t->dev.vpt = h.off_vpt ? reinterpret_cast<const float *>(base + h.off_vpt) : nullptr;
-    t->slot_next = 0;
-    *out = t;
-    return TT_OK;
+    st = adopt_blob(h, d_blob, (cudaStream_t)s, out);
+    if (st != TT_OK) cudaFree(d_blob);
+    return st;
+}
+
+tt_status tt_tree_download(const tt_tree *t, void *host_blob, size_t bytes) {
+    if (!t || !host_blob || bytes < t->bytes) return TT_ERR_INVALID_ARG;
+    const cudaError_t e = cudaMemcpy(host_blob, t->d_blob, t->bytes, cudaMemcpyDeviceToHost);
+    return e == cudaSuccess ? TT_OK : cuda_fail(e);
 }
 
 tt_status tt_tree_upload(const tt_tree_desc *d, tt_stream s, tt_tree **out) {

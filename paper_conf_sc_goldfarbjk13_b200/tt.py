@@ -23,6 +23,7 @@ from ._lib import TTError, check
 __all__ = [
     "HostTree", "Tree", "Stats", "TTError",
     "build_kd", "build_oct", "build_vp", "tt_tree_pack", "tt_tree_from_blob", "tt_tree_upload",
+    "tt_build_oct_device", "tt_tree_download",
     "tt_sort_points", "tt_traverse_bh", "tt_traverse_pc", "tt_traverse_knn", "tt_traverse_vp",
     "build_info",
 ]
@@ -187,6 +188,24 @@ def tt_tree_from_blob(blob, stream=None) -> Tree:
                                         C.byref(h))
     check(st, "tt_tree_from_blob")
     return Tree(h)
+
+
+def tt_build_oct_device(bodies: torch.Tensor, stream=None) -> Tree:
+    """NEXT-1: build the Barnes-Hut oct-tree on the GPU from (n, 4) device bodies."""
+    _dev(bodies, torch.float32, "bodies", 4)
+    if bodies.shape[1] != 4 or not bodies.is_contiguous():
+        raise ValueError("bodies must be a contiguous (n, 4) float32 tensor")
+    h = C.c_void_p()
+    check(L.load().tt_build_oct_device(bodies.data_ptr(), bodies.shape[0], C.c_void_p(_stream_handle(stream)),
+                                       C.byref(h)), "tt_build_oct_device")
+    return Tree(h)
+
+
+def tt_tree_download(tree: Tree) -> np.ndarray:
+    """The packed device blob, copied to a host uint8 array."""
+    out = np.empty(tree.device_bytes, dtype=np.uint8)
+    check(L.load().tt_tree_download(tree._h, _np_ptr(out), out.size), "tt_tree_download")
+    return out
 
 
 # ------------------------------------------------------------------ launches

@@ -383,3 +383,18 @@ def test_recursive_baseline_matches_oracle(bh_small, knn_small, vp_small, pc_set
     refv = oracle.vp(otv, q, stats=True)
     idx, d2 = P.tt_traverse_vp(treev, dev(q), mode="independent", variant="recursive")
     assert np.array_equal(idx.cpu().numpy(), refv.out[0]) and np.array_equal(d2.cpu().numpy(), refv.out[1])
+
+
+# ------------------------------------------------- GPU tree build (NEXT-1)
+@pytest.mark.parametrize("n,dups", [(1, False), (2, False), (3001, True), (20011, True), (1_000_000, False)])
+def test_gpu_oct_build_is_byte_identical_to_host_pack(n, dups):
+    """tt_build_oct_device emits exactly the blob tt_tree_pack makes from the
+    host builder (itself bit-identical to the oracle's builder)."""
+    b = ttgen.plummer(n, seed=217)
+    if dups and n > 20:
+        b[5, :3] = b[6, :3] = b[7, :3]  # depth-32 bucket
+    host_blob = P.build_oct(b).pack()
+    t = P.tt_build_oct_device(dev(b))
+    gpu_blob = P.tt_tree_download(t)
+    assert gpu_blob.size == host_blob.size
+    assert np.array_equal(gpu_blob, host_blob)
