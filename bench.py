@@ -49,9 +49,10 @@ def parse():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--workload", choices=["bh", "knn", "vp", "pc", "bh16m", "knn16m"], default="bh",
+    ap.add_argument("--workload", choices=["bh", "knn", "vp", "pc", "bh16m", "knn16m", "bhsteps"], default="bh",
                     help="bh/knn/vp/pc: configs[0..3] (weak scaling, M points per rank); "
-                         "bh16m/knn16m: configs[4] (16M points split over the ranks, strong scaling)")
+                         "bh16m/knn16m: configs[4] (16M points split over the ranks, strong scaling); "
+                         "bhsteps: full BH time steps (GPU build + sort + force + leapfrog), 1 GPU")
     ap.add_argument("--mode", default="auto", choices=["auto", "lockstep", "independent"])
     ap.add_argument("--unsorted", action="store_true", help="skip tt_sort_points (paper's 'unsorted' column)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -275,6 +276,41 @@ def run_reference(args, rank, world):
 
 
 # ------------------------------------------------------------------- ours
+def run_bh_steps(args):
+    """NEXT-4 workload: a bench step = one BH time step of configs[1] on one GPU
+    (tt_build_oct_device + tt_sort_points + tt_traverse_bh + tt_kick_drift)."""
+    import torch
+    from paper_conf_sc_goldfarbjk13_b200 import nbody
+    c = dict(ttgen.CONFIGS["bh_1m_plummer"])
+    n = args.points_per_rank or c["n"]
+    b = ttgen.plummer(n, c["seed"])
+    v = ttgen.plummer_velocities(b, c["seed"] + 1000)
+    B = torch.from_numpy(b).cuda()
+    V = torch.from_numpy(v).cuda()
+    dt = 1e-3
+    acc, _ = nbody.forces(B, c["theta"], c["eps"])
+    for _ in range(args.warmup):
+        acc = nbody.simulate(B, V, 1, dt, c["theta"], c["eps"], acc=acc)
+    torch.cuda.synchronize()
+    stream = torch.cuda.current_stream()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    with ClockSampler(0) as clk:
+        for i in range(args.steps):
+            evs[i][0].record(stream)
+            acc = nbody.simulate(B, V, 1, dt, c["theta"], c["eps"], acc=acc)
+            evs[i][1].record(stream)
+        torch.cuda.synchronize()
+    ms = statistics.mean(a.elapsed_time(b_) for a, b_ in evs)
+    line = {"metric": METRIC, "value": n / (ms / 1e3), "unit": "points/s (body-steps/s)", "n_gpus": 1,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": "bh_1m_plummer time steps", "bodies": n, "dt": dt,
+                       "step": "GPU build + sort + force + kick-drift (leapfrog KDK)", "params": c,
+                       "l2": "not flushed: a time step rewrites the bodies and rebuilds the tree"},
+            "clocks": clk.summary()}
+    print(json.dumps(line), flush=True)
+
+
 def run_ours(args, rank, world, local_rank):
     import torch
     import torch.distributed as dist
@@ -549,6 +585,10 @@ def main():
             sys.exit(2)
     if args.impl == "reference":
         run_reference(args, rank, world)
+        return
+    if args.workload == "bhsteps":
+        if rank == 0:
+            run_bh_steps(args)
         return
     if world > 1:
         import torch

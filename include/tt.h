@@ -245,6 +245,14 @@ tt_status tt_traverse_knn(const tt_tree *t, const float *q, int64_t n, int32_t l
 tt_status tt_traverse_vp(const tt_tree *t, const float *q, int64_t n, int32_t ld, int32_t *idx_out,
                          float *d2_out, const tt_traverse_opts *opts, tt_stream s);
 
+/* NEXT-4: one kick-drift update of a Barnes-Hut time step (leapfrog KDK is
+ * kick(dt/2)+drift(dt), rebuild + force pass, kick(dt/2)):
+ * v += acc * dt_kick; x += v * dt_drift.  bodies (x,y,z,m), vel (vx,vy,vz,-)
+ * and acc (ax,ay,az,-) are n float4 rows in device memory (16-B aligned);
+ * fp32 with one rounding per operation; asynchronous on `s`.              */
+tt_status tt_kick_drift(float *bodies, float *vel, const float *acc, int64_t n, float dt_kick, float dt_drift,
+                        tt_stream s);
+
 /* ------------------------------------------------------------------------ */
 const char *tt_status_string(tt_status s);
 /* Last CUDA error code seen by the library (cudaError_t as int), 0 if none. */

@@ -12,5 +12,7 @@ _lib.load()
 
 from . import tt  # noqa: E402
 from .tt import *  # noqa: E402,F401,F403
+from . import nbody  # noqa: E402
+from .nbody import tt_kick_drift  # noqa: E402,F401
 
-__all__ = ["tt", "TTError"] + list(tt.__all__)
+__all__ = ["tt", "nbody", "TTError", "tt_kick_drift"] + list(tt.__all__)

@@ -352,4 +352,16 @@ tt_status tt_traverse_vp(const tt_tree *t, const float *q, int64_t n, int32_t ld
                                                             : tt_launch_vp(p, t->hdr.dim, cfg));
 }
 
+tt_status tt_kick_drift(float *bodies, float *vel, const float *acc, int64_t n, float dt_kick, float dt_drift,
+                        tt_stream s) {
+    if (n < 0) return TT_ERR_INVALID_ARG;
+    if (n == 0) return TT_OK;
+    if (!bodies || !vel || !acc || !aligned(bodies, 16) || !aligned(vel, 16) || !aligned(acc, 16))
+        return TT_ERR_INVALID_ARG;
+    tt_status st = have_device();
+    if (st != TT_OK) return st;
+    const int e = tt_launch_kick_drift(bodies, vel, acc, n, dt_kick, dt_drift, s);
+    return e ? cuda_fail((cudaError_t)e) : TT_OK;
+}
+
 }  // extern "C"

@@ -165,6 +165,8 @@ inline int tt_stage_count(const tt_blob_header &h, int bytes_per_node, int budge
 // cudaMalloc'd device blob; returns a cudaError_t.
 int tt_build_oct_gpu_impl(const float *bodies, long long n, void *stream, tt_blob_header *hdr, void **blob);
 
+int tt_launch_kick_drift(float *x, float *v, const float *a, long long n, float dtk, float dtd, void *stream);
+
 // Host helpers (host_build.cpp / pack.cpp)
 size_t tt_pack_size_impl(const tt_tree_desc *d, int *status);
 int tt_pack_impl(const tt_tree_desc *d, void *blob, size_t bytes);

@@ -398,3 +398,59 @@ def test_gpu_oct_build_is_byte_identical_to_host_pack(n, dups):
     gpu_blob = P.tt_tree_download(t)
     assert gpu_blob.size == host_blob.size
     assert np.array_equal(gpu_blob, host_blob)
+
+
+# ------------------------------------------------ BH time stepping (NEXT-4)
+def test_kick_drift_is_the_fp32_update():
+    from paper_conf_sc_goldfarbjk13_b200 import tt_kick_drift
+    rng = np.random.default_rng(5)
+    x = rng.standard_normal((1000, 4)).astype(np.float32)
+    v = rng.standard_normal((1000, 4)).astype(np.float32)
+    a = rng.standard_normal((1000, 4)).astype(np.float32)
+    X, V, A = dev(x), dev(v), dev(a)
+    tt_kick_drift(X, V, A, 0.01, 0.02)
+    v1 = (v[:, :3] + (a[:, :3] * np.float32(0.01)).astype(np.float32)).astype(np.float32)
+    x1 = (x[:, :3] + (v1 * np.float32(0.02)).astype(np.float32)).astype(np.float32)
+    assert np.array_equal(V.cpu().numpy()[:, :3], v1) and np.array_equal(X.cpu().numpy()[:, :3], x1)
+    assert np.array_equal(X.cpu().numpy()[:, 3], x[:, 3])  # masses untouched
+
+
+def test_two_body_circular_orbit_is_kept():
+    """Physics pin of the whole time step (GPU build + sort + BH force + leapfrog):
+    two equal masses on a softened circular orbit keep their separation and
+    speed over a quarter orbit."""
+    from paper_conf_sc_goldfarbjk13_b200 import nbody
+    d, m, eps = 1.0, 0.5, 0.01
+    f = m * m * d / (d * d + eps * eps) ** 1.5          # softened pair force
+    vc = np.sqrt(f * (d / 2) / m)                         # m v^2 / (d/2) = f
+    b = np.array([[-d / 2, 0, 0, m], [d / 2, 0, 0, m]], np.float32)
+    v = np.array([[0, -vc, 0, 0], [0, vc, 0, 0]], np.float32)
+    period = 2 * np.pi * (d / 2) / vc
+    steps = 250
+    B, V = dev(b), dev(v)
+    nbody.simulate(B, V, steps, period / 4 / steps, theta=0.5, eps=eps)
+    bb, vv = B.cpu().numpy().astype(np.float64), V.cpu().numpy().astype(np.float64)
+    sep = np.linalg.norm(bb[1, :3] - bb[0, :3])
+    assert abs(sep - d) < 1e-4
+    assert np.allclose(np.linalg.norm(vv[:, :3], axis=1), vc, rtol=1e-4)
+    assert np.allclose(bb[0, :3] + bb[1, :3], 0, atol=1e-5)  # centre of mass stays put
+    # quarter orbit: bodies moved from the x axis to the y axis
+    assert abs(bb[1, 1] - d / 2) < 1e-3 and abs(bb[1, 0]) < 1e-3
+
+
+def test_plummer_steps_forces_match_oracle_each_step():
+    """Five time steps of a 20k Plummer sphere: after every step the GPU force
+    pass on the moved bodies matches the fp64 oracle on the same positions."""
+    from paper_conf_sc_goldfarbjk13_b200 import nbody
+    b = ttgen.plummer(20000, seed=218)
+    v = ttgen.plummer_velocities(b, seed=219)
+    B, V = dev(b), dev(v)
+    acc = None
+    for s in range(5):
+        acc = nbody.simulate(B, V, 1, 1e-3, theta=0.5, eps=0.05, acc=acc)
+        x = B.cpu().numpy()
+        ref = oracle.bh(oracle.build_oct(x), x, 0.5, 0.05, self_ids=np.arange(len(x))).out[0]
+        assert rel_err(acc.cpu().numpy(), ref).max() <= BH_TOL
+    p = (B.cpu().numpy()[:, 3:4].astype(np.float64) * V.cpu().numpy()[:, :3]).sum(0)
+    p0 = (b[:, 3:4].astype(np.float64) * v[:, :3]).sum(0)
+    assert np.abs(p - p0).max() < 1e-4

@@ -21,7 +21,7 @@ from __future__ import annotations
 
 import numpy as np
 
-__all__ = ["uniform", "plummer", "gaussian_mixture", "permutation", "CONFIGS"]
+__all__ = ["uniform", "plummer", "plummer_velocities", "gaussian_mixture", "permutation", "CONFIGS"]
 
 
 def uniform(n: int, dim: int, seed: int) -> np.ndarray:
@@ -50,6 +50,35 @@ def plummer(n: int, seed: int) -> np.ndarray:
     out[:, 1] = scale * r * sint * np.sin(phi)
     out[:, 2] = scale * r * cost
     out[:, 3] = 1.0 / max(n, 1)
+    return out.astype(np.float32)
+
+
+def plummer_velocities(bodies: np.ndarray, seed: int) -> np.ndarray:
+    """(n, 4) float32 rows (vx, vy, vz, 0) for `plummer` bodies: Aarseth,
+    Henon & Wielen (1974) von Neumann rejection for q = v / v_esc with
+    g(q) ~ q^2 (1 - q^2)^{7/2}, v_esc = sqrt(2) (1 + r^2)^{-1/4}, isotropic
+    direction, in the same standard units as the positions (velocities scaled
+    by sqrt(16 / (3 pi))).  Separate RNG stream: positions are unchanged."""
+    rng = np.random.default_rng(seed)
+    n = len(bodies)
+    pscale = 3.0 * np.pi / 16.0
+    r = np.linalg.norm(np.asarray(bodies, np.float64)[:, :3], axis=1) / pscale
+    q = np.empty(n)
+    todo = np.arange(n)
+    while len(todo):
+        x = rng.random(len(todo))
+        y = rng.random(len(todo)) * 0.1
+        ok = y < x * x * (1.0 - x * x) ** 3.5
+        q[todo[ok]] = x[ok]
+        todo = todo[~ok]
+    v = q * np.sqrt(2.0) * (1.0 + r * r) ** -0.25 * np.sqrt(16.0 / (3.0 * np.pi))
+    cost = rng.random(n) * 2.0 - 1.0
+    phi = rng.random(n) * (2.0 * np.pi)
+    sint = np.sqrt(np.maximum(0.0, 1.0 - cost * cost))
+    out = np.zeros((n, 4))
+    out[:, 0] = v * sint * np.cos(phi)
+    out[:, 1] = v * sint * np.sin(phi)
+    out[:, 2] = v * cost
     return out.astype(np.float32)
 
 
