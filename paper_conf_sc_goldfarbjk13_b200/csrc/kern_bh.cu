@@ -164,19 +164,23 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
         unsigned fetches = 0, steps = 0;
         if (lock) {
             int cur = 0;
+            // kernel parameters pinned in registers for the hot loop (otherwise
+            // re-read from the constant bank every iteration)
+            const tt_oct_rec *grec = g_rec;
+            int dbits = dsq_bits;
+            float e2 = eps2;
+            asm volatile("" : "+l"(grec), "+r"(dbits), "+f"(e2));
             for (;;) {
 #pragma unroll 1
                 for (int k = 0; k < kFlush; ++k) {
-                    float4 g;
-                    int4 t;
                     // lockstep: one warp-uniform address, served by L1 (top levels
                     // included -- they are also at [0, top) of the global array);
                     // measured 2.7% faster than the smem/global select here
-                    g = __ldg(reinterpret_cast<const float4 *>(&g_rec[cur].gx));
-                    t = __ldg(reinterpret_cast<const int4 *>(&g_rec[cur].first_child));
+                    const float4 g = __ldg(reinterpret_cast<const float4 *>(&grec[cur].gx));
+                    const int4 t = __ldg(reinterpret_cast<const int4 *>(&grec[cur].first_child));
                     if (STATS) ++steps;
                     const int lvl = t.w;
-                    const float dl = dsq(lvl);
+                    const float dl = EXP_DSQ ? dsq_at(dbits, lvl) : s_dsq[lvl];
                     bool any_open = false;
 #pragma unroll
                     for (int j = 0; j < kBPL; ++j) {
@@ -189,7 +193,14 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
                         const bool open = active && t.x >= 0 && drsq < dl;
                         if (STATS) bd[j].visits += active;
                         bd[j].wait = active ? (open ? INT_MAX : lvl) : bd[j].wait;
-                        if (active && !open && t.z != bd[j].self) bd[j].acc.add(g.w, dx, dy, dz, drsq, eps2);
+                        // branch-free update: in a warp step some lane almost always
+                        // interacts, so predication beats a divergent branch
+                        const bool inter = active && !open && t.z != bd[j].self;
+                        const float inv = rsqrt_ftz(__fadd_rn(drsq, e2));
+                        const float f = inter ? g.w * (inv * inv) * inv : 0.0f;
+                        bd[j].acc.x = fmaf(f, dx, bd[j].acc.x);
+                        bd[j].acc.y = fmaf(f, dy, bd[j].acc.y);
+                        bd[j].acc.z = fmaf(f, dz, bd[j].acc.z);
                         any_open |= open;
                     }
                     cur = __any_sync(TT_FULL, any_open) ? t.x : t.y;
@@ -217,7 +228,11 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
                         const float dz = __fsub_rn(g.z, bd[j].b.z);
                         const float drsq = __fadd_rn(__fadd_rn(sx, sy), __fmul_rn(dz, dz));
                         const bool open = t.x >= 0 && drsq < dsq(t.w);
-                        if (!open && t.z != bd[j].self) bd[j].acc.add(g.w, dx, dy, dz, drsq, eps2);
+                        const float inv = rsqrt_ftz(__fadd_rn(drsq, eps2));
+                        const float f = (!open && t.z != bd[j].self) ? g.w * (inv * inv) * inv : 0.0f;
+                        bd[j].acc.x = fmaf(f, dx, bd[j].acc.x);
+                        bd[j].acc.y = fmaf(f, dy, bd[j].acc.y);
+                        bd[j].acc.z = fmaf(f, dz, bd[j].acc.z);
                         cur = open ? t.x : t.y;
                         if (cur == TT_END) break;
                     }
