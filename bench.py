@@ -412,8 +412,9 @@ def run_ours(args, rank, world, local_rank):
     traverse(q_shard, out_shard, order_buf, st)
     torch.cuda.synchronize()
     visits = int(st.visits.to(torch.int64).sum().item())
-    wf = int(st.warp_fetches.to(torch.int64).sum().item())
-    lock_frac = float((st.warp_mode == 1).float().mean().item())
+    tiles = -(-m // P._lib.TILE_POINTS[tree.kind])
+    wf = int(st.warp_fetches[:tiles].to(torch.int64).sum().item())
+    lock_frac = float((st.warp_mode[:tiles] == 1).float().mean().item())
     del st
 
     for _ in range(args.warmup):
@@ -565,7 +566,10 @@ def run_ours(args, rank, world, local_rank):
         "node_visits_per_sec": visits_tot / (kms / 1e3),
         "visits_per_point": visits / m,
         "lockstep_warp_fraction": lock_frac,
-        "work_expansion_fetch_over_visits": (wf * 32.0 / visits) if visits else None,
+        # lane-slots offered by the warp fetches / useful visits (lockstep tiles)
+        "work_expansion_fetch_over_visits": (wf * P._lib.TILE_POINTS[tree.kind] / visits)
+        if visits and lock_frac > 0.99 else None,
+        "warp_tile_points": P._lib.TILE_POINTS[tree.kind],
         "traverse_ms": kms, "upload_ms": upload_ms, "tree_build_ms": build_ms, "tree_build": build_where,
         "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": (launches or 0) * args.steps,
         "gpu_launches_per_step": launches,

@@ -71,6 +71,9 @@ typedef void *tt_stream; /* cudaStream_t */
 #define TT_MAX_HEIGHT 48      /* rope-stack capacity bound (levels)            */
 #define TT_MAX_DIM 16         /* point dimensionality supported by the kernels */
 #define TT_MAX_K 32           /* kNN k supported by the kernels                */
+#define TT_BH_POINTS_PER_LANE 2 /* a BH warp tile holds 32*2 = 64 bodies (2 per
+                                   lane); its tt_stats warp_* entry covers 64
+                                   points (other kernels: 32 points, 1 per lane) */
 
 /* ------------------------------------------------------------------------ */
 /* Host-side tree construction (build rules: DESIGN.md R3, R8a, R9, R12).   */
@@ -186,10 +189,11 @@ tt_status tt_sort_points(const tt_tree *t, const float *pts, int64_t n, int32_t 
 typedef struct tt_stats {
     uint32_t *visits;        /* [n] per point: truncation tests it performed (the
                                 paper's per-point node count)      */
-    uint32_t *warp_fetches;  /* [ceil(n/32)] node records fetched by the warp
-                                (lockstep: one per step; independent: per lane) */
-    uint32_t *warp_steps;    /* [ceil(n/32)] loop iterations of the warp         */
-    uint8_t *warp_mode;      /* [ceil(n/32)] 1 = lockstep, 2 = independent      */
+    uint32_t *warp_fetches;  /* [ceil(n/T)] node records fetched by the warp tile
+                                (lockstep: one per step; independent: per lane);
+                                T = 32 points per tile (BH: 32*TT_BH_POINTS_PER_LANE) */
+    uint32_t *warp_steps;    /* [ceil(n/T)] loop iterations of the warp          */
+    uint8_t *warp_mode;      /* [ceil(n/T)] 1 = lockstep, 2 = independent       */
 } tt_stats;
 
 typedef struct tt_traverse_opts {

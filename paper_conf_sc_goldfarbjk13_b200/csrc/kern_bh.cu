@@ -65,7 +65,7 @@ struct Acc {
     }
 };
 
-constexpr int kBPL = 1;  // bodies per lane (2 measured: no gain, 64 regs -> 32 warps/SM)
+constexpr int kBPL = TT_BH_POINTS_PER_LANE;  // bodies per lane (2: -4% time vs 1)
 
 struct Body {
     float4 b;

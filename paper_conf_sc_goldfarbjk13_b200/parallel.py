@@ -19,10 +19,11 @@ import torch
 import torch.distributed as dist
 
 
-def shard_range(n: int, rank: int, world: int, align: int = 32) -> tuple[int, int]:
+def shard_range(n: int, rank: int, world: int, align: int = 64) -> tuple[int, int]:
     """Contiguous shard [lo, hi) of n points for `rank`, boundaries on multiples
-    of `align` (one warp tile) so every warp of a shard is a warp of the
-    unsharded launch: sharded results are then bit-identical to one launch."""
+    of `align` (a warp tile: 64 points for BH, 32 otherwise) so every warp of a
+    shard is a warp of the unsharded launch: sharded results are then
+    bit-identical to one launch."""
     chunk = -(-n // world)
     chunk = -(-chunk // align) * align
     lo = min(rank * chunk, n)
@@ -64,10 +65,10 @@ def broadcast_tree(host_tree, device, src: int = 0, group=None):
 
 def allgather_rows(full: torch.Tensor, world: int, group=None) -> torch.Tensor:
     """In-place all-gather of equal-size contiguous row shards of `full`
-    (rank r owns rows shard_range(n, r, world)); needs n % (32 * world) == 0."""
+    (rank r owns rows shard_range(n, r, world)); needs n % (64 * world) == 0."""
     n = full.shape[0]
-    if n % (32 * world):
-        raise ValueError("allgather_rows needs equal warp-aligned shards (n % (32*world) == 0)")
+    if n % (64 * world):
+        raise ValueError("allgather_rows needs equal warp-aligned shards (n % (64*world) == 0)")
     rank = dist.get_rank(group)
     lo, hi = shard_range(n, rank, world)
     wire = _wire(full.device, group)

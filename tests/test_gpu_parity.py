@@ -105,7 +105,8 @@ def test_bh_within_1e4_and_same_openings(bh_small, mode, sorted_):
         # a BH warp tile holds 64 bodies (2 per lane): its fetches are the union
         # of 64 traversals
         o = order.cpu().numpy() if sorted_ else np.arange(len(b))
-        union = oracle.unguided_warp_union(ot, b[o], 0.5, W=32)
+        W = 32 * P._lib.BH_POINTS_PER_LANE  # a BH warp tile holds 64 bodies
+        union = oracle.unguided_warp_union(ot, b[o], 0.5, W=W)
         assert np.array_equal(st.warp_fetches.cpu().numpy()[:len(union)], union)
 
 

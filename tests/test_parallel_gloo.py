@@ -37,7 +37,7 @@ def _worker(rank, world, port, q):
         blob = PAR.broadcast_blob(local if rank == 0 else None, "cpu")
         ok_blob = bool(np.array_equal(blob.numpy(), local))
         # results: each rank fills its own warp-aligned shard, then all-gather
-        n = 32 * world * 50
+        n = 64 * world * 50
         full = torch.full((n, 4), -1.0)
         lo, hi = PAR.shard_range(n, rank, world)
         full[lo:hi] = torch.arange(lo, hi, dtype=torch.float32)[:, None] + torch.tensor([0.0, 0.25, 0.5, 0.75])
@@ -73,6 +73,6 @@ def test_shard_range_partitions_warp_aligned(n, world):
     covered = np.zeros(n, np.int32)
     for r in range(world):
         lo, hi = shard_range(n, r, world)
-        assert lo % 32 == 0 or lo == n
+        assert lo % 64 == 0 or lo == n
         covered[lo:hi] += 1
     assert np.all(covered == 1)
