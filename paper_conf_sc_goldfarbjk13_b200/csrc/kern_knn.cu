@@ -13,7 +13,14 @@
 // push of §3.2.2 with its immediate pop folded away.
 // can_correlate (reading R5a): prune iff the k-heap is full and the tight box
 // distance exceeds the current k-th best -- conservative under the pinned
-// arithmetic, so the result is exactly the brute-force definition.
+// arithmetic, so the result is exactly the brute-force definition.  The box
+// distance of a child is computed while its parent is expanded (the blob
+// stores both children's boxes with the parent, `cbox`) and travels on the
+// rope stack with the node as Fig.7's non-invariant argument;
+// the test itself is made when the node is popped, against the k-th best of
+// that moment -- the same decision as testing at the visit, but a popped node
+// that is pruned costs no memory access, and an expanded node is one
+// independent load group (record + children's boxes).
 // Per-lane k-best list: KT register slots kept sorted ascending on (d2, id);
 // the first KT-k slots hold (-inf) sentinels, so the k-th best is always
 // slot KT-1 (static register index).
@@ -61,17 +68,6 @@ struct KBest {
     }
 };
 
-template <int DIM>
-__device__ __forceinline__ void ld_box(const float *s_box, const float *g_box, int dp, int top, int cur,
-                                       float (&lo)[DIM], float (&hi)[DIM]) {
-    if (cur < top) {
-        load_row_smem<DIM>(lo, s_box + (size_t)cur * 2 * dp);
-        load_row_smem<DIM>(hi, s_box + (size_t)cur * 2 * dp + dp);
-    } else {
-        load_row_nc<DIM>(lo, g_box + (size_t)cur * 2 * dp);
-        load_row_nc<DIM>(hi, g_box + (size_t)cur * 2 * dp + dp);
-    }
-}
 __device__ __forceinline__ void ld_rec(const unsigned char *s_rec, const tt_kd_rec *g_rec, int top, int cur,
                                        int4 &t, int4 &u) {
     if (cur < top) {
@@ -83,16 +79,26 @@ __device__ __forceinline__ void ld_rec(const unsigned char *s_rec, const tt_kd_r
     }
 }
 
-// Bring both children's box row and record towards L1 (one is the next node).
-template <int DP>
-__device__ __forceinline__ void prefetch_children(int4 t, int top, const tt_kd_rec *g_rec, const float *g_box) {
-    if (t.x >= top) {
-        prefetch_l1(g_rec + t.x);
-        prefetch_l1(g_box + (size_t)t.x * 2 * DP);
-    }
-    if (t.y >= top) {
-        prefetch_l1(g_rec + t.y);
-        prefetch_l1(g_box + (size_t)t.y * 2 * DP);
+// box distances of node `cur`'s two children (from the parent's cbox row)
+template <int DIM>
+__device__ __forceinline__ void child_lbs(const float *s_cbox, const float *g_cbox, int dp, int top, int cur,
+                                          const float (&q)[DIM], float &lb_left, float &lb_right) {
+    float lo[DIM], hi[DIM];
+    const float *row = (cur < top ? s_cbox : g_cbox) + (size_t)cur * 4 * dp;
+    if (cur < top) {
+        load_row_smem<DIM>(lo, row);
+        load_row_smem<DIM>(hi, row + dp);
+        lb_left = pinned_boxd2<DIM>(q, lo, hi);
+        load_row_smem<DIM>(lo, row + 2 * dp);
+        load_row_smem<DIM>(hi, row + 3 * dp);
+        lb_right = pinned_boxd2<DIM>(q, lo, hi);
+    } else {
+        load_row_nc<DIM>(lo, row);
+        load_row_nc<DIM>(hi, row + dp);
+        lb_left = pinned_boxd2<DIM>(q, lo, hi);
+        load_row_nc<DIM>(lo, row + 2 * dp);
+        load_row_nc<DIM>(hi, row + 3 * dp);
+        lb_right = pinned_boxd2<DIM>(q, lo, hi);
     }
 }
 
@@ -119,22 +125,28 @@ __global__ void __launch_bounds__(kBlock) knn_kernel(const tt_knn_params P, int 
     uint64_t *bar = reinterpret_cast<uint64_t *>(smem);
     const int top = P.c.top_count;
     unsigned char *s_rec = smem + kSmemHdr;
-    float *s_box = reinterpret_cast<float *>(s_rec + (size_t)top * 32);
-    int *s_stack = reinterpret_cast<int *>(reinterpret_cast<unsigned char *>(s_box) + (size_t)top * 8 * DP);
+    float *s_cbox = reinterpret_cast<float *>(s_rec + (size_t)top * 32);
+    unsigned char *s_stack = reinterpret_cast<unsigned char *>(s_cbox) + (size_t)top * 16 * DP;
     const tt_kd_rec *g_rec = static_cast<const tt_kd_rec *>(P.c.tree.rec);
-    const float *g_box = P.c.tree.box;
-    StageChunk ch[2] = {{s_rec, g_rec, (unsigned)top * 32u}, {s_box, g_box, (unsigned)top * 8u * DP}};
+    const float *g_cbox = P.c.tree.cbox;
+    StageChunk ch[2] = {{s_rec, g_rec, (unsigned)top * 32u}, {s_cbox, g_cbox, (unsigned)top * 16u * DP}};
     stage_top(bar, ch);
 
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
-    // per-warp region: N mode [cap][32] ints; L mode [cap] nodes + [cap] masks
-    int *w_stk = s_stack + (size_t)warp * cap * 32;
-    int *w_node = w_stk;
-    unsigned *w_mask = reinterpret_cast<unsigned *>(w_stk + cap);
+    // per-warp region of cap*32*8 bytes:
+    //   N: node[cap][32], lb[cap][32]       (per-lane stacks, lane-interleaved)
+    //   L: lb[cap][32], node[cap], mask[cap] (warp-uniform part owned by lane 0)
+    unsigned char *wreg = s_stack + (size_t)warp * cap * 32 * 8;
+    int *n_node = reinterpret_cast<int *>(wreg);
+    float *n_lb = reinterpret_cast<float *>(wreg + (size_t)cap * 32 * 4);
+    float *l_lb = reinterpret_cast<float *>(wreg);
+    int *l_node = reinterpret_cast<int *>(wreg + (size_t)cap * 32 * 4);
+    unsigned *l_mask = reinterpret_cast<unsigned *>(l_node + cap);
     const long long n = P.c.n;
     const long long ntiles = (n + 31) >> 5;
     const int k = P.k;
+    const float INF = __int_as_float(0x7f800000);
 
     for (;;) {
         const long long tile = next_tile(P.c.counter);
@@ -172,29 +184,33 @@ __global__ void __launch_bounds__(kBlock) knn_kernel(const tt_knn_params P, int 
         if (!lock) {
             int sp = 0;
             int cur = valid ? 0 : TT_END;
+            float lb = 0.f;  // the root is never pruned: the list starts empty
             while (cur != TT_END) {
                 if (STATS) ++visits;
-                bool prune = false;
-                if (kb.worst() < __int_as_float(0x7f800000)) {  // list full
-                    float lo[DIM], hi[DIM];
-                    ld_box<DIM>(s_box, g_box, DP, top, cur, lo, hi);
-                    prune = pinned_boxd2<DIM>(q, lo, hi) > kb.worst();
-                }
-                if (!prune) {
+                if (!(kb.worst() < INF && lb > kb.worst())) {  // can_correlate
                     int4 t, u;
                     ld_rec(s_rec, g_rec, top, cur, t, u);
                     if (t.x < 0) {
                         leaf_update<DIM, KT>(P, u.z, u.w, DP, q, kb);
                     } else {
-                        prefetch_children<DP>(t, top, g_rec, g_box);
+                        float lbl, lbr;
+                        child_lbs<DIM>(s_cbox, g_cbox, DP, top, cur, q, lbl, lbr);
                         const bool left_near = select_dim<DIM>(q, u.y) < __int_as_float(u.x);
-                        w_stk[sp * 32 + lane] = left_near ? t.y : t.x;  // push far
+                        n_node[sp * 32 + lane] = left_near ? t.y : t.x;  // push far with its bound
+                        n_lb[sp * 32 + lane] = left_near ? lbr : lbl;
                         ++sp;
                         cur = left_near ? t.x : t.y;                     // visit near
+                        lb = left_near ? lbl : lbr;
                         continue;
                     }
                 }
-                cur = sp > 0 ? w_stk[(--sp) * 32 + lane] : TT_END;
+                if (sp > 0) {
+                    --sp;
+                    cur = n_node[sp * 32 + lane];
+                    lb = n_lb[sp * 32 + lane];
+                } else {
+                    cur = TT_END;
+                }
             }
             if (STATS) {
                 fetches = warp_sum(visits);
@@ -204,32 +220,35 @@ __global__ void __launch_bounds__(kBlock) knn_kernel(const tt_knn_params P, int 
             int sp = 0;
             int cur = 0;
             unsigned mask = vmask;
+            float lb = 0.f;
             for (;;) {
                 const bool in = (mask >> lane) & 1u;
                 if (STATS) {
                     ++steps;
                     visits += in;
                 }
-                float lo[DIM], hi[DIM];
-                ld_box<DIM>(s_box, g_box, DP, top, cur, lo, hi);
-                const bool active =
-                    in && !(kb.worst() < __int_as_float(0x7f800000) && pinned_boxd2<DIM>(q, lo, hi) > kb.worst());
+                const bool active = in && !(kb.worst() < INF && lb > kb.worst());
                 const unsigned act = __ballot_sync(TT_FULL, active);
                 if (act) {
+                    if (STATS) ++fetches;
                     int4 t, u;
                     ld_rec(s_rec, g_rec, top, cur, t, u);
                     if (t.x < 0) {
                         if (active) leaf_update<DIM, KT>(P, u.z, u.w, DP, q, kb);
                     } else {
+                        float lbl, lbr;
+                        child_lbs<DIM>(s_cbox, g_cbox, DP, top, cur, q, lbl, lbr);
                         const bool pref_left = active && select_dim<DIM>(q, u.y) < __int_as_float(u.x);
                         const int votes = __popc(__ballot_sync(TT_FULL, pref_left));
                         const bool left_first = 2 * votes >= __popc(act);
                         if (lane == 0) {  // push second (warp-uniform entry)
-                            w_node[sp] = left_first ? t.y : t.x;
-                            w_mask[sp] = act;
+                            l_node[sp] = left_first ? t.y : t.x;
+                            l_mask[sp] = act;
                         }
+                        l_lb[sp * 32 + lane] = left_first ? lbr : lbl;
                         ++sp;
                         cur = left_first ? t.x : t.y;
+                        lb = left_first ? lbl : lbr;
                         mask = act;
                         continue;
                     }
@@ -240,13 +259,13 @@ __global__ void __launch_bounds__(kBlock) knn_kernel(const tt_knn_params P, int 
                 int e_node = 0;
                 unsigned e_mask = 0;
                 if (lane == 0) {
-                    e_node = w_node[sp];
-                    e_mask = w_mask[sp];
+                    e_node = l_node[sp];
+                    e_mask = l_mask[sp];
                 }
                 cur = __shfl_sync(TT_FULL, e_node, 0);
                 mask = __shfl_sync(TT_FULL, e_mask, 0);
+                lb = l_lb[sp * 32 + lane];
             }
-            fetches = steps;
         }
         if (valid) {
 #pragma unroll
@@ -270,7 +289,7 @@ template <int DIM, int KT, bool STATS>
 int launch(const tt_knn_params &p, const tt_launch_cfg &cfg) {
     constexpr int DP = (DIM + 3) & ~3;
     const int cap = p.c.height + 2;
-    const size_t smem = kSmemHdr + (size_t)p.c.top_count * (32 + 8 * DP) + (size_t)kWarps * cap * 32 * 4;
+    const size_t smem = kSmemHdr + (size_t)p.c.top_count * (32 + 16 * DP) + (size_t)kWarps * cap * 32 * 8;
     auto kern = knn_kernel<DIM, KT, STATS>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return (int)e;

@@ -111,6 +111,8 @@ void plan(const tt_tree_desc *d, tt_blob_header &h, std::vector<int32_t> *newidx
         off = align256(off + (uint64_t)d->n_points * h.dp * sizeof(float));
         h.off_pid = off;
         off = align256(off + (uint64_t)d->n_points * sizeof(int32_t));
+        h.off_cbox = off;
+        off = align256(off + (uint64_t)d->n_nodes * 4 * h.dp * sizeof(float));
     } else if (d->kind == TT_KIND_VP) {
         h.off_vpt = off;
         off = align256(off + (uint64_t)d->n_nodes * h.dp * sizeof(float));
@@ -192,6 +194,20 @@ int tt_pack_impl(const tt_tree_desc *d, void *blob, size_t bytes) {
                 b[k] = d->lo[v * d->dim + k];
                 b[h.dp + k] = d->hi[v * d->dim + k];
             }
+        }
+        // children's boxes stored with the parent: the kNN walk tests a child's
+        // box while expanding the parent (one load group per visited node)
+        auto *cbox = reinterpret_cast<float *>(base + h.off_cbox);
+        for (int64_t v = 0; v < N; ++v) {
+            const int32_t l = d->first_child[v];
+            if (l < 0) continue;
+            const int32_t kids[2] = {l, d->skip[l]};
+            float *dst = cbox + (size_t)nx[(size_t)v] * 4 * h.dp;
+            for (int c = 0; c < 2; ++c)
+                for (int k = 0; k < d->dim; ++k) {
+                    dst[c * 2 * h.dp + k] = d->lo[(int64_t)kids[c] * d->dim + k];
+                    dst[c * 2 * h.dp + h.dp + k] = d->hi[(int64_t)kids[c] * d->dim + k];
+                }
         }
         auto *pts = reinterpret_cast<float *>(base + h.off_pts);
         auto *pid = reinterpret_cast<int32_t *>(base + h.off_pid);

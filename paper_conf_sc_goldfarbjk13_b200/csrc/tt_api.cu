@@ -107,6 +107,7 @@ tt_status adopt_blob(const tt_blob_header &h, void *d_blob, cudaStream_t cs, tt_
     t->dev.pts = h.off_pts ? reinterpret_cast<const float *>(base + h.off_pts) : nullptr;
     t->dev.pid = h.off_pid ? reinterpret_cast<const int32_t *>(base + h.off_pid) : nullptr;
     t->dev.vpt = h.off_vpt ? reinterpret_cast<const float *>(base + h.off_vpt) : nullptr;
+    t->dev.cbox = h.off_cbox ? reinterpret_cast<const float *>(base + h.off_cbox) : nullptr;
     t->slot_next = 0;
     *out = t;
     return TT_OK;
@@ -313,7 +314,7 @@ tt_status tt_traverse_knn(const tt_tree *t, const float *q, int64_t n, int32_t l
                           float *d2_out, const tt_traverse_opts *opts, tt_stream s) {
     tt_knn_params p;
     tt_launch_cfg cfg;
-    tt_status st = setup_common(t, TT_KIND_KD, n, opts, kAutoKNN, 32 + 8 * t->hdr.dp, kTopKNN, p.c, cfg, s);
+    tt_status st = setup_common(t, TT_KIND_KD, n, opts, kAutoKNN, 32 + 16 * t->hdr.dp, kTopKNN, p.c, cfg, s);
     if (st != TT_OK) return st;
     if (k < 1) return TT_ERR_INVALID_ARG;
     if (k > TT_MAX_K) return TT_ERR_UNSUPPORTED;

@@ -11,7 +11,7 @@
 #include "../../include/tt.h"
 
 #define TT_BLOB_MAGIC 0x31425454u /* "TTB1" */
-#define TT_BLOB_VERSION 1u
+#define TT_BLOB_VERSION 2u
 #define TT_END (-1)               /* rope past the last node = end of traversal */
 #define TT_TOP_BYTES (32 * 1024)  /* shared-memory budget for the staged top levels */
 #define TT_COUNTER_SLOTS 256      /* tile-scheduler counter slots per tree */
@@ -59,6 +59,7 @@ struct tt_blob_header {
     double root_center[3], root_side;
     uint64_t off_rec, off_box, off_pts, off_pid, off_vpt, total;
     uint64_t rec_bytes; // bytes per record in the rec section (32 or 16)
+    uint64_t off_cbox;  // KD: children's boxes per node [n][2 children][lo dp, hi dp] (0 = leaf)
 };
 
 // Device-side view of an uploaded tree.
@@ -69,6 +70,7 @@ struct tt_dev_tree {
     const float *pts;     // KD: [n_points][dp] tree order
     const int32_t *pid;   // KD: [n_points]; VP: [n_nodes]
     const float *vpt;     // VP: [n_nodes][dp]
+    const float *cbox;    // KD: [n_nodes][2][2*dp] boxes of the two children
 };
 
 // ---------------------------------------------------------------------------

@@ -88,7 +88,7 @@ HDR = np.dtype([("magic", "<u4"), ("version", "<u4"), ("kind", "<i4"), ("dim", "
                 ("height", "<i4"), ("leaf_size", "<i4"), ("top_levels", "<i4"), ("top_count", "<i4"),
                 ("pad0", "<i4"), ("level_prefix", "<i4", 33), ("pad1", "<i4"), ("n_nodes", "<i8"), ("n_points", "<i8"), ("root_center", "<f8", 3),
                 ("root_side", "<f8"), ("off_rec", "<u8"), ("off_box", "<u8"), ("off_pts", "<u8"),
-                ("off_pid", "<u8"), ("off_vpt", "<u8"), ("total", "<u8"), ("rec_bytes", "<u8")])
+                ("off_pid", "<u8"), ("off_vpt", "<u8"), ("total", "<u8"), ("rec_bytes", "<u8"), ("off_cbox", "<u8")])
 
 
 def _walk_preorder(first_child, skip, n):
@@ -149,6 +149,12 @@ def test_kd_blob_children_and_points():
     box = np.frombuffer(blob[hd["off_box"]:hd["off_box"] + 8 * dp * h.n_nodes].tobytes(), "<f4")
     box = box.reshape(h.n_nodes, 2, dp)
     assert np.array_equal(box[seq, 0, :7], h.array("lo")) and np.array_equal(box[seq, 1, :7], h.array("hi"))
+    # children's boxes stored with the parent (kNN layout)
+    cbox = np.frombuffer(blob[hd["off_cbox"]:hd["off_cbox"] + 16 * dp * h.n_nodes].tobytes(), "<f4")
+    cbox = cbox.reshape(h.n_nodes, 2, 2, dp)
+    for v in np.nonzero(inner)[0][:500]:
+        for c, kid in enumerate((rec["left"][v], rec["right"][v])):
+            assert np.array_equal(cbox[v, c, 0], box[kid, 0]) and np.array_equal(cbox[v, c, 1], box[kid, 1])
 
 
 # ------------------------------------------------------------ error paths
