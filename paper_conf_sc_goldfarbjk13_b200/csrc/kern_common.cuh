@@ -108,6 +108,13 @@ __device__ __forceinline__ void sqr2_rn(float a0, float a1, float &r0, float &r1
         : "f"(a0), "f"(a1));
 }
 
+// max(a, b, c) in one FMNMX3 (sm_100 three-input min/max)
+__device__ __forceinline__ float max3(float a, float b, float c) {
+    float r;
+    asm("max.f32 %0, %1, %2, %3;" : "=f"(r) : "f"(a), "f"(b), "f"(c));
+    return r;
+}
+
 // per-dimension squared differences rn(rn(q_d - p_d)^2) into sq[]
 template <int DIM>
 __device__ __forceinline__ void sq_diffs(const float (&q)[DIM], const float *p, float (&sq)[DIM]) {
@@ -142,11 +149,11 @@ __device__ __forceinline__ float pinned_boxd2(const float (&q)[DIM], const float
         float a0, a1, b0, b1;
         sub2_rn(lo[d], lo[d + 1], q[d], q[d + 1], a0, a1);
         sub2_rn(q[d], q[d + 1], hi[d], hi[d + 1], b0, b1);
-        sqr2_rn(fmaxf(fmaxf(a0, b0), 0.0f), fmaxf(fmaxf(a1, b1), 0.0f), sq[d], sq[d + 1]);
+        sqr2_rn(max3(a0, b0, 0.0f), max3(a1, b1, 0.0f), sq[d], sq[d + 1]);
     }
     if (DIM & 1) {
         const int d = DIM - 1;
-        const float t = fmaxf(fmaxf(__fsub_rn(lo[d], q[d]), __fsub_rn(q[d], hi[d])), 0.0f);
+        const float t = max3(__fsub_rn(lo[d], q[d]), __fsub_rn(q[d], hi[d]), 0.0f);
         sq[d] = __fmul_rn(t, t);
     }
     float s = sq[0];
