@@ -273,6 +273,7 @@ int tt_build_oct_gpu_impl(const float *bodies_f, long long n, void *stream, tt_b
                           void **blob_out) {
     cudaStream_t s = (cudaStream_t)stream;
     const float4 *bodies = reinterpret_cast<const float4 *>(bodies_f);
+    tt_keep_pool_memory();
     Scratch W{s};
     const unsigned G = grid_for(n);
 

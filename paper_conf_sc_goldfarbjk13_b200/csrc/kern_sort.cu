@@ -105,9 +105,25 @@ void launch_keys(const tt_tree *t, const float *pts, long long n, int ld, unsign
 
 }  // namespace
 
+// Keep freed stream-ordered scratch in the device's default pool across
+// synchronisations (the default release threshold of 0 returns it to the OS
+// at every sync, and the next cudaMallocAsync maps fresh memory: ~ms).
+void tt_keep_pool_memory() {
+    static int done_dev = -1;
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev == done_dev) return;
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+        uint64_t thr = UINT64_MAX;
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+    done_dev = dev;
+}
+
 int tt_launch_sort(const tt_tree *t, const float *pts, int64_t n, int32_t ld, uint32_t *perm, uint64_t *keys_out,
                    void *stream) {
     cudaStream_t s = (cudaStream_t)stream;
+    tt_keep_pool_memory();
     unsigned long long *keys = nullptr, *keys_alt = nullptr;
     uint32_t *vals = nullptr;
     void *tmp = nullptr;

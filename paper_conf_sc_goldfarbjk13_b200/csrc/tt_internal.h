@@ -169,6 +169,9 @@ int tt_build_oct_gpu_impl(const float *bodies, long long n, void *stream, tt_blo
 
 int tt_launch_kick_drift(float *x, float *v, const float *a, long long n, float dtk, float dtd, void *stream);
 
+// Default mempool keeps freed stream-ordered scratch across syncs (kern_sort.cu).
+void tt_keep_pool_memory();
+
 // Host helpers (host_build.cpp / pack.cpp)
 size_t tt_pack_size_impl(const tt_tree_desc *d, int *status);
 int tt_pack_impl(const tt_tree_desc *d, void *blob, size_t bytes);
