@@ -60,7 +60,8 @@ def parse():
     ap.add_argument("--points-per-rank", type=int, default=0, help="override M (testing)")
     ap.add_argument("--auto-min-depth", type=int, default=None, help="AUTO-mode threshold (default: kernel's)")
     ap.add_argument("--device-build", action="store_true",
-                    help="BH: build the oct-tree on the GPU (tt_build_oct_device) instead of host build + upload")
+                    help="build the tree on the GPU (tt_build_oct_device / tt_build_kd_device) instead of host "
+                         "build + upload")
     ap.add_argument("--variant", default="autoropes", choices=["autoropes", "recursive"],
                     help="recursive = the paper's naive recursive GPU baseline (ablation, N mode)")
     return ap.parse_args()
@@ -329,14 +330,15 @@ def run_ours(args, rank, world, local_rank):
 
     # a0: tree (rank 0 builds; NCCL broadcast for N > 1) -- timed separately
     t0 = time.perf_counter()
-    if args.device_build and name == "bh":
-        # every rank builds the identical tree from the identical bodies (NEXT-1)
-        bodies_dev = torch.from_numpy(np.ascontiguousarray(w["data"])).to(device)
+    if args.device_build and name in ("bh", "knn", "pc"):
+        # every rank builds the identical tree from the identical points (NEXT-1)
+        data_dev = torch.from_numpy(np.ascontiguousarray(w["data"])).to(device)
         torch.cuda.synchronize()
         t0 = time.perf_counter()
-        tree = P.tt_build_oct_device(bodies_dev)
+        tree = (P.tt_build_oct_device(data_dev) if name == "bh"
+                else P.tt_build_kd_device(data_dev, w["cfg"]["leaf"]))
         t1 = time.perf_counter()
-        del bodies_dev
+        del data_dev
     elif world == 1:
         host = host_tree(P, name, w)
         t1 = time.perf_counter()
@@ -348,7 +350,8 @@ def run_ours(args, rank, world, local_rank):
     torch.cuda.synchronize()
     t2 = time.perf_counter()
     build_ms, upload_ms = 1e3 * (t1 - t0), 1e3 * (t2 - t1)
-    build_where = "device (tt_build_oct_device)" if (args.device_build and name == "bh") else "host (tt_build_*)"
+    build_where = ("device (tt_build_*_device)" if (args.device_build and name in ("bh", "knn", "pc"))
+                   else "host (tt_build_*)")
 
     q_all = torch.from_numpy(np.ascontiguousarray(w["queries"])).to(device)
     q_shard = q_all[lo:hi]

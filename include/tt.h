@@ -157,6 +157,12 @@ tt_status tt_tree_upload(const tt_tree_desc *d, tt_stream s, tt_tree **out);
  * (build rules R8a/R9).  Synchronises `s`.  Errors: TT_ERR_INVALID_ARG,
  * TT_ERR_TREE_TOO_DEEP (never for R9 trees: height <= 33), TT_ERR_CUDA/OOM. */
 tt_status tt_build_oct_device(const float *bodies, int64_t n, tt_stream s, tt_tree **out);
+/* NEXT-1: build a kd-tree (median splits, reading R3) on the GPU from device
+ * points (n rows of `ld` floats, dim <= TT_MAX_DIM) straight into the packed
+ * device layout -- the bytes tt_tree_pack produces for tt_build_kd.
+ * Synchronises `s` once per tree level.                                    */
+tt_status tt_build_kd_device(const float *pts, int64_t n, int32_t dim, int32_t ld, int32_t leaf_size, tt_stream s,
+                             tt_tree **out);
 /* Copy the packed device blob back to host memory (bytes >= device_bytes of
  * tt_tree_get_info); synchronous.  E.g. to checkpoint a tree.              */
 tt_status tt_tree_download(const tt_tree *t, void *host_blob, size_t bytes);

@@ -204,6 +204,21 @@ tt_status tt_build_oct_device(const float *bodies, int64_t n, tt_stream s, tt_tr
     return st;
 }
 
+tt_status tt_build_kd_device(const float *pts, int64_t n, int32_t dim, int32_t ld, int32_t leaf_size, tt_stream s,
+                             tt_tree **out) {
+    if (!pts || !out || n <= 0 || n > INT32_MAX / 2 || dim <= 0 || dim > TT_MAX_DIM || ld < dim || leaf_size <= 0)
+        return TT_ERR_INVALID_ARG;
+    tt_status st = have_device();
+    if (st != TT_OK) return st;
+    tt_blob_header h;
+    void *d_blob = nullptr;
+    const int e = tt_build_kd_gpu_impl(pts, n, dim, ld, leaf_size, s, &h, &d_blob);
+    if (e) return cuda_fail((cudaError_t)e);
+    st = adopt_blob(h, d_blob, (cudaStream_t)s, out);
+    if (st != TT_OK) cudaFree(d_blob);
+    return st;
+}
+
 tt_status tt_tree_download(const tt_tree *t, void *host_blob, size_t bytes) {
     if (!t || !host_blob || bytes < t->bytes) return TT_ERR_INVALID_ARG;
     const cudaError_t e = cudaMemcpy(host_blob, t->d_blob, t->bytes, cudaMemcpyDeviceToHost);

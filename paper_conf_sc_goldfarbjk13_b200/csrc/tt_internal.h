@@ -169,6 +169,9 @@ int tt_build_oct_gpu_impl(const float *bodies, long long n, void *stream, tt_blo
 
 int tt_launch_kick_drift(float *x, float *v, const float *a, long long n, float dtk, float dtd, void *stream);
 
+int tt_build_kd_gpu_impl(const float *pts, long long n, int dim, int ld, int leaf, void *stream, tt_blob_header *hdr,
+                         void **blob);
+
 // Default mempool keeps freed stream-ordered scratch across syncs (kern_sort.cu).
 void tt_keep_pool_memory();
 

@@ -455,3 +455,17 @@ def test_plummer_steps_forces_match_oracle_each_step():
     p = (B.cpu().numpy()[:, 3:4].astype(np.float64) * V.cpu().numpy()[:, :3]).sum(0)
     p0 = (b[:, 3:4].astype(np.float64) * v[:, :3]).sum(0)
     assert np.abs(p - p0).max() < 1e-4
+
+
+@pytest.mark.parametrize("n,dim,leaf", [(1, 3, 1), (2, 3, 1), (10_000, 3, 1), (20_011, 7, 8), (5_000, 16, 4),
+                                        (1_000_000, 7, 8)])
+def test_gpu_kd_build_is_byte_identical_to_host_pack(n, dim, leaf):
+    p = ttgen.gaussian_mixture(n, dim, seed=220, components=6)
+    if n > 100:
+        p[50:60] = p[7]  # duplicates: ties broken by id
+    host_blob = P.build_kd(p, leaf).pack()
+    t = P.tt_build_kd_device(dev(p), leaf)
+    gpu_blob = P.tt_tree_download(t)
+    assert gpu_blob.size == host_blob.size
+    diff = np.nonzero(gpu_blob != host_blob)[0]
+    assert diff.size == 0, f"{diff.size} bytes differ, first at {diff[:8]}"
