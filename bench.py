@@ -330,12 +330,13 @@ def run_ours(args, rank, world, local_rank):
 
     # a0: tree (rank 0 builds; NCCL broadcast for N > 1) -- timed separately
     t0 = time.perf_counter()
-    if args.device_build and name in ("bh", "knn", "pc"):
+    if args.device_build:
         # every rank builds the identical tree from the identical points (NEXT-1)
         data_dev = torch.from_numpy(np.ascontiguousarray(w["data"])).to(device)
         torch.cuda.synchronize()
         t0 = time.perf_counter()
         tree = (P.tt_build_oct_device(data_dev) if name == "bh"
+                else P.tt_build_vp_device(data_dev) if name == "vp"
                 else P.tt_build_kd_device(data_dev, w["cfg"]["leaf"]))
         t1 = time.perf_counter()
         del data_dev
@@ -350,8 +351,7 @@ def run_ours(args, rank, world, local_rank):
     torch.cuda.synchronize()
     t2 = time.perf_counter()
     build_ms, upload_ms = 1e3 * (t1 - t0), 1e3 * (t2 - t1)
-    build_where = ("device (tt_build_*_device)" if (args.device_build and name in ("bh", "knn", "pc"))
-                   else "host (tt_build_*)")
+    build_where = "device (tt_build_*_device)" if args.device_build else "host (tt_build_*)"
 
     q_all = torch.from_numpy(np.ascontiguousarray(w["queries"])).to(device)
     q_shard = q_all[lo:hi]

@@ -163,6 +163,9 @@ tt_status tt_build_oct_device(const float *bodies, int64_t n, tt_stream s, tt_tr
  * Synchronises `s` once per tree level.                                    */
 tt_status tt_build_kd_device(const float *pts, int64_t n, int32_t dim, int32_t ld, int32_t leaf_size, tt_stream s,
                              tt_tree **out);
+/* NEXT-1: build a vantage-point tree (reading R12) on the GPU, same contract
+ * as tt_build_kd_device (bytes identical to tt_tree_pack of tt_build_vp). */
+tt_status tt_build_vp_device(const float *pts, int64_t n, int32_t dim, int32_t ld, tt_stream s, tt_tree **out);
 /* Copy the packed device blob back to host memory (bytes >= device_bytes of
  * tt_tree_get_info); synchronous.  E.g. to checkpoint a tree.              */
 tt_status tt_tree_download(const tt_tree *t, void *host_blob, size_t bytes);

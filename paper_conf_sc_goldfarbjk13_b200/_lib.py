@@ -82,6 +82,7 @@ SIGNATURES = {
     "tt_tree_upload": (I32, [P, P, P]),
     "tt_build_oct_device": (I32, [P, I64, P, P]),
     "tt_build_kd_device": (I32, [P, I64, I32, I32, I32, P, P]),
+    "tt_build_vp_device": (I32, [P, I64, I32, I32, P, P]),
     "tt_tree_download": (I32, [P, P, SZ]),
     "tt_kick_drift": (I32, [P, P, P, I64, F, F, P]),
     "tt_tree_free": (I32, [P]),

@@ -172,6 +172,9 @@ int tt_launch_kick_drift(float *x, float *v, const float *a, long long n, float 
 int tt_build_kd_gpu_impl(const float *pts, long long n, int dim, int ld, int leaf, void *stream, tt_blob_header *hdr,
                          void **blob);
 
+int tt_build_vp_gpu_impl(const float *pts, long long n, int dim, int ld, void *stream, tt_blob_header *hdr,
+                         void **blob);
+
 // Default mempool keeps freed stream-ordered scratch across syncs (kern_sort.cu).
 void tt_keep_pool_memory();
 

@@ -469,3 +469,16 @@ def test_gpu_kd_build_is_byte_identical_to_host_pack(n, dim, leaf):
     assert gpu_blob.size == host_blob.size
     diff = np.nonzero(gpu_blob != host_blob)[0]
     assert diff.size == 0, f"{diff.size} bytes differ, first at {diff[:8]}"
+
+
+@pytest.mark.parametrize("n,dim", [(1, 3), (2, 3), (3, 2), (5_000, 16), (20_011, 7), (1_000_000, 16)])
+def test_gpu_vp_build_is_byte_identical_to_host_pack(n, dim):
+    p = ttgen.gaussian_mixture(n, dim, seed=221, components=6)
+    if n > 100:
+        p[50:60] = p[7]  # equal distances: ties broken by id
+    host_blob = P.build_vp(p).pack()
+    t = P.tt_build_vp_device(dev(p))
+    gpu_blob = P.tt_tree_download(t)
+    assert gpu_blob.size == host_blob.size
+    diff = np.nonzero(gpu_blob != host_blob)[0]
+    assert diff.size == 0, f"{diff.size} bytes differ, first at {diff[:8]}"
