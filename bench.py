@@ -212,6 +212,21 @@ def load_counts(workload: str, mode: str):
         return None
 
 
+def libtt_sha256() -> str:
+    """Hash of libtt's sources and build script (nvcc output bytes are not
+    reproducible; the sources decide the instruction stream)."""
+    import glob
+    import hashlib
+    h = hashlib.sha256()
+    pkg = os.path.join(ROOT, "paper_conf_sc_goldfarbjk13_b200")
+    files = sorted(glob.glob(os.path.join(pkg, "csrc", "*"))) + [os.path.join(pkg, "build.py"),
+                                                                  os.path.join(ROOT, "include", "tt.h")]
+    for f in files:
+        h.update(os.path.basename(f).encode())
+        h.update(open(f, "rb").read())
+    return h.hexdigest()
+
+
 def measured_peaks():
     try:
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))), "measured"
@@ -531,23 +546,33 @@ def run_ours(args, rank, world, local_rank):
     clocks = clk.summary()
     sm_mhz = clocks.get("sm_mhz") or float(peaks.get("sm_max_mhz", 1965.0))
     nsm = torch.cuda.get_device_properties(device).multi_processor_count
-    issue = None
-    if cnt:
+    # The kernels are not HBM-bound (trees L2-resident, lockstep broadcast):
+    # the binding roof is instruction issue (ncu issue-slot utilisation), so
+    # the primary roofline is executed warp instructions per second against
+    # 148 SMs x 4 schedulers x clock; SURVEY §8(d)'s effective node-fetch
+    # bandwidth (the north_star's "% HBM peak") is reported alongside.
+    hbm_eff = {"bound": "hbm", "achieved": round(achieved, 1), "peak": hbm, "unit": "GB/s",
+               "frac": round(achieved / hbm, 4), "peak_source": peak_src,
+               "alg_bytes_per_launch": int(alg_bytes),
+               "alg_bytes_def": f"useful visits x {bpv} B record + {BYTES_PER_POINT_IO[name]} B/point I/O "
+                                "(SURVEY 8(d)); served by L1/L2 and warp broadcast, not HBM",
+               "warp_fetch_bytes_per_launch": int(wf * bpv)}
+    common = {"kernel": kernel_name, "kernel_ms": round(kms, 4),
+              "kernel_share_of_step": round(kms / ms, 4) if world == 1 else None,
+              "traffic": int(cnt["dram_bytes_per_point"] * m) if cnt else None,
+              "traffic_def": "ncu dram__bytes_read.sum + dram__bytes_write.sum per launch (scaled per point)"}
+    if cnt and cnt.get("so_sha256") == libtt_sha256():
         inst = cnt["warp_inst_per_point"] * m
-        issue_peak = nsm * 4 * sm_mhz * 1e6 / 1e9  # warp instructions / ns -> G/s
-        issue = {"bound": "issue", "achieved": round(inst / (kms / 1e3) / 1e9, 1), "peak": round(issue_peak, 1),
-                 "unit": "Gwarp-inst/s", "frac": round(inst / (kms / 1e3) / 1e9 / issue_peak, 4),
-                 "inst_per_launch": int(inst), "source": f"ncu smsp__inst_executed ({cnt['round']}) x live time",
-                 "peak_def": f"{nsm} SMs x 4 schedulers x 1 warp-inst/clk x {sm_mhz:.0f} MHz"}
-    roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": hbm, "unit": "GB/s",
-                "frac": round(achieved / hbm, 4),
-                "traffic": int(cnt["dram_bytes_per_point"] * m) if cnt else None,
-                "issue": issue,
-                "peak_source": peak_src, "kernel": kernel_name, "kernel_ms": round(kms, 4),
-                "kernel_share_of_step": round(kms / ms, 4) if world == 1 else None,
-                "alg_bytes_per_launch": int(alg_bytes),
-                "alg_bytes_def": f"useful visits x {bpv} B record + {BYTES_PER_POINT_IO[name]} B/point I/O",
-                "warp_fetch_bytes_per_launch": int(wf * bpv)}
+        issue_peak = nsm * 4 * sm_mhz * 1e6 / 1e9  # warp instructions per ns -> G/s
+        roofline = {"bound": "issue", "achieved": round(inst / (kms / 1e3) / 1e9, 1), "peak": round(issue_peak, 1),
+                    "unit": "Gwarp-inst/s", "frac": round(inst / (kms / 1e3) / 1e9 / issue_peak, 4),
+                    "inst_per_launch": int(inst),
+                    "achieved_def": f"ncu smsp__inst_executed of this libtt.so ({cnt['round']}) / live kernel time",
+                    "peak_def": f"{nsm} SMs x 4 schedulers x 1 warp-inst/clk x {sm_mhz:.0f} MHz (B200_PROFILING)",
+                    **common, "hbm_effective": hbm_eff}
+    else:
+        roofline = {**hbm_eff, **common, "issue": None,
+                    "note": "no ncu instruction count for this libtt.so build: HBM-effective roofline only"}
     cpu = None
     if world == 1 and not args.no_cpu_baseline:
         try:
