@@ -194,10 +194,14 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
                         if (STATS) bd[j].visits += active;
                         bd[j].wait = active ? (open ? INT_MAX : lvl) : bd[j].wait;
                         // branch-free update: in a warp step some lane almost always
-                        // interacts, so predication beats a divergent branch
-                        const bool inter = active && !open && t.z != bd[j].self;
+                        // interacts, so predication beats a divergent branch; the
+                        // three conditions fold into one LOP3 + one select
+                        const unsigned inter = (unsigned)active & (unsigned)!open & (unsigned)(t.z != bd[j].self);
                         const float inv = rsqrt_ftz(__fadd_rn(drsq, e2));
-                        const float f = inter ? g.w * (inv * inv) * inv : 0.0f;
+                        float mw;
+                        asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %1, 0;\n\tselp.f32 %0, %2, 0f00000000, p;\n\t}"
+                            : "=f"(mw) : "r"(inter), "f"(g.w));
+                        const float f = mw * (inv * inv) * inv;
                         bd[j].acc.x = fmaf(f, dx, bd[j].acc.x);
                         bd[j].acc.y = fmaf(f, dy, bd[j].acc.y);
                         bd[j].acc.z = fmaf(f, dz, bd[j].acc.z);
