@@ -21,7 +21,7 @@
 #include <cstring>
 #include <vector>
 
-#include "kern_common.cuh"
+#include "build_common.cuh"
 
 namespace {
 
@@ -224,45 +224,6 @@ __global__ void count_fresh_kernel(long long n, const int *rstart, const unsigne
         if (rstart[i] == i && fresh2[i]) atomicAdd(flag, 1);
 }
 
-unsigned gridn(long long n) {
-    long long g = (n + 255) / 256;
-    if (g > 148 * 8) g = 148 * 8;
-    return (unsigned)(g < 1 ? 1 : g);
-}
-
-inline uint64_t align256(uint64_t x) { return (x + 255) & ~uint64_t(255); }
-
-struct Scratch {
-    cudaStream_t s;
-    cudaError_t e = cudaSuccess;
-    std::vector<void *> ptrs;
-    template <class T>
-    T *get(size_t count) {
-        void *p = nullptr;
-        if (e == cudaSuccess) e = cudaMallocAsync(&p, count * sizeof(T) + 16, s);
-        if (e == cudaSuccess) ptrs.push_back(p);
-        return static_cast<T *>(p);
-    }
-    ~Scratch() {
-        for (void *p : ptrs) cudaFreeAsync(p, s);
-    }
-};
-
-// ---------------------------------------------------------------- packing
-__global__ void level_hist_kernel(const int *level, long long nn, unsigned *hist) {
-    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < nn; v += (long long)gridDim.x * blockDim.x)
-        atomicAdd(hist + level[v], 1u);
-}
-__global__ void flag_kernel(const int *level, long long nn, int top_levels, int l, int *flag) {
-    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < nn; v += (long long)gridDim.x * blockDim.x)
-        flag[v] = l < 0 ? (level[v] >= top_levels) : (level[v] == l);
-}
-__global__ void assign_kernel(const int *level, const int *rank, long long nn, int top_levels, int l, int offset,
-                              int *newidx) {
-    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < nn; v += (long long)gridDim.x * blockDim.x)
-        if (l < 0 ? level[v] >= top_levels : level[v] == l) newidx[v] = offset + rank[v];
-}
-
 __global__ void kd_records_kernel(long long nn, int D, int dp, NodeOut o, const int *newidx, tt_kd_rec *rec,
                                   float *box, float *cbox) {
     for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < nn; v += (long long)gridDim.x * blockDim.x) {
@@ -310,7 +271,7 @@ int tt_build_kd_gpu_impl(const float *pts, long long n, int D, int ld, int L, vo
     cudaStream_t s = (cudaStream_t)stream;
     tt_keep_pool_memory();
     Scratch W{s};
-    const unsigned G = gridn(n);
+    const unsigned G = build_grid(n);
     int *ids = W.get<int>(n), *ids2 = W.get<int>(n);
     Level lv;
     lv.rstart = W.get<int>(n);
@@ -342,7 +303,6 @@ int tt_build_kd_gpu_impl(const float *pts, long long n, int D, int ld, int L, vo
     if (W.e) return W.e;
     cudaError_t e;
     init_kernel<<<G, 256, 0, s>>>(n, ids, lv.rstart, lv.cnt, lv.pre, lv.fresh);
-    int height = 0;
     for (int level = 0;; ++level) {
         box_init_kernel<<<G, 256, 0, s>>>(n, D, lv.rstart, lv.fresh, lv.blo, lv.bhi);
         box_kernel<<<G, 256, 0, s>>>(n, D, pts, ld, ids, lv.rstart, lv.fresh, lv.blo, lv.bhi);
@@ -364,48 +324,19 @@ int tt_build_kd_gpu_impl(const float *pts, long long n, int D, int ld, int L, vo
         int hf = 0;
         if ((e = cudaMemcpyAsync(&hf, flag, sizeof(int), cudaMemcpyDeviceToHost, s))) return e;
         if ((e = cudaStreamSynchronize(s))) return e;
-        height = level;
         if (!hf) break;
         if (level > TT_MAX_HEIGHT) return cudaErrorInvalidValue;
     }
 
     // header + top-first renumbering (pack.cpp plan)
     const int dp = (D + 3) & ~3;
-    unsigned *hist = W.get<unsigned>(64);
-    int *newidx = W.get<int>(nn), *fl = W.get<int>(nn + 1), *rank = W.get<int>(nn + 1);
-    size_t sb2 = 0;
-    cub::DeviceScan::ExclusiveSum(nullptr, sb2, fl, rank, (int)nn, s);
-    void *st2 = W.get<unsigned char>(sb2);
-    if (W.e) return W.e;
-    const unsigned GN = gridn(nn);
-    if ((e = cudaMemsetAsync(hist, 0, 64 * sizeof(unsigned), s))) return e;
-    level_hist_kernel<<<GN, 256, 0, s>>>(o.level, nn, hist);
-    unsigned hh[64];
-    if ((e = cudaMemcpyAsync(hh, hist, sizeof(hh), cudaMemcpyDeviceToHost, s))) return e;
-    if ((e = cudaStreamSynchronize(s))) return e;
     tt_blob_header h;
-    std::memset(&h, 0, sizeof(h));
-    h.magic = TT_BLOB_MAGIC;
-    h.version = TT_BLOB_VERSION;
-    h.kind = TT_KIND_KD;
-    h.dim = D;
-    h.dp = dp;
-    h.height = height;
-    h.leaf_size = L;
-    h.n_nodes = nn;
-    h.n_points = n;
-    const int sbytes = 32 + 8 * dp;
-    long long acc = 0;
-    int Lv = 0;
-    h.level_prefix[0] = 0;
-    while (Lv <= height && Lv < TT_TOP_LEVELS_MAX && (acc + (long long)hh[Lv]) * sbytes <= TT_TOP_BYTES) {
-        acc += hh[Lv];
-        ++Lv;
-        h.level_prefix[Lv] = (int32_t)acc;
-    }
-    h.top_levels = Lv;
-    h.top_count = (int32_t)acc;
+    header_base(h, TT_KIND_KD, D, L, nn, n);
     h.rec_bytes = 32;
+    int *newidx = W.get<int>(nn);
+    if (W.e) return W.e;
+    if ((e = renumber_top_first(o.level, nn, 32 + 8 * dp, h, newidx, W))) return e;
+    const unsigned GN = build_grid(nn);
     uint64_t off = align256(sizeof(tt_blob_header));
     h.off_rec = off;
     off = align256(off + (uint64_t)nn * 32);
@@ -418,21 +349,9 @@ int tt_build_kd_gpu_impl(const float *pts, long long n, int D, int ld, int L, vo
     h.off_cbox = off;
     off = align256(off + (uint64_t)nn * 4 * dp * 4);
     h.total = off;
-    for (int l = -1; l < h.top_levels; ++l) {
-        flag_kernel<<<GN, 256, 0, s>>>(o.level, nn, h.top_levels, l, fl);
-        size_t q = sb2;
-        if ((e = cub::DeviceScan::ExclusiveSum(st2, q, fl, rank, (int)nn, s))) return e;
-        assign_kernel<<<GN, 256, 0, s>>>(o.level, rank, nn, h.top_levels, l, l < 0 ? h.top_count : h.level_prefix[l],
-                                         newidx);
-    }
     void *blob = nullptr;
-    if ((e = cudaMalloc(&blob, h.total))) return e;
+    if ((e = alloc_blob(h, s, &blob))) return e;
     auto *base = static_cast<unsigned char *>(blob);
-    if ((e = cudaMemsetAsync(blob, 0, h.total, s)) ||
-        (e = cudaMemcpyAsync(blob, &h, sizeof(h), cudaMemcpyHostToDevice, s))) {
-        cudaFree(blob);
-        return e;
-    }
     kd_records_kernel<<<GN, 256, 0, s>>>(nn, D, dp, o, newidx, reinterpret_cast<tt_kd_rec *>(base + h.off_rec),
                                          reinterpret_cast<float *>(base + h.off_box),
                                          reinterpret_cast<float *>(base + h.off_cbox));

@@ -25,7 +25,7 @@
 #include <cstring>
 #include <vector>
 
-#include "kern_common.cuh"
+#include "build_common.cuh"
 
 namespace {
 
@@ -174,34 +174,6 @@ __global__ void moments_kernel(const float4 *bodies, long long n_nodes, int lvl,
     }
 }
 
-__global__ void level_hist_kernel(const int *level, long long n_nodes, unsigned *hist /*[64]*/) {
-    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < n_nodes;
-         v += (long long)gridDim.x * blockDim.x)
-        atomicAdd(hist + level[v], 1u);
-}
-
-// flag[v] = 1 if node v is outside the top region (for the rest's renumbering),
-// lflag[v] = 1 if node v is on level `l`
-__global__ void flag_kernel(const int *level, long long n_nodes, int top_levels, int l, int *flag) {
-    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < n_nodes;
-         v += (long long)gridDim.x * blockDim.x)
-        flag[v] = l < 0 ? (level[v] >= top_levels) : (level[v] == l);
-}
-
-__global__ void assign_top_kernel(const int *level, const int *rank, long long n_nodes, int l, int offset,
-                                  int *newidx) {
-    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < n_nodes;
-         v += (long long)gridDim.x * blockDim.x)
-        if (level[v] == l) newidx[v] = offset + rank[v];
-}
-
-__global__ void assign_rest_kernel(const int *level, const int *rank, long long n_nodes, int top_levels,
-                                   int top_count, int *newidx) {
-    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < n_nodes;
-         v += (long long)gridDim.x * blockDim.x)
-        if (level[v] >= top_levels) newidx[v] = top_count + rank[v];
-}
-
 __global__ void records_kernel(long long n_nodes, NodeArrays A, const int *newidx, tt_oct_rec *rec) {
     for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < n_nodes;
          v += (long long)gridDim.x * blockDim.x) {
@@ -239,31 +211,6 @@ __global__ void gather_u64(const unsigned long long *src, const unsigned *perm, 
         dst[i] = src[perm[i]];
 }
 
-unsigned grid_for(long long n) {
-    long long g = (n + 255) / 256;
-    if (g > 148 * 8) g = 148 * 8;
-    return (unsigned)(g < 1 ? 1 : g);
-}
-
-inline uint64_t align256(uint64_t x) { return (x + 255) & ~uint64_t(255); }
-
-// Stream-ordered scratch allocations released at scope exit.
-struct Scratch {
-    cudaStream_t s;
-    cudaError_t e = cudaSuccess;
-    std::vector<void *> ptrs;
-    template <class T>
-    T *get(size_t count) {
-        void *p = nullptr;
-        if (e == cudaSuccess) e = cudaMallocAsync(&p, count * sizeof(T) + 16, s);
-        if (e == cudaSuccess) ptrs.push_back(p);
-        return static_cast<T *>(p);
-    }
-    ~Scratch() {
-        for (void *p : ptrs) cudaFreeAsync(p, s);
-    }
-};
-
 }  // namespace
 
 // Build on `stream`: writes the host copy of the blob header and a cudaMalloc'd
@@ -275,7 +222,7 @@ int tt_build_oct_gpu_impl(const float *bodies_f, long long n, void *stream, tt_b
     const float4 *bodies = reinterpret_cast<const float4 *>(bodies_f);
     tt_keep_pool_memory();
     Scratch W{s};
-    const unsigned G = grid_for(n);
+    const unsigned G = build_grid(n);
 
     // 1. root cube
     float *d_box = W.get<float>(6);
@@ -340,7 +287,7 @@ int tt_build_oct_gpu_impl(const float *bodies_f, long long n, void *stream, tt_b
     A.m1 = W.get<double>(3 * n_nodes);
     unsigned *hist = W.get<unsigned>(64);
     if (W.e) return W.e;
-    const unsigned GN = grid_for(n_nodes);
+    const unsigned GN = build_grid(n_nodes);
     emit_kernel<<<G, 256, 0, s>>>(k0s, k1s, ids_s, dn, base, n, n_nodes, A);
     if ((e = cudaMemsetAsync(hist, 0, 64 * sizeof(unsigned), s))) return e;
     level_hist_kernel<<<GN, 256, 0, s>>>(A.level, n_nodes, hist);
@@ -356,52 +303,18 @@ int tt_build_oct_gpu_impl(const float *bodies_f, long long n, void *stream, tt_b
 
     // 6. header (same plan as pack.cpp), renumbering, records
     tt_blob_header h;
-    std::memset(&h, 0, sizeof(h));
-    h.magic = TT_BLOB_MAGIC;
-    h.version = TT_BLOB_VERSION;
-    h.kind = TT_KIND_OCT;
-    h.dim = 3;
-    h.dp = 4;
-    h.height = height;
-    h.leaf_size = 1;
-    h.n_nodes = n_nodes;
-    h.n_points = n;
+    header_base(h, TT_KIND_OCT, 3, 1, n_nodes, n);
     for (int d = 0; d < 3; ++d) h.root_center[d] = cube.c[d];
     h.root_side = cube.side;
-    long long acc = 0;
-    int L = 0;
-    h.level_prefix[0] = 0;
-    while (L <= height && L < TT_TOP_LEVELS_MAX && (acc + (long long)hh[L]) * 32 <= TT_TOP_BYTES) {
-        acc += hh[L];
-        ++L;
-        h.level_prefix[L] = (int32_t)acc;
-    }
-    h.top_levels = L;
-    h.top_count = (int32_t)acc;
     h.rec_bytes = 32;
+    int *newidx = W.get<int>(n_nodes);
+    if (W.e) return W.e;
+    if ((e = renumber_top_first(A.level, n_nodes, 32, h, newidx, W))) return e;
     h.off_rec = align256(sizeof(tt_blob_header));
     h.total = align256(h.off_rec + (uint64_t)n_nodes * 32);
-
-    int *newidx = W.get<int>(n_nodes), *flag = W.get<int>(n_nodes + 1), *rank = W.get<int>(n_nodes + 1);
-    size_t sb2 = 0;
-    cub::DeviceScan::ExclusiveSum(nullptr, sb2, flag, rank, (int)n_nodes, s);
-    void *st2 = W.get<unsigned char>(sb2);
-    if (W.e) return W.e;
-    for (int l = -1; l < h.top_levels; ++l) {
-        flag_kernel<<<GN, 256, 0, s>>>(A.level, n_nodes, h.top_levels, l, flag);
-        size_t q = sb2;
-        if ((e = cub::DeviceScan::ExclusiveSum(st2, q, flag, rank, (int)n_nodes, s))) return e;
-        if (l < 0) assign_rest_kernel<<<GN, 256, 0, s>>>(A.level, rank, n_nodes, h.top_levels, h.top_count, newidx);
-        else assign_top_kernel<<<GN, 256, 0, s>>>(A.level, rank, n_nodes, l, h.level_prefix[l], newidx);
-    }
     void *blob = nullptr;
-    if ((e = cudaMalloc(&blob, h.total))) return e;
+    if ((e = alloc_blob(h, s, &blob))) return e;
     auto *base_b = static_cast<unsigned char *>(blob);
-    if ((e = cudaMemsetAsync(blob, 0, h.total, s)) ||
-        (e = cudaMemcpyAsync(blob, &h, sizeof(h), cudaMemcpyHostToDevice, s))) {
-        cudaFree(blob);
-        return e;
-    }
     auto *rec = reinterpret_cast<tt_oct_rec *>(base_b + h.off_rec);
     records_kernel<<<GN, 256, 0, s>>>(n_nodes, A, newidx, rec);
     leaf_fix_kernel<<<GN, 256, 0, s>>>(bodies, n_nodes, A, newidx, rec);

@@ -16,7 +16,7 @@
 #include <cstring>
 #include <vector>
 
-#include "kern_common.cuh"
+#include "build_common.cuh"
 
 namespace {
 
@@ -118,20 +118,6 @@ __global__ void vcount_fresh_kernel(long long n, const int *rstart, const unsign
         if (rstart[i] == i && fresh[i]) atomicAdd(flag, 1);
 }
 
-__global__ void vhist_kernel(const int *level, long long nn, unsigned *hist) {
-    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < nn; v += (long long)gridDim.x * blockDim.x)
-        atomicAdd(hist + level[v], 1u);
-}
-__global__ void vflag_kernel(const int *level, long long nn, int top_levels, int l, int *flag) {
-    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < nn; v += (long long)gridDim.x * blockDim.x)
-        flag[v] = l < 0 ? (level[v] >= top_levels) : (level[v] == l);
-}
-__global__ void vassign_kernel(const int *level, const int *rank, long long nn, int top_levels, int l, int offset,
-                               int *newidx) {
-    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < nn; v += (long long)gridDim.x * blockDim.x)
-        if (l < 0 ? level[v] >= top_levels : level[v] == l) newidx[v] = offset + rank[v];
-}
-
 __global__ void vp_records_kernel(long long nn, int D, int dp, const float *pts, int ld, VpOut o, const int *newidx,
                                   tt_vp_rec *rec, float *vpt, int *pid) {
     for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < nn; v += (long long)gridDim.x * blockDim.x) {
@@ -147,36 +133,12 @@ __global__ void vp_records_kernel(long long nn, int D, int dp, const float *pts,
     }
 }
 
-unsigned vgrid(long long n) {
-    long long g = (n + 255) / 256;
-    if (g > 148 * 8) g = 148 * 8;
-    return (unsigned)(g < 1 ? 1 : g);
-}
-
-inline uint64_t align256v(uint64_t x) { return (x + 255) & ~uint64_t(255); }
-
-struct VScratch {
-    cudaStream_t s;
-    cudaError_t e = cudaSuccess;
-    std::vector<void *> ptrs;
-    template <class T>
-    T *get(size_t count) {
-        void *p = nullptr;
-        if (e == cudaSuccess) e = cudaMallocAsync(&p, count * sizeof(T) + 16, s);
-        if (e == cudaSuccess) ptrs.push_back(p);
-        return static_cast<T *>(p);
-    }
-    ~VScratch() {
-        for (void *p : ptrs) cudaFreeAsync(p, s);
-    }
-};
-
 template <int DIM>
 int build_vp(const float *pts, long long n, int ld, cudaStream_t s, tt_blob_header *hdr_out, void **blob_out) {
     constexpr int D = DIM;
     tt_keep_pool_memory();
-    VScratch W{s};
-    const unsigned G = vgrid(n);
+    Scratch W{s};
+    const unsigned G = build_grid(n);
     int *ids = W.get<int>(n), *ids2 = W.get<int>(n);
     int *rstart = W.get<int>(n), *cnt = W.get<int>(n), *cnt2 = W.get<int>(n), *pre = W.get<int>(n),
         *pre2 = W.get<int>(n);
@@ -201,7 +163,6 @@ int build_vp(const float *pts, long long n, int ld, cudaStream_t s, tt_blob_head
     if (W.e) return W.e;
     cudaError_t e;
     vinit_kernel<<<G, 256, 0, s>>>(n, ids, rstart, cnt, pre, fresh);
-    int height = 0;
     for (int level = 0;; ++level) {
         for (int pass = 1; pass <= 2; ++pass) {
             vkey_kernel<DIM><<<G, 256, 0, s>>>(n, pass, pts, ld, ids, rstart, fresh, key);
@@ -219,68 +180,27 @@ int build_vp(const float *pts, long long n, int ld, cudaStream_t s, tt_blob_head
         int hf = 0;
         if ((e = cudaMemcpyAsync(&hf, flag, sizeof(int), cudaMemcpyDeviceToHost, s))) return e;
         if ((e = cudaStreamSynchronize(s))) return e;
-        height = level;
         if (!hf) break;
         if (level > TT_MAX_HEIGHT) return cudaErrorInvalidValue;
     }
     const int dp = (D + 3) & ~3;
-    unsigned *hist = W.get<unsigned>(64);
-    int *newidx = W.get<int>(nn), *fl = W.get<int>(nn + 1), *rank = W.get<int>(nn + 1);
-    size_t sb2 = 0;
-    cub::DeviceScan::ExclusiveSum(nullptr, sb2, fl, rank, (int)nn, s);
-    void *st2 = W.get<unsigned char>(sb2);
-    if (W.e) return W.e;
-    if ((e = cudaMemsetAsync(hist, 0, 64 * sizeof(unsigned), s))) return e;
-    vhist_kernel<<<G, 256, 0, s>>>(o.level, nn, hist);
-    unsigned hh[64];
-    if ((e = cudaMemcpyAsync(hh, hist, sizeof(hh), cudaMemcpyDeviceToHost, s))) return e;
-    if ((e = cudaStreamSynchronize(s))) return e;
     tt_blob_header h;
-    std::memset(&h, 0, sizeof(h));
-    h.magic = TT_BLOB_MAGIC;
-    h.version = TT_BLOB_VERSION;
-    h.kind = TT_KIND_VP;
-    h.dim = D;
-    h.dp = dp;
-    h.height = height;
-    h.leaf_size = 1;
-    h.n_nodes = nn;
-    h.n_points = n;
-    const int sbytes = 16 + 4 * dp;
-    long long acc = 0;
-    int Lv = 0;
-    h.level_prefix[0] = 0;
-    while (Lv <= height && Lv < TT_TOP_LEVELS_MAX && (acc + (long long)hh[Lv]) * sbytes <= TT_TOP_BYTES) {
-        acc += hh[Lv];
-        ++Lv;
-        h.level_prefix[Lv] = (int32_t)acc;
-    }
-    h.top_levels = Lv;
-    h.top_count = (int32_t)acc;
+    header_base(h, TT_KIND_VP, D, 1, nn, n);
     h.rec_bytes = 16;
-    uint64_t off = align256v(sizeof(tt_blob_header));
+    int *newidx = W.get<int>(nn);
+    if (W.e) return W.e;
+    if ((e = renumber_top_first(o.level, nn, 16 + 4 * dp, h, newidx, W))) return e;
+    uint64_t off = align256(sizeof(tt_blob_header));
     h.off_rec = off;
-    off = align256v(off + (uint64_t)nn * 16);
+    off = align256(off + (uint64_t)nn * 16);
     h.off_vpt = off;
-    off = align256v(off + (uint64_t)nn * dp * 4);
+    off = align256(off + (uint64_t)nn * dp * 4);
     h.off_pid = off;
-    off = align256v(off + (uint64_t)nn * 4);
+    off = align256(off + (uint64_t)nn * 4);
     h.total = off;
-    for (int l = -1; l < h.top_levels; ++l) {
-        vflag_kernel<<<G, 256, 0, s>>>(o.level, nn, h.top_levels, l, fl);
-        size_t q = sb2;
-        if ((e = cub::DeviceScan::ExclusiveSum(st2, q, fl, rank, (int)nn, s))) return e;
-        vassign_kernel<<<G, 256, 0, s>>>(o.level, rank, nn, h.top_levels, l, l < 0 ? h.top_count : h.level_prefix[l],
-                                          newidx);
-    }
     void *blob = nullptr;
-    if ((e = cudaMalloc(&blob, h.total))) return e;
+    if ((e = alloc_blob(h, s, &blob))) return e;
     auto *base = static_cast<unsigned char *>(blob);
-    if ((e = cudaMemsetAsync(blob, 0, h.total, s)) ||
-        (e = cudaMemcpyAsync(blob, &h, sizeof(h), cudaMemcpyHostToDevice, s))) {
-        cudaFree(blob);
-        return e;
-    }
     vp_records_kernel<<<G, 256, 0, s>>>(nn, D, dp, pts, ld, o, newidx, reinterpret_cast<tt_vp_rec *>(base + h.off_rec),
                                         reinterpret_cast<float *>(base + h.off_vpt),
                                         reinterpret_cast<int *>(base + h.off_pid));
