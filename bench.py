@@ -212,15 +212,19 @@ def load_counts(workload: str, mode: str):
         return None
 
 
-def libtt_sha256() -> str:
-    """Hash of libtt's sources and build script (nvcc output bytes are not
-    reproducible; the sources decide the instruction stream)."""
-    import glob
+KERNEL_SOURCE = {"bh": "kern_bh.cu", "pc": "kern_pc.cu", "knn": "kern_knn.cu", "vp": "kern_vp.cu"}
+
+
+def kernel_sha256(workload: str) -> str:
+    """Hash of the sources that decide the traversal kernel's instruction
+    stream for `workload` (its kern_*.cu, the shared device headers and the
+    build flags); nvcc output bytes themselves are not reproducible."""
     import hashlib
-    h = hashlib.sha256()
+    kind = workload.rstrip("0123456789m").replace("steps", "")  # bh16m -> bh, bhsteps -> bh
     pkg = os.path.join(ROOT, "paper_conf_sc_goldfarbjk13_b200")
-    files = sorted(glob.glob(os.path.join(pkg, "csrc", "*"))) + [os.path.join(pkg, "build.py"),
-                                                                  os.path.join(ROOT, "include", "tt.h")]
+    files = [os.path.join(pkg, "csrc", f) for f in (KERNEL_SOURCE[kind], "kern_common.cuh", "tt_internal.h")]
+    files.append(os.path.join(pkg, "build.py"))
+    h = hashlib.sha256()
     for f in files:
         h.update(os.path.basename(f).encode())
         h.update(open(f, "rb").read())
@@ -542,7 +546,7 @@ def run_ours(args, rank, world, local_rank):
     alg_bytes = visits * bpv + m * BYTES_PER_POINT_IO[name]  # per launch on rank 0
     achieved = alg_bytes / (kms / 1e3) / 1e9
     kernel_name = {"bh": "bh_kernel", "pc": "pc_kernel", "knn": "knn_kernel", "vp": "vp_kernel"}[name]
-    cnt = load_counts(name, args.mode) if not args.unsorted else None
+    cnt = load_counts(name, args.mode) if not args.unsorted and args.variant == "autoropes" else None
     clocks = clk.summary()
     sm_mhz = clocks.get("sm_mhz") or float(peaks.get("sm_max_mhz", 1965.0))
     nsm = torch.cuda.get_device_properties(device).multi_processor_count
@@ -561,18 +565,18 @@ def run_ours(args, rank, world, local_rank):
               "kernel_share_of_step": round(kms / ms, 4) if world == 1 else None,
               "traffic": int(cnt["dram_bytes_per_point"] * m) if cnt else None,
               "traffic_def": "ncu dram__bytes_read.sum + dram__bytes_write.sum per launch (scaled per point)"}
-    if cnt and cnt.get("so_sha256") == libtt_sha256():
+    if cnt and cnt.get("src_sha256") == kernel_sha256(name):
         inst = cnt["warp_inst_per_point"] * m
         issue_peak = nsm * 4 * sm_mhz * 1e6 / 1e9  # warp instructions per ns -> G/s
         roofline = {"bound": "issue", "achieved": round(inst / (kms / 1e3) / 1e9, 1), "peak": round(issue_peak, 1),
                     "unit": "Gwarp-inst/s", "frac": round(inst / (kms / 1e3) / 1e9 / issue_peak, 4),
                     "inst_per_launch": int(inst),
-                    "achieved_def": f"ncu smsp__inst_executed of this libtt.so ({cnt['round']}) / live kernel time",
+                    "achieved_def": f"ncu smsp__inst_executed of this kernel source ({cnt['round']}) / live kernel time",
                     "peak_def": f"{nsm} SMs x 4 schedulers x 1 warp-inst/clk x {sm_mhz:.0f} MHz (B200_PROFILING)",
                     **common, "hbm_effective": hbm_eff}
     else:
         roofline = {**hbm_eff, **common, "issue": None,
-                    "note": "no ncu instruction count for this libtt.so build: HBM-effective roofline only"}
+                    "note": "no ncu instruction count for this kernel source: HBM-effective roofline only"}
     cpu = None
     if world == 1 and not args.no_cpu_baseline:
         try:

@@ -11,13 +11,19 @@
 //   outside child: lb = r_out_min - d, sc = d + r_out_min
 // and the truncation test at pop is lb - tau > eps_vp * (sc + tau) with
 // tau = sqrt(best d2) (reading R12: conservative slack eps_vp = 2^-12).
-// A stack entry stores (parent << 1 | side) and the lane's distance d to the
-// parent's vantage point; (lb, sc) and the child index are recomputed at pop
-// from the parent's 16-B header with the same fp32 operations as at push, so
-// the arguments are bit-identical while an entry costs 8 B instead of 12.
-// N mode: lane-interleaved per-lane stacks in shared memory; L mode: per-warp
-// {parent|side, mask} stack plus per-lane d, majority vote on the call set
-// (§4.3, tie -> inside first).
+// (lb, sc) are recomputed at pop from the lane's distance d to the parent's
+// vantage point and the parent's radius on that side, with the same fp32
+// operations as at push, so the arguments are bit-identical while an entry
+// costs one float per lane:
+//   L mode: per-warp entries {child << 1 | side, radius, mask} (lane 0 owns
+//     them, pops are shuffled out) plus d[cap][32]; majority vote on the call
+//     set (§4.3, tie -> inside first).
+//   N mode, INDEPENDENT launches: per-lane {parent << 1 | side, d}; the child
+//     and radius come from the parent's 16-B header at pop.
+//   N mode inside an AUTO launch (rare warps): per-lane {parent << 1 | side}
+//     only; d is recomputed from the parent's vantage point at pop.
+// The narrow layout halves the shared-memory stack of AUTO/LOCKSTEP launches,
+// which the SM gives back to L1 for the (L2-resident) tree.
 #include "kern_common.cuh"
 
 namespace {
@@ -28,6 +34,11 @@ constexpr int kBlock = 256;
 constexpr int kWarps = kBlock / 32;
 constexpr int kSmemHdr = 128;
 #define TT_VP_EPS 0x1p-12f
+
+// shared-memory rope stack bytes of one warp (see the header comment)
+__host__ __device__ constexpr size_t vp_stack_bytes(int cap, bool wide) {
+    return wide ? (size_t)cap * 32 * 8 : (size_t)cap * (32 * 4 + 16);
+}
 
 // tau = sqrt_rn(best d2) is kept in a register, recomputed only when the
 // best improves (same value as recomputing it at every pop).
@@ -71,15 +82,14 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
 
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
-    // per-warp region of cap*32*8 bytes:
-    //   N: ent[cap][32] (parent<<1|side), d[cap][32]
-    //   L: d[cap][32], ent[cap], mask[cap]
-    unsigned char *wreg = s_stack + (size_t)warp * cap * 32 * 8;
+    const bool wide = P.c.mode == TT_MODE_INDEPENDENT;
+    // per-warp region (vp_stack_bytes): wide: ent[cap][32], d[cap][32];
+    // narrow: d (or N-mode ent)[cap][32], then int4 l_e[cap]
+    unsigned char *wreg = s_stack + (size_t)warp * vp_stack_bytes(cap, wide);
     int *n_ent = reinterpret_cast<int *>(wreg);
     float *n_d = reinterpret_cast<float *>(wreg + (size_t)cap * 32 * 4);
     float *l_d = reinterpret_cast<float *>(wreg);
-    int *l_ent = reinterpret_cast<int *>(wreg + (size_t)cap * 32 * 4);
-    unsigned *l_mask = reinterpret_cast<unsigned *>(l_ent + cap);
+    int4 *l_e = reinterpret_cast<int4 *>(wreg + (size_t)cap * 32 * 4);
     const unsigned char *s_hdr_base = s_rec;
     const unsigned char *g_hdr_base = reinterpret_cast<const unsigned char *>(g_rec);
     auto hdr = [&](int node) -> int4 {
@@ -152,7 +162,7 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
                     const int second = first_side ? t.x : t.y;
                     if (second != TT_END) {
                         n_ent[sp * 32 + lane] = (cur << 1) | (first_side ^ 1);
-                        n_d[sp * 32 + lane] = d;
+                        if (wide) n_d[sp * 32 + lane] = d;
                         ++sp;
                     }
                     const int first = child_args(t, first_side, d, lb, sc);
@@ -164,7 +174,16 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
                 if (sp > 0) {
                     --sp;
                     const int e = n_ent[sp * 32 + lane];
-                    cur = child_args(hdr(e >> 1), e & 1, n_d[sp * 32 + lane], lb, sc);
+                    float d;
+                    if (wide) {
+                        d = n_d[sp * 32 + lane];
+                    } else {  // same operands and operations as at push
+                        int4 tp;
+                        float v[DIM];
+                        ld_node<DIM>(s_rec, s_vpt, g_rec, g_vpt, DP, top, e >> 1, tp, v);
+                        d = __fsqrt_rn(pinned_d2<DIM>(q, v));
+                    }
+                    cur = child_args(hdr(e >> 1), e & 1, d, lb, sc);
                 } else {
                     cur = TT_END;
                 }
@@ -210,10 +229,8 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
                     const int first_side = 2 * votes >= __popc(act) ? 0 : 1;
                     const int second = first_side ? t.x : t.y;
                     if (second != TT_END) {
-                        if (lane == 0) {  // warp-uniform part of the entry
-                            l_ent[sp] = (cur << 1) | (first_side ^ 1);
-                            l_mask[sp] = act;
-                        }
+                        if (lane == 0)  // warp-uniform part: child|side, its radius, mask
+                            l_e[sp] = make_int4((second << 1) | (first_side ^ 1), first_side ? t.z : t.w, (int)act, 0);
                         l_d[sp * 32 + lane] = d;
                         ++sp;
                     }
@@ -227,15 +244,15 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
                 if (sp == 0) break;
                 --sp;
                 // lane 0 owns the warp-uniform part of the stack; broadcast its pop
-                int e0 = 0;
-                unsigned m0 = 0;
-                if (lane == 0) {
-                    e0 = l_ent[sp];
-                    m0 = l_mask[sp];
-                }
-                const int e = __shfl_sync(TT_FULL, e0, 0);
-                mask = __shfl_sync(TT_FULL, m0, 0);
-                cur = child_args(hdr(e >> 1), e & 1, l_d[sp * 32 + lane], lb, sc);
+                int4 e4 = make_int4(0, 0, 0, 0);
+                if (lane == 0) e4 = l_e[sp];
+                const int e = __shfl_sync(TT_FULL, e4.x, 0);
+                const float r = __int_as_float(__shfl_sync(TT_FULL, e4.y, 0));
+                mask = (unsigned)__shfl_sync(TT_FULL, e4.z, 0);
+                const float dd = l_d[sp * 32 + lane];
+                lb = (e & 1) ? __fsub_rn(r, dd) : __fsub_rn(dd, r);  // as child_args
+                sc = __fadd_rn(dd, r);
+                cur = e >> 1;
             }
         }
         if (valid) {
@@ -253,7 +270,8 @@ template <int DIM, bool STATS>
 int launch(const tt_vp_params &p, const tt_launch_cfg &cfg) {
     constexpr int DP = (DIM + 3) & ~3;
     const int cap = p.c.height + 2;
-    const size_t smem = kSmemHdr + (size_t)p.c.top_count * (16 + 4 * DP) + (size_t)kWarps * cap * 32 * 8;
+    const size_t smem = kSmemHdr + (size_t)p.c.top_count * (16 + 4 * DP) +
+                        (size_t)kWarps * vp_stack_bytes(cap, p.c.mode == TT_MODE_INDEPENDENT);
     auto kern = vp_kernel<DIM, STATS>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return (int)e;

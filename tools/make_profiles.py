@@ -51,7 +51,6 @@ def main(argv):
     counts = json.load(open(counts_path)) if os.path.exists(counts_path) else {}
     sys.path.insert(0, ROOT)
     import bench  # noqa: E402
-    so_sha = bench.libtt_sha256()  # sources of the build the captures ran
     for rep in sorted(glob.glob(os.path.join(ROOT, "gpurun_out", "prof_*.ncu-rep"))):
         tag = os.path.basename(rep)[len("prof_"):-len(".ncu-rep")]  # e.g. bh_auto
         w, mode = tag.split("_", 1)
@@ -89,7 +88,7 @@ def main(argv):
                     "dram_bytes_per_point": (rb * scale + (wb or 0) * scale_w) / pts,
                     "warp_inst_per_point": inst / pts,
                     "ncu_duration": dur, "issue_slots_busy_pct": num("Issue Slots Busy"),
-                    "so_sha256": so_sha,
+                    "src_sha256": bench.kernel_sha256(w),
                 }
         open(os.path.join(outdir, f"ncu_{tag}.md"), "w").write("\n".join(lines) + "\n")
     lb = os.path.join(ROOT, "gpurun_out", "launches_bh.csv")
