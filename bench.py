@@ -55,6 +55,8 @@ def parse():
                          "bhsteps: full BH time steps (GPU build + sort + force + leapfrog), 1 GPU")
     ap.add_argument("--mode", default="auto", choices=["auto", "lockstep", "independent"])
     ap.add_argument("--unsorted", action="store_true", help="skip tt_sort_points (paper's 'unsorted' column)")
+    ap.add_argument("--no-schedule", action="store_true",
+                    help="skip tt_schedule_tiles (longest-first tile order after the sort; kd/vp trees)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--points-per-rank", type=int, default=0, help="override M (testing)")
@@ -414,9 +416,14 @@ def run_ours(args, rank, world, local_rank):
     if args.unsorted:
         order_buf.copy_(torch.arange(m, dtype=torch.int32, device=device))
 
+    # a1b pays only when there are more tiles than resident warps (148 SMs x 32)
+    lpt = not args.unsorted and not args.no_schedule and tree.kind != "oct" and m // 32 > 148 * 32
+
     def step(kev=None, collective=True):
         if not args.unsorted:
             P.tt_sort_points(tree, q_shard, out=order_buf)  # a1
+            if lpt:
+                P.tt_schedule_tiles(tree, q_shard, order_buf, out=order_buf)  # a1b
         if kev:
             kev[0].record(stream)
         traverse(q_shard, out_shard, order_buf)            # a2-a5
@@ -430,6 +437,8 @@ def run_ours(args, rank, world, local_rank):
     # stats pass (untimed): per-point useful visits, warp fetches, modes
     if not args.unsorted:
         P.tt_sort_points(tree, q_shard, out=order_buf)
+        if lpt:
+            P.tt_schedule_tiles(tree, q_shard, order_buf, out=order_buf)
     st = P.Stats.alloc(m, device)
     traverse(q_shard, out_shard, order_buf, st)
     torch.cuda.synchronize()
@@ -497,6 +506,8 @@ def run_ours(args, rank, world, local_rank):
         def e2e_step():
             q_dev.copy_(q_host, non_blocking=True)
             P.tt_sort_points(tree, q_dev, out=perm)
+            if lpt:
+                P.tt_schedule_tiles(tree, q_dev, perm, out=perm)
             if name == "bh":
                 P.tt_traverse_bh(tree, q_dev, c["theta"], c["eps"], out=res_dev, order=perm, mode=args.mode,
                                  self_ids=self_ids)
@@ -530,7 +541,7 @@ def run_ours(args, rank, world, local_rank):
         d2h = sum(r.numel() * r.element_size() for r in (res_host if isinstance(res_host, tuple) else (res_host,)))
         e2e = {"value": n_all / (ems / 1e3), "unit": "points/s", "ms_per_step": ems,
                "h2d_bytes_per_step": int(q_host.numel() * q_host.element_size()), "d2h_bytes_per_step": int(d2h),
-               "note": "public API (tt_sort_points + tt_traverse_*) on pinned host buffers; H2D, D2H inside"}
+               "note": "public API (tt_sort_points + tt_schedule_tiles + tt_traverse_*) on pinned host buffers; H2D, D2H inside"}
 
     # keep the GPU busy until the sampler has seen the load (>= 5 samples)
     t_soak = time.perf_counter()
@@ -591,6 +602,7 @@ def run_ours(args, rank, world, local_rank):
         "vs_baseline": None, "dtype": "f32", "data": "synthetic",
         "config": {"workload": w["workload"], "points_per_rank": m, "global_points": n_all,
                    "tree_points": w["n_data"], "mode": args.mode, "sorted": not args.unsorted,
+                   "tile_schedule": "longest-first" if lpt else "in-order",
                    "auto_min_depth": args.auto_min_depth, "variant": args.variant,
                    "parallelism": f"dp{world} (points sharded, tree replicated)",
                    "l2": "flushed between timed steps (512 MiB write)",

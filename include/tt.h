@@ -193,6 +193,22 @@ tt_status tt_tree_get_info(const tt_tree *t, tt_tree_info *out);
 tt_status tt_sort_points(const tt_tree *t, const float *pts, int64_t n, int32_t ld,
                          uint32_t *perm_out, uint64_t *keys_out, tt_stream s);
 
+/* a1b: longest-first tile schedule (Graham's LPT rule over
+ * the persistent kernels' warp tiles).  Reorders whole tiles of perm_in --
+ * T consecutive entries, T = 32 for kd/vp trees (the kNN, PC and VP kernels'
+ * tile) -- so that tiles with the largest estimated traversal cost come
+ * first; the entries inside a tile and the ragged last tile (n mod T) keep
+ * their places, and equal estimates keep their order.  Estimate per point,
+ * from one greedy descent: kd -> largest pinned d2 to the points of the leaf
+ * the split rule reaches; vp -> smallest distance to a vantage point on the
+ * inside-iff-d<=r_in path; tile = the largest over its points.  Oct trees:
+ * a plain copy (BH tiles are near-uniform, §4.6).  Traversal results never
+ * depend on the order, only the schedule does.  pts: device, n rows of `ld`
+ * floats (the points perm_in indexes); perm_in/perm_out: device [n], may be
+ * the same buffer.  Temporary device memory is stream-ordered.            */
+tt_status tt_schedule_tiles(const tt_tree *t, const float *pts, int64_t n, int32_t ld,
+                            const uint32_t *perm_in, uint32_t *perm_out, tt_stream s);
+
 /* ------------------------------------------------------------------------ */
 /* a2-a6: traversal launch options (all optional; pass NULL for defaults).  */
 typedef struct tt_stats {

@@ -88,6 +88,7 @@ SIGNATURES = {
     "tt_tree_free": (I32, [P]),
     "tt_tree_get_info": (I32, [P, P]),
     "tt_sort_points": (I32, [P, P, I64, I32, P, P, P]),
+    "tt_schedule_tiles": (I32, [P, P, I64, I32, P, P, P]),
     "tt_traverse_bh": (I32, [P, P, P, I64, F, F, P, P, P]),
     "tt_traverse_pc": (I32, [P, P, I64, I32, F, P, P, P]),
     "tt_traverse_knn": (I32, [P, P, I64, I32, I32, P, P, P, P]),

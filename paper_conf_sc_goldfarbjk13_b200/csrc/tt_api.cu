@@ -6,6 +6,7 @@
 #include <atomic>
 #include <limits>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 
@@ -51,6 +52,7 @@ tt_status setup_common(const tt_tree *t, int kind, int64_t n, const tt_traverse_
     if (n < 0 || n > (int64_t)0xffffffffu * 32) return TT_ERR_INVALID_ARG;
     std::memset(&c, 0, sizeof(c));
     c.tree = t->dev;
+    if (const char *ev = std::getenv("TT_STAGE_BYTES")) stage_budget = std::atoi(ev);  // tuning sweeps only
     c.top_count = tt_stage_count(t->hdr, stage_bytes_per_node, stage_budget);
     c.height = t->hdr.height;
     c.n = n;
@@ -295,6 +297,20 @@ tt_status tt_sort_points(const tt_tree *t, const float *pts, int64_t n, int32_t 
     tt_status st = have_device();
     if (st != TT_OK) return st;
     int e = tt_launch_sort(t, pts, n, ld, perm_out, keys_out, s);
+    return e ? cuda_fail((cudaError_t)e) : TT_OK;
+}
+
+tt_status tt_schedule_tiles(const tt_tree *t, const float *pts, int64_t n, int32_t ld, const uint32_t *perm_in,
+                            uint32_t *perm_out, tt_stream s) {
+    if (!t || n < 0 || n > INT32_MAX) return TT_ERR_INVALID_ARG;
+    if (n == 0) return TT_OK;
+    if (!pts || !perm_in || !perm_out) return TT_ERR_INVALID_ARG;
+    if (ld < (t->hdr.kind == TT_KIND_OCT ? 3 : t->hdr.dim)) return TT_ERR_INVALID_ARG;
+    if (t->hdr.kind != TT_KIND_OCT && !dim_supported(t->hdr.dim)) return TT_ERR_UNSUPPORTED;
+    tt_status st = have_device();
+    if (st != TT_OK) return st;
+    const int tile = t->hdr.kind == TT_KIND_OCT ? 32 * TT_BH_POINTS_PER_LANE : 32;
+    int e = tt_launch_schedule(t, pts, n, ld, perm_in, perm_out, tile, s);
     return e ? cuda_fail((cudaError_t)e) : TT_OK;
 }
 

@@ -151,6 +151,8 @@ int tt_launch_knn_recursive(const tt_knn_params &p, int dim, const tt_launch_cfg
 int tt_launch_vp_recursive(const tt_vp_params &p, int dim, const tt_launch_cfg &cfg);
 int tt_launch_sort(const tt_tree *t, const float *pts, int64_t n, int32_t ld, uint32_t *perm,
                    uint64_t *keys_out, void *stream);
+int tt_launch_schedule(const tt_tree *t, const float *pts, int64_t n, int32_t ld, const uint32_t *perm_in,
+                       uint32_t *perm_out, int tile, void *stream);
 
 // Nodes of the largest level-complete top prefix whose staged bytes fit `budget`.
 inline int tt_stage_count(const tt_blob_header &h, int bytes_per_node, int budget) {

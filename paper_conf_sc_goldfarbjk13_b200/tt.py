@@ -24,7 +24,7 @@ __all__ = [
     "HostTree", "Tree", "Stats", "TTError",
     "build_kd", "build_oct", "build_vp", "tt_tree_pack", "tt_tree_from_blob", "tt_tree_upload",
     "tt_build_oct_device", "tt_build_kd_device", "tt_build_vp_device", "tt_tree_download",
-    "tt_sort_points", "tt_traverse_bh", "tt_traverse_pc", "tt_traverse_knn", "tt_traverse_vp",
+    "tt_sort_points", "tt_schedule_tiles", "tt_traverse_bh", "tt_traverse_pc", "tt_traverse_knn", "tt_traverse_vp",
     "build_info",
 ]
 
@@ -291,6 +291,23 @@ def tt_sort_points(tree: Tree, pts: torch.Tensor, out: torch.Tensor | None = Non
         kp = keys.data_ptr()
     check(L.load().tt_sort_points(tree._h, pts.data_ptr(), n, pts.stride(0), out.data_ptr(), kp,
                                   C.c_void_p(_stream_handle(stream))), "tt_sort_points")
+    return out
+
+
+def tt_schedule_tiles(tree: Tree, pts: torch.Tensor, perm: torch.Tensor, out: torch.Tensor | None = None,
+                      stream=None) -> torch.Tensor:
+    """a1b: `perm` with whole warp tiles reordered longest-estimated-first
+    (include/tt.h).  out may be perm itself (in place)."""
+    _dev(pts, torch.float32, "pts", 3 if tree.kind == "oct" else tree.dim)
+    _dev(perm, torch.int32, "perm")
+    n = perm.numel()
+    if out is None:
+        out = torch.empty_like(perm)
+    _dev(out, torch.int32, "out")
+    if out.numel() != n:
+        raise ValueError("out must have perm's length")
+    check(L.load().tt_schedule_tiles(tree._h, pts.data_ptr(), n, pts.stride(0), perm.data_ptr(), out.data_ptr(),
+                                     C.c_void_p(_stream_handle(stream))), "tt_schedule_tiles")
     return out
 
 

@@ -279,6 +279,92 @@ def test_vp_config4_full_size_sampled():
 
 
 # ---------------------------------------------------------------------- sort
+def _pinned_d2(q, p):
+    """fp32 sequential squared distance, one rounding per operation (R0)."""
+    t = (q[..., 0] - p[..., 0]).astype(np.float32)
+    s = (t * t).astype(np.float32)
+    for d in range(1, q.shape[-1]):
+        t = (q[..., d] - p[..., d]).astype(np.float32)
+        s = (s + (t * t).astype(np.float32)).astype(np.float32)
+    return s
+
+
+def _tiles(a, T):
+    nfull = len(a) // T
+    return [tuple(a[i * T:(i + 1) * T]) for i in range(nfull)], a[nfull * T:]
+
+
+def _check_tile_permutation(perm, sched, T):
+    tp, tail_p = _tiles(perm, T)
+    ts, tail_s = _tiles(sched, T)
+    assert np.array_equal(tail_p, tail_s)  # ragged last tile stays last
+    assert sorted(tp) == sorted(ts)        # whole tiles move, contents untouched
+    return tp, ts
+
+
+def test_schedule_tiles_kd_longest_first(knn_small):
+    """a1b on a kd tree: whole tiles reordered by the estimate recomputed here
+    (leaf by the split rule, largest pinned d2 to its points), non-increasing,
+    ties in point-sort order."""
+    p, q, ot, tree = knn_small
+    qd = dev(q)
+    perm = P.tt_sort_points(tree, qd)
+    sched = P.tt_schedule_tiles(tree, qd, perm).cpu().numpy()
+    perm = perm.cpu().numpy()
+    tp, ts = _check_tile_permutation(perm, sched, 32)
+    sd, sp = ot.i64(oracle.F_SPLITDIM), ot.f32(oracle.F_SPLIT)
+    ch, pb, pc = ot.children(), ot.i64(oracle.F_PBEGIN), ot.i64(oracle.F_PCOUNT)
+    tpts = p[ot.tree_order()]
+    cur = np.zeros(len(q), np.int64)
+    for _ in range(ot.height + 1):
+        inner = ch[cur, 0] >= 0
+        x = q[np.arange(len(q)), np.maximum(sd[cur], 0)]
+        cur = np.where(inner, np.where(x < sp[cur], ch[cur, 0], ch[cur, 1]), cur)
+    est = np.zeros(len(q), np.float32)
+    for j in range(int(pc.max())):
+        has = j < pc[cur]
+        d2 = _pinned_d2(q, tpts[pb[cur] + np.minimum(j, pc[cur] - 1)])
+        est = np.where(has, np.maximum(est, d2), est)
+    key = {t: est[list(t)].max() for t in tp}
+    ks = np.array([key[t] for t in ts])
+    assert np.all(ks[:-1] >= ks[1:])
+    pos = {t: i for i, t in enumerate(tp)}
+    for a, b in zip(ts[:-1], ts[1:]):  # stable among equal estimates
+        if key[a] == key[b]:
+            assert pos[a] < pos[b]
+
+
+def test_schedule_tiles_results_unchanged(knn_small, vp_small):
+    """Traversal results do not depend on the tile schedule (kNN, VP; in-place
+    call; oct trees get a copy)."""
+    p, q, ot, tree = knn_small
+    qd = dev(q)
+    perm = P.tt_sort_points(tree, qd)
+    sched = P.tt_schedule_tiles(tree, qd, perm.clone())
+    again = perm.clone()
+    P.tt_schedule_tiles(tree, qd, again, out=again)
+    assert torch.equal(sched, again)
+    assert not torch.equal(sched, perm)
+    for mode in MODES:
+        a = P.tt_traverse_knn(tree, qd, 8, order=perm, mode=mode)
+        b = P.tt_traverse_knn(tree, qd, 8, order=sched, mode=mode)
+        assert torch.equal(a[0], b[0]) and torch.equal(a[1], b[1])
+    p, q, ot, tree = vp_small
+    qd = dev(q)
+    perm = P.tt_sort_points(tree, qd)
+    sched = P.tt_schedule_tiles(tree, qd, perm)
+    _check_tile_permutation(perm.cpu().numpy(), sched.cpu().numpy(), 32)
+    for mode in MODES:
+        a = P.tt_traverse_vp(tree, qd, order=perm, mode=mode)
+        b = P.tt_traverse_vp(tree, qd, order=sched, mode=mode)
+        assert torch.equal(a[0], b[0]) and torch.equal(a[1], b[1])
+    b = ttgen.plummer(3000, seed=214)
+    t_oct = P.tt_tree_upload(P.build_oct(b))
+    bd = dev(b)
+    perm = P.tt_sort_points(t_oct, bd)
+    assert torch.equal(P.tt_schedule_tiles(t_oct, bd, perm), perm)
+
+
 def test_sort_points_matches_oracle_for_every_kind():
     b = ttgen.plummer(30000, seed=210)
     p7 = ttgen.gaussian_mixture(30000, 7, seed=211, components=8)
