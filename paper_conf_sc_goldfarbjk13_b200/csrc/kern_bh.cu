@@ -163,6 +163,24 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
 
         unsigned fetches = 0, steps = 0;
         if (lock) {
+            // The warp's two bodies per lane run as one FP32x2 pair: every
+            // per-body operation of a step (differences, squares, the pinned
+            // sum, the softened inverse cube, the accumulation) is one packed
+            // FADD2 / FMUL2 / FFMA2 for both bodies, each half rounded exactly
+            // like the scalar op (rn(g - b) = rn(g + (-b)): negation is exact),
+            // so results are bit-identical to the scalar form.
+            static_assert(kBPL == 2, "packed lockstep loop is written for body pairs");
+            // negated coordinate pairs, formed once per tile: rn(-0 + (-b)) = -b
+            // exactly; the opaque -0 addend keeps ptxas from folding this into a
+            // negate modifier that re-assembles the pairs every step
+            const float nz = opaque_neg_zero(n);  // -0, see sqr2_rn
+            const float2 nz2 = make_float2(nz, nz);
+            const float2 nbx = add2_rn(nz2, make_float2(-bd[0].b.x, -bd[1].b.x));
+            const float2 nby = add2_rn(nz2, make_float2(-bd[0].b.y, -bd[1].b.y));
+            const float2 nbz = add2_rn(nz2, make_float2(-bd[0].b.z, -bd[1].b.z));
+            const int self0 = bd[0].self, self1 = bd[1].self;
+            int w0 = bd[0].wait, w1 = bd[1].wait;
+            float2 ax = make_float2(0.f, 0.f), ay = ax, az = ax;
             int cur = 0;
             // kernel parameters pinned in registers for the hot loop (otherwise
             // re-read from the constant bank every iteration)
@@ -170,6 +188,7 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
             int dbits = dsq_bits;
             float e2 = eps2;
             asm volatile("" : "+l"(grec), "+r"(dbits), "+f"(e2));
+            const float2 e22 = make_float2(e2, e2);
             for (;;) {
 #pragma unroll 1
                 for (int k = 0; k < kFlush; ++k) {
@@ -181,37 +200,42 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
                     if (STATS) ++steps;
                     const int lvl = t.w;
                     const float dl = EXP_DSQ ? dsq_at(dbits, lvl) : s_dsq[lvl];
-                    bool any_open = false;
-#pragma unroll
-                    for (int j = 0; j < kBPL; ++j) {
-                        const bool active = lvl <= bd[j].wait;
-                        float dx, dy, sx, sy;
-                        sub2_rn(g.x, g.y, bd[j].b.x, bd[j].b.y, dx, dy);
-                        sqr2_rn(dx, dy, sx, sy);
-                        const float dz = __fsub_rn(g.z, bd[j].b.z);
-                        const float drsq = __fadd_rn(__fadd_rn(sx, sy), __fmul_rn(dz, dz));
-                        const bool open = active && t.x >= 0 && drsq < dl;
-                        if (STATS) bd[j].visits += active;
-                        bd[j].wait = active ? (open ? INT_MAX : lvl) : bd[j].wait;
-                        // branch-free update: in a warp step some lane almost always
-                        // interacts, so predication beats a divergent branch; the
-                        // three conditions fold into one LOP3 + one select
-                        const unsigned inter = (unsigned)active & (unsigned)!open & (unsigned)(t.z != bd[j].self);
-                        const float inv = rsqrt_ftz(__fadd_rn(drsq, e2));
-                        float mw;
-                        asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %1, 0;\n\tselp.f32 %0, %2, 0f00000000, p;\n\t}"
-                            : "=f"(mw) : "r"(inter), "f"(g.w));
-                        const float f = mw * (inv * inv) * inv;
-                        bd[j].acc.x = fmaf(f, dx, bd[j].acc.x);
-                        bd[j].acc.y = fmaf(f, dy, bd[j].acc.y);
-                        bd[j].acc.z = fmaf(f, dz, bd[j].acc.z);
-                        any_open |= open;
+                    const float2 dx = add2_rn(make_float2(g.x, g.x), nbx);
+                    const float2 dy = add2_rn(make_float2(g.y, g.y), nby);
+                    const float2 dz = add2_rn(make_float2(g.z, g.z), nbz);
+                    // rn(rn(rn(dx^2) + rn(dy^2)) + rn(dz^2)): the pinned order (R0)
+                    const float2 drsq = add2_rn(add2_rn(sqr2_rn(dx, nz), sqr2_rn(dy, nz)), sqr2_rn(dz, nz));
+                    const bool a0 = lvl <= w0, a1 = lvl <= w1;
+                    const bool cell = t.x >= 0;
+                    const bool o0 = a0 && cell && drsq.x < dl;
+                    const bool o1 = a1 && cell && drsq.y < dl;
+                    if (STATS) {
+                        bd[0].visits += a0;
+                        bd[1].visits += a1;
                     }
-                    cur = __any_sync(TT_FULL, any_open) ? t.x : t.y;
+                    // active ? (open ? follow : wait at lvl) : keep -- as a min
+                    // (an inactive lane has lvl > wait)
+                    w0 = o0 ? INT_MAX : min(w0, lvl);
+                    w1 = o1 ? INT_MAX : min(w1, lvl);
+                    // branch-free update (some lane almost always interacts)
+                    const float2 mw = make_float2(a0 && !o0 && t.z != self0 ? g.w : 0.f, a1 && !o1 && t.z != self1 ? g.w : 0.f);
+                    const float2 r = add2_rn(drsq, e22);
+                    const float2 inv = make_float2(rsqrt_ftz(r.x), rsqrt_ftz(r.y));
+                    const float2 f = mul2_rn(mul2_rn(mw, mul2_rn(inv, inv)), inv);
+                    ax = fma2_rn(f, dx, ax);
+                    ay = fma2_rn(f, dy, ay);
+                    az = fma2_rn(f, dz, az);
+                    cur = __any_sync(TT_FULL, o0 || o1) ? t.x : t.y;
                     if (cur == TT_END) break;
                 }
-#pragma unroll
-                for (int j = 0; j < kBPL; ++j) bd[j].acc.flush();  // warp-uniform
+                // fp32 partials -> fp64 (warp-uniform cadence)
+                bd[0].acc.X += (double)ax.x;
+                bd[0].acc.Y += (double)ay.x;
+                bd[0].acc.Z += (double)az.x;
+                bd[1].acc.X += (double)ax.y;
+                bd[1].acc.Y += (double)ay.y;
+                bd[1].acc.Z += (double)az.y;
+                ax = ay = az = make_float2(0.f, 0.f);
                 if (cur == TT_END) break;
             }
             fetches = steps;

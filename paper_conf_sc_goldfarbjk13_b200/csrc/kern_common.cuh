@@ -108,6 +108,44 @@ __device__ __forceinline__ void sqr2_rn(float a0, float a1, float &r0, float &r1
         : "f"(a0), "f"(a1));
 }
 
+// Packed FP32x2 pair ops on float2: one FADD2 / FMUL2 / FFMA2, each half
+// rounded exactly like the scalar op.
+__device__ __forceinline__ float2 add2_rn(float2 a, float2 b) {
+    float2 r;
+    asm("{\n\t.reg .b64 x, y, z;\n\tmov.b64 x, {%2, %3};\n\tmov.b64 y, {%4, %5};\n\t"
+        "add.rn.f32x2 z, x, y;\n\tmov.b64 {%0, %1}, z;\n\t}"
+        : "=f"(r.x), "=f"(r.y)
+        : "f"(a.x), "f"(a.y), "f"(b.x), "f"(b.y));
+    return r;
+}
+__device__ __forceinline__ float2 mul2_rn(float2 a, float2 b) {
+    float2 r;
+    asm("{\n\t.reg .b64 x, y, z;\n\tmov.b64 x, {%2, %3};\n\tmov.b64 y, {%4, %5};\n\t"
+        "mul.rn.f32x2 z, x, y;\n\tmov.b64 {%0, %1}, z;\n\t}"
+        : "=f"(r.x), "=f"(r.y)
+        : "f"(a.x), "f"(a.y), "f"(b.x), "f"(b.y));
+    return r;
+}
+__device__ __forceinline__ float2 fma2_rn(float2 a, float2 b, float2 c) {
+    float2 r;
+    asm("{\n\t.reg .b64 x, y, w, z;\n\tmov.b64 x, {%2, %3};\n\tmov.b64 y, {%4, %5};\n\t"
+        "mov.b64 w, {%6, %7};\n\tfma.rn.f32x2 z, x, y, w;\n\tmov.b64 {%0, %1}, z;\n\t}"
+        : "=f"(r.x), "=f"(r.y)
+        : "f"(a.x), "f"(a.y), "f"(b.x), "f"(b.y), "f"(c.x), "f"(c.y));
+    return r;
+}
+
+// rn(a*a) as fma.rn(a, a, z) with z = -0: exactly rn(a*a) (adding -0 changes
+// nothing, +0 stays +0), and an FFMA2 result is never fused into the following
+// add.  ptxas fuses mul.rn.f32x2 into a dependent add.rn.f32x2 despite the
+// explicit rounding (seen in SASS, also with --fmad=false), and it folds a
+// literal -0 addend back into a multiply -- so z must be a value it cannot
+// prove is -0: callers pass opaque_neg_zero(), derived from a kernel parameter.
+__device__ __forceinline__ float2 sqr2_rn(float2 a, float z) { return fma2_rn(a, a, make_float2(z, z)); }
+__device__ __forceinline__ float opaque_neg_zero(long long never_negative) {
+    return __int_as_float((int)(0x80000000u | (unsigned)(never_negative < 0)));
+}
+
 // max(a, b, c) in one FMNMX3 (sm_100 three-input min/max)
 __device__ __forceinline__ float max3(float a, float b, float c) {
     float r;
