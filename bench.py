@@ -52,7 +52,7 @@ def parse():
     ap.add_argument("--workload", choices=["bh", "knn", "vp", "pc", "bh16m", "knn16m", "bhsteps"], default="bh",
                     help="bh/knn/vp/pc: configs[0..3] (weak scaling, M points per rank); "
                          "bh16m/knn16m: configs[4] (16M points split over the ranks, strong scaling); "
-                         "bhsteps: full BH time steps (GPU build + sort + force + leapfrog), 1 GPU")
+                         "bhsteps: full BH time steps (GPU build + sort + force + leapfrog), bodies sharded over the ranks (strong scaling)")
     ap.add_argument("--mode", default="auto", choices=["auto", "lockstep", "independent"])
     ap.add_argument("--unsorted", action="store_true", help="skip tt_sort_points (paper's 'unsorted' column)")
     ap.add_argument("--no-schedule", action="store_true",
@@ -136,6 +136,12 @@ class ClockSampler:
                  "-i", str(self.gpu)], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
+            # nvidia-smi's start-up (NVML init) takes driver locks that stall
+            # this process's CUDA API calls: let it reach its first sample
+            # before the caller starts the timed region
+            t0 = time.time()
+            while not self.lines and self.proc.poll() is None and time.time() - t0 < 10:
+                time.sleep(0.01)
         except OSError:
             self.proc = None
         return self
@@ -298,37 +304,53 @@ def run_reference(args, rank, world):
 
 
 # ------------------------------------------------------------------- ours
-def run_bh_steps(args):
-    """NEXT-4 workload: a bench step = one BH time step of configs[1] on one GPU
-    (tt_build_oct_device + tt_sort_points + tt_traverse_bh + tt_kick_drift)."""
+def run_bh_steps(args, rank, world):
+    """NEXT-4 workload: a bench step = one BH time step of configs[1]
+    (tt_build_oct_device + tt_sort_points + tt_traverse_bh + tt_kick_drift_permuted,
+    + all-gather of positions / velocities / ids for N > 1).  Strong scaling:
+    the same 1M-body system on every N; each rank integrates its warp-aligned
+    shard of the sorted order (nbody.simulate_sharded)."""
     import torch
+    import torch.distributed as dist
     from paper_conf_sc_goldfarbjk13_b200 import nbody
+    from paper_conf_sc_goldfarbjk13_b200 import parallel as PAR
     c = dict(ttgen.CONFIGS["bh_1m_plummer"])
     n = args.points_per_rank or c["n"]
+    n = -(-n // (64 * world)) * (64 * world)  # equal warp-aligned shards
     b = ttgen.plummer(n, c["seed"])
     v = ttgen.plummer_velocities(b, c["seed"] + 1000)
-    B = torch.from_numpy(b).cuda()
-    V = torch.from_numpy(v).cuda()
+    dev = torch.device("cuda", torch.cuda.current_device())
+    B, V = torch.from_numpy(b).to(dev), torch.from_numpy(v).to(dev)
+    ids = torch.arange(n, dtype=torch.int32, device=dev)
     dt = 1e-3
-    acc, _ = nbody.forces(B, c["theta"], c["eps"])
     for _ in range(args.warmup):
-        acc = nbody.simulate(B, V, 1, dt, c["theta"], c["eps"], acc=acc)
+        B, V, ids = nbody.simulate_sharded(B, V, ids, 1, dt, c["theta"], c["eps"], final_kick=False)
     torch.cuda.synchronize()
     stream = torch.cuda.current_stream()
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    with ClockSampler(0) as clk:
+    if world > 1:
+        dist.barrier()
+    with ClockSampler(torch.cuda.current_device()) as clk:
         for i in range(args.steps):
             evs[i][0].record(stream)
-            acc = nbody.simulate(B, V, 1, dt, c["theta"], c["eps"], acc=acc)
+            B, V, ids = nbody.simulate_sharded(B, V, ids, 1, dt, c["theta"], c["eps"], final_kick=False)
             evs[i][1].record(stream)
         torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
     ms = statistics.mean(a.elapsed_time(b_) for a, b_ in evs)
-    line = {"metric": METRIC, "value": n / (ms / 1e3), "unit": "points/s (body-steps/s)", "n_gpus": 1,
+    if world > 1:
+        ms = PAR.max_over_ranks(ms, dev)
+    if rank != 0:
+        return
+    line = {"metric": METRIC, "value": n / (ms / 1e3), "unit": "points/s (body-steps/s)", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": "bh_1m_plummer time steps", "bodies": n, "dt": dt,
-                       "step": "GPU build + sort + force + kick-drift (leapfrog KDK)", "params": c,
-                       "l2": "not flushed: a time step rewrites the bodies and rebuilds the tree"},
+                       "step": "GPU build + sort + force (own shard) + gathered kick-drift (leapfrog KDK)"
+                               + (" + all-gather of x, v, ids" if world > 1 else ""),
+                       "parallelism": f"dp{world} (bodies sharded by sorted order, tree rebuilt on every rank)",
+                       "params": c, "l2": "not flushed: a time step rewrites the bodies and rebuilds the tree"},
             "clocks": clk.summary()}
     print(json.dumps(line), flush=True)
 
@@ -634,10 +656,6 @@ def main():
     if args.impl == "reference":
         run_reference(args, rank, world)
         return
-    if args.workload == "bhsteps":
-        if rank == 0:
-            run_bh_steps(args)
-        return
     if world > 1:
         import torch
         import torch.distributed as dist
@@ -649,7 +667,10 @@ def main():
         else:
             dist.init_process_group(backend)
     try:
-        run_ours(args, rank, world, local_rank)
+        if args.workload == "bhsteps":
+            run_bh_steps(args, rank, world)
+        else:
+            run_ours(args, rank, world, local_rank)
     finally:
         if world > 1:
             import torch.distributed as dist

@@ -282,6 +282,20 @@ tt_status tt_traverse_vp(const tt_tree *t, const float *q, int64_t n, int32_t ld
 tt_status tt_kick_drift(float *bodies, float *vel, const float *acc, int64_t n, float dt_kick, float dt_drift,
                         tt_stream s);
 
+/* NEXT-4, sharded time step: the same update, gathered
+ * through a permutation: for j < n, with i = perm[j],
+ *   vel_out[j]    = vel[i] + acc[i] * dt_kick      (x, y, z; w copied)
+ *   bodies_out[j] = bodies[i] + vel_out[j] * dt_drift (x, y, z; mass copied)
+ *   ids_out[j]    = ids[i]                           (if ids != NULL)
+ * perm is typically a contiguous slice of tt_sort_points' permutation, so a
+ * rank's shard of the sorted order is written contiguously and the bodies
+ * travel in sorted order.  Inputs and outputs are device float4 rows (16-B
+ * aligned) and must not overlap; perm entries index the input rows and are
+ * not range-checked (caller's contract).  Asynchronous on `s`.            */
+tt_status tt_kick_drift_permuted(const float *bodies, const float *vel, const float *acc, const int32_t *perm,
+                                 const int32_t *ids, int64_t n, float dt_kick, float dt_drift, float *bodies_out,
+                                 float *vel_out, int32_t *ids_out, tt_stream s);
+
 /* ------------------------------------------------------------------------ */
 const char *tt_status_string(tt_status s);
 /* Last CUDA error code seen by the library (cudaError_t as int), 0 if none. */

@@ -13,6 +13,6 @@ _lib.load()
 from . import tt  # noqa: E402
 from .tt import *  # noqa: E402,F401,F403
 from . import nbody  # noqa: E402
-from .nbody import tt_kick_drift  # noqa: E402,F401
+from .nbody import tt_kick_drift, tt_kick_drift_permuted  # noqa: E402,F401
 
-__all__ = ["tt", "nbody", "TTError", "tt_kick_drift"] + list(tt.__all__)
+__all__ = ["tt", "nbody", "TTError", "tt_kick_drift", "tt_kick_drift_permuted"] + list(tt.__all__)

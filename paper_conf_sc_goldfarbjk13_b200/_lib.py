@@ -85,6 +85,7 @@ SIGNATURES = {
     "tt_build_vp_device": (I32, [P, I64, I32, I32, P, P]),
     "tt_tree_download": (I32, [P, P, SZ]),
     "tt_kick_drift": (I32, [P, P, P, I64, F, F, P]),
+    "tt_kick_drift_permuted": (I32, [P, P, P, P, P, I64, F, F, P, P, P, P]),
     "tt_tree_free": (I32, [P]),
     "tt_tree_get_info": (I32, [P, P]),
     "tt_sort_points": (I32, [P, P, I64, I32, P, P, P]),

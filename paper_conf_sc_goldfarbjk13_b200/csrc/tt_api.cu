@@ -415,4 +415,19 @@ tt_status tt_kick_drift(float *bodies, float *vel, const float *acc, int64_t n, 
     return e ? cuda_fail((cudaError_t)e) : TT_OK;
 }
 
+tt_status tt_kick_drift_permuted(const float *bodies, const float *vel, const float *acc, const int32_t *perm,
+                                 const int32_t *ids, int64_t n, float dt_kick, float dt_drift, float *bodies_out,
+                                 float *vel_out, int32_t *ids_out, tt_stream s) {
+    if (n < 0) return TT_ERR_INVALID_ARG;
+    if (n == 0) return TT_OK;
+    if (!bodies || !vel || !acc || !perm || !bodies_out || !vel_out || (ids && !ids_out) || !aligned(bodies, 16) ||
+        !aligned(vel, 16) || !aligned(acc, 16) || !aligned(bodies_out, 16) || !aligned(vel_out, 16))
+        return TT_ERR_INVALID_ARG;
+    tt_status st = have_device();
+    if (st != TT_OK) return st;
+    const int e = tt_launch_kick_drift_permuted(bodies, vel, acc, perm, ids, n, dt_kick, dt_drift, bodies_out, vel_out,
+                                                ids ? ids_out : nullptr, s);
+    return e ? cuda_fail((cudaError_t)e) : TT_OK;
+}
+
 }  // extern "C"

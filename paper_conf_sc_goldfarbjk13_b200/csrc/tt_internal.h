@@ -170,6 +170,8 @@ inline int tt_stage_count(const tt_blob_header &h, int bytes_per_node, int budge
 int tt_build_oct_gpu_impl(const float *bodies, long long n, void *stream, tt_blob_header *hdr, void **blob);
 
 int tt_launch_kick_drift(float *x, float *v, const float *a, long long n, float dtk, float dtd, void *stream);
+int tt_launch_kick_drift_permuted(const float *x, const float *v, const float *a, const int *perm, const int *ids,
+                                  long long n, float dtk, float dtd, float *xo, float *vo, int *ido, void *stream);
 
 int tt_build_kd_gpu_impl(const float *pts, long long n, int dim, int ld, int leaf, void *stream, tt_blob_header *hdr,
                          void **blob);

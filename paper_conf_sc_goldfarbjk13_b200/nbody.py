@@ -12,6 +12,14 @@ Integration is leapfrog kick-drift-kick, with consecutive half kicks merged:
   step 0:     kick(dt/2) + drift(dt), force
   step s > 0: kick(dt)   + drift(dt), force
   end:        kick(dt/2)
+
+``simulate_sharded`` is the multi-GPU form (one process per GPU, DESIGN.md
+§9.1): every rank holds all bodies in the order of the last point sort and
+rebuilds the same tree (the GPU build is deterministic, so no broadcast);
+it computes forces and the kick-drift for its warp-aligned shard of the
+sorted order only (tt_kick_drift_permuted writes the shard contiguously),
+and one all-gather per state array is the step's exchange.  Per-body results
+do not depend on the number of ranks.
 """
 from __future__ import annotations
 
@@ -36,6 +44,30 @@ def tt_kick_drift(bodies: torch.Tensor, vel: torch.Tensor, acc: torch.Tensor, dt
           "tt_kick_drift")
 
 
+def tt_kick_drift_permuted(bodies: torch.Tensor, vel: torch.Tensor, acc: torch.Tensor, perm: torch.Tensor,
+                           dt_kick: float, dt_drift: float, bodies_out: torch.Tensor, vel_out: torch.Tensor,
+                           ids: torch.Tensor | None = None, ids_out: torch.Tensor | None = None, stream=None) -> None:
+    """Row j of (bodies_out, vel_out, ids_out) = row perm[j] of the inputs after
+    v += acc * dt_kick; x += v * dt_drift (include/tt.h).  len(perm) rows."""
+    for name, t in (("bodies", bodies), ("vel", vel), ("acc", acc), ("bodies_out", bodies_out),
+                    ("vel_out", vel_out)):
+        _dev(t, torch.float32, name, 4)
+        if not t.is_contiguous():
+            raise ValueError(f"{name} must be a contiguous (n, 4) tensor")
+    _dev(perm, torch.int32, "perm")
+    n = perm.numel()
+    if bodies_out.shape[0] < n or vel_out.shape[0] < n:
+        raise ValueError("outputs need len(perm) rows")
+    ip = iop = None
+    if ids is not None:
+        _dev(ids, torch.int32, "ids")
+        _dev(ids_out, torch.int32, "ids_out")
+        ip, iop = ids.data_ptr(), ids_out.data_ptr()
+    check(L.load().tt_kick_drift_permuted(bodies.data_ptr(), vel.data_ptr(), acc.data_ptr(), perm.data_ptr(), ip, n,
+                                          float(dt_kick), float(dt_drift), bodies_out.data_ptr(), vel_out.data_ptr(),
+                                          iop, C.c_void_p(_stream_handle(stream))), "tt_kick_drift_permuted")
+
+
 def forces(bodies: torch.Tensor, theta: float, eps: float, out: torch.Tensor | None = None, mode="auto",
            stats=None):
     """One force pass on the current positions: GPU build, sort, traverse."""
@@ -57,3 +89,56 @@ def simulate(bodies: torch.Tensor, vel: torch.Tensor, steps: int, dt: float, the
     if steps:
         tt_kick_drift(bodies, vel, acc, 0.5 * dt, 0.0)
     return acc
+
+
+def simulate_sharded(bodies: torch.Tensor, vel: torch.Tensor, ids: torch.Tensor, steps: int, dt: float,
+                     theta: float = 0.5, eps: float = 0.05, mode="auto", group=None, final_kick: bool = True):
+    """Leapfrog KDK over `steps` steps with the bodies sharded across the ranks
+    of `group` (None and no process group: one rank).  Every rank passes the
+    same full (n, 4) bodies / vel and (n,) int32 ids; n must be a multiple of
+    64 * world (warp-aligned equal shards).  Returns (bodies, vel, ids), full
+    and identical on every rank, in the order of the last point sort (ids
+    carries the original body index of every row).
+
+    Step s: tree = build(x); perm = sort(x); a = force(x) for the rank's lanes
+    perm[lo:hi]; kick(dt/2 if s == 0 else dt) + drift(dt) gathered through
+    perm[lo:hi] into rows [lo, hi); all-gather.  With final_kick, one more
+    force pass and the closing kick(dt/2) (drift 0)."""
+    import torch.distributed as dist
+    from .parallel import allgather_rows, shard_range
+    world = dist.get_world_size(group) if dist.is_initialized() else 1
+    rank = dist.get_rank(group) if dist.is_initialized() else 0
+    n = bodies.shape[0]
+    if n % (64 * world):
+        raise ValueError("simulate_sharded needs n % (64 * world) == 0")
+    lo, hi = shard_range(n, rank, world)
+    x, v, i = bodies, vel, ids
+    xo, vo, io = torch.empty_like(x), torch.empty_like(v), torch.empty_like(i)
+    acc = torch.empty_like(x)
+
+    def half(dtk, dtd):
+        nonlocal x, v, i, xo, vo, io
+        tree = tt_build_oct_device(x)
+        perm = tt_sort_points(tree, x)
+        mine = perm[lo:hi]
+        tt_traverse_bh(tree, x, theta, eps, out=acc, order=mine, mode=mode)
+        tt_kick_drift_permuted(x, v, acc, mine, dtk, dtd, xo[lo:hi], vo[lo:hi], i, io[lo:hi])
+        if world > 1:
+            allgather_rows(xo, world, group)
+            allgather_rows(vo, world, group)
+            _allgather_ids(io, world, group)
+        x, xo = xo, x
+        v, vo = vo, v
+        i, io = io, i
+
+    for s in range(steps):
+        half(dt * (0.5 if s == 0 else 1.0), dt)
+    if steps and final_kick:
+        half(0.5 * dt, 0.0)
+    return x, v, i
+
+
+def _allgather_ids(ids: torch.Tensor, world: int, group=None):
+    """In-place all-gather of an int32 (n,) id column (rows as for allgather_rows)."""
+    from .parallel import allgather_rows
+    allgather_rows(ids.view(-1, 1), world, group)

@@ -44,6 +44,11 @@ def _worker(rank, world, port, q):
         PAR.allgather_rows(full, world)
         want = torch.arange(n, dtype=torch.float32)[:, None] + torch.tensor([0.0, 0.25, 0.5, 0.75])
         ok_gather = bool(torch.equal(full, want))
+        # int32 id column (the sharded time step's body ids), same row sharding
+        ids = torch.full((n,), -1, dtype=torch.int32)
+        ids[lo:hi] = torch.arange(lo, hi, dtype=torch.int32) * 3
+        PAR.allgather_rows(ids.view(-1, 1), world)
+        ok_gather = ok_gather and bool(torch.equal(ids, torch.arange(n, dtype=torch.int32) * 3))
         mx = PAR.max_over_ranks(float(rank + 1) * 1.5, "cpu")
         q.put((rank, ok_blob, ok_gather, mx))
         dist.destroy_process_group()
