@@ -64,8 +64,9 @@ def parse():
     ap.add_argument("--device-build", action="store_true",
                     help="build the tree on the GPU (tt_build_oct_device / tt_build_kd_device) instead of host "
                          "build + upload")
-    ap.add_argument("--variant", default="autoropes", choices=["autoropes", "recursive"],
-                    help="recursive = the paper's naive recursive GPU baseline (ablation, N mode)")
+    ap.add_argument("--variant", default="autoropes", choices=["autoropes", "recursive", "stack"],
+                    help="recursive = the paper's naive recursive GPU baseline (ablation, N mode); "
+                         "stack = explicit rope stacks, Fig.9b (ablation, BH and PC)")
     return ap.parse_args()
 
 
@@ -465,7 +466,8 @@ def run_ours(args, rank, world, local_rank):
     traverse(q_shard, out_shard, order_buf, st)
     torch.cuda.synchronize()
     visits = int(st.visits.to(torch.int64).sum().item())
-    tiles = -(-m // P._lib.TILE_POINTS[tree.kind])
+    tile_pts = P._lib.TILE_POINTS[tree.kind] if args.variant == "autoropes" else 32
+    tiles = -(-m // tile_pts)
     wf = int(st.warp_fetches[:tiles].to(torch.int64).sum().item())
     lock_frac = float((st.warp_mode[:tiles] == 1).float().mean().item())
     del st
@@ -633,9 +635,9 @@ def run_ours(args, rank, world, local_rank):
         "visits_per_point": visits / m,
         "lockstep_warp_fraction": lock_frac,
         # lane-slots offered by the warp fetches / useful visits (lockstep tiles)
-        "work_expansion_fetch_over_visits": (wf * P._lib.TILE_POINTS[tree.kind] / visits)
+        "work_expansion_fetch_over_visits": (wf * tile_pts / visits)
         if visits and lock_frac > 0.99 else None,
-        "warp_tile_points": P._lib.TILE_POINTS[tree.kind],
+        "warp_tile_points": tile_pts,
         "traverse_ms": kms, "upload_ms": upload_ms, "tree_build_ms": build_ms, "tree_build": build_where,
         "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": (launches or 0) * args.steps,
         "gpu_launches_per_step": launches,

@@ -238,12 +238,20 @@ typedef struct tt_traverse_opts {
                                 1 = naive recursive baseline (P:L1084-1090,
                                 independent mode only -- LOCKSTEP is
                                 TT_ERR_UNSUPPORTED; it fills stats->visits only,
-                                the warp_* arrays are left untouched)           */
+                                the warp_* arrays are left untouched);
+                                2 = explicit rope stack, the paper's Fig.9b
+                                form (BH and PC only, else TT_ERR_UNSUPPORTED):
+                                independent = per-thread stacks interleaved in
+                                global memory, lockstep = one (node, mask)
+                                stack per warp in shared memory;
+                                AUTO = BH lockstep, PC independent; 32-point
+                                warp tiles                                     */
 } tt_traverse_opts;
 
 typedef enum tt_variant {
     TT_VARIANT_AUTOROPES = 0,
-    TT_VARIANT_RECURSIVE = 1
+    TT_VARIANT_RECURSIVE = 1,
+    TT_VARIANT_STACK = 2
 } tt_variant;
 
 /* Barnes-Hut force pass (Fig.9): bodies float4 (x,y,z,m) rows;

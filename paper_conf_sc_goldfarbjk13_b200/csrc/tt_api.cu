@@ -78,7 +78,9 @@ tt_status setup_common(const tt_tree *t, int kind, int64_t n, const tt_traverse_
         if (o->block_threads != 0 && o->block_threads != 256) return TT_ERR_UNSUPPORTED;
         if (o->ctas_per_sm < 0) return TT_ERR_INVALID_ARG;
         cfg.ctas_per_sm = o->ctas_per_sm;
-        if (o->variant != TT_VARIANT_AUTOROPES && o->variant != TT_VARIANT_RECURSIVE) return TT_ERR_INVALID_ARG;
+        if (o->variant != TT_VARIANT_AUTOROPES && o->variant != TT_VARIANT_RECURSIVE &&
+            o->variant != TT_VARIANT_STACK)
+            return TT_ERR_INVALID_ARG;
         if (o->variant == TT_VARIANT_RECURSIVE && o->mode == TT_MODE_LOCKSTEP) return TT_ERR_UNSUPPORTED;
         cfg.variant = o->variant;
     }
@@ -336,7 +338,9 @@ tt_status tt_traverse_bh(const tt_tree *t, const float *bodies, const int32_t *s
     }
     p.eps2 = eps * eps;
     p.acc = reinterpret_cast<float4 *>(acc_out);
-    return finish_launch(cfg.variant == TT_VARIANT_RECURSIVE ? tt_launch_bh_recursive(p, cfg) : tt_launch_bh(p, cfg));
+    return finish_launch(cfg.variant == TT_VARIANT_RECURSIVE ? tt_launch_bh_recursive(p, cfg)
+                         : cfg.variant == TT_VARIANT_STACK   ? tt_launch_bh_stack(p, cfg)
+                                                             : tt_launch_bh(p, cfg));
 }
 
 tt_status tt_traverse_pc(const tt_tree *t, const float *q, int64_t n, int32_t ld, float radius, uint32_t *count_out,
@@ -357,7 +361,8 @@ tt_status tt_traverse_pc(const tt_tree *t, const float *q, int64_t n, int32_t ld
     p.r2 = radius * radius;  // rn(r*r), reading R1
     p.count = count_out;
     return finish_launch(cfg.variant == TT_VARIANT_RECURSIVE ? tt_launch_pc_recursive(p, t->hdr.dim, cfg)
-                                                            : tt_launch_pc(p, t->hdr.dim, cfg));
+                         : cfg.variant == TT_VARIANT_STACK   ? tt_launch_pc_stack(p, t->hdr.dim, cfg)
+                                                             : tt_launch_pc(p, t->hdr.dim, cfg));
 }
 
 tt_status tt_traverse_knn(const tt_tree *t, const float *q, int64_t n, int32_t ld, int32_t k, int32_t *idx_out,
@@ -379,6 +384,7 @@ tt_status tt_traverse_knn(const tt_tree *t, const float *q, int64_t n, int32_t l
     p.k = k;
     p.idx = idx_out;
     p.d2 = d2_out;
+    if (cfg.variant == TT_VARIANT_STACK) return TT_ERR_UNSUPPORTED;  // guided kernels already keep rope stacks
     return finish_launch(cfg.variant == TT_VARIANT_RECURSIVE ? tt_launch_knn_recursive(p, t->hdr.dim, cfg)
                                                             : tt_launch_knn(p, t->hdr.dim, cfg));
 }
@@ -399,6 +405,7 @@ tt_status tt_traverse_vp(const tt_tree *t, const float *q, int64_t n, int32_t ld
     p.ld = ld;
     p.idx = idx_out;
     p.d2 = d2_out;
+    if (cfg.variant == TT_VARIANT_STACK) return TT_ERR_UNSUPPORTED;  // guided kernels already keep rope stacks
     return finish_launch(cfg.variant == TT_VARIANT_RECURSIVE ? tt_launch_vp_recursive(p, t->hdr.dim, cfg)
                                                             : tt_launch_vp(p, t->hdr.dim, cfg));
 }

@@ -472,6 +472,60 @@ def test_recursive_baseline_matches_oracle(bh_small, knn_small, vp_small, pc_set
     assert np.array_equal(idx.cpu().numpy(), refv.out[0]) and np.array_equal(d2.cpu().numpy(), refv.out[1])
 
 
+# ------------------------------------ explicit rope-stack variant (NEXT-3)
+@pytest.mark.parametrize("mode", MODES)
+@pytest.mark.parametrize("sorted_", [False, True])
+def test_stack_variant_matches_oracle(bh_small, pc_setup, mode, sorted_):
+    """Fig.9b's explicit rope stacks (per-thread interleaved global stacks in
+    independent mode, one (node, mask) smem stack per warp in lockstep):
+    same results and per-point visits as the oracle; a lockstep warp pops
+    exactly the union of its 32 lanes' traversals (Fig.8)."""
+    b, ot, ref, tree = bh_small
+    bd = dev(b)
+    order = P.tt_sort_points(tree, bd) if sorted_ else None
+    st = P.Stats.alloc(len(b), "cuda")
+    acc = P.tt_traverse_bh(tree, bd, 0.5, 0.05, order=order, mode=mode, stats=st, variant="stack").cpu().numpy()
+    assert rel_err(acc, ref.out[0]).max() <= BH_TOL
+    assert np.array_equal(st.visits.cpu().numpy(), ref.visits)
+    o = order.cpu().numpy() if sorted_ else np.arange(len(b))
+    if mode != "independent":  # AUTO = lockstep for BH
+        union = oracle.unguided_warp_union(ot, b[o], 0.5, W=32)
+        assert np.array_equal(st.warp_fetches.cpu().numpy()[:len(union)], union)
+    c, p, otp, refp, treep = pc_setup
+    q = dev(p)
+    order = P.tt_sort_points(treep, q) if sorted_ else None
+    st = P.Stats.alloc(len(p), "cuda")
+    cnt = P.tt_traverse_pc(treep, q, c["radius"], order=order, mode=mode, stats=st, variant="stack")
+    assert np.array_equal(cnt.cpu().numpy().astype(np.uint32), refp.out[0])
+    assert np.array_equal(st.visits.cpu().numpy(), refp.visits)
+    if mode == "lockstep":
+        o = order.cpu().numpy() if sorted_ else np.arange(len(p))
+        union = oracle.unguided_warp_union(otp, p[o], c["radius"])
+        assert np.array_equal(st.warp_fetches.cpu().numpy(), union)
+
+
+def test_stack_variant_edge_cases():
+    """theta = 0 (every cell opens: the direct sum), duplicate bodies, a ragged
+    last warp, buckets; kNN/VP report the variant as unsupported."""
+    from tests import brute
+    b = ttgen.plummer(1001, seed=240)
+    b[10, :3] = b[11, :3] = b[12, :3]
+    tree = P.tt_tree_upload(P.build_oct(b))
+    for mode in MODES:
+        acc = P.tt_traverse_bh(tree, dev(b), 0.0, 0.05, mode=mode, variant="stack").cpu().numpy()
+        assert rel_err(acc, brute.direct_sum(b, 0.05)).max() <= BH_TOL
+    p = ttgen.gaussian_mixture(3000, 7, seed=241, components=6)
+    q = ttgen.gaussian_mixture(777, 7, seed=242, components=6)
+    ot = oracle.build_kd(p, 8)
+    ref = oracle.pc(ot, q, 0.15)
+    t = P.tt_tree_upload(P.build_kd(p, 8))
+    for mode in MODES:
+        cnt = P.tt_traverse_pc(t, dev(q), 0.15, mode=mode, variant="stack")
+        assert np.array_equal(cnt.cpu().numpy().astype(np.uint32), ref.out[0])
+    with pytest.raises(P.TTError):
+        P.tt_traverse_knn(t, dev(q), 4, variant="stack")
+
+
 # ------------------------------------------------- GPU tree build (NEXT-1)
 @pytest.mark.parametrize("n,dups", [(1, False), (2, False), (3001, True), (20011, True), (1_000_000, False)])
 def test_gpu_oct_build_is_byte_identical_to_host_pack(n, dups):
