@@ -184,19 +184,23 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
             int cur = 0;
             // kernel parameters pinned in registers for the hot loop (otherwise
             // re-read from the constant bank every iteration)
-            const tt_oct_rec *grec = g_rec;
-            int dbits = dsq_bits;
-            float e2 = eps2;
-            asm volatile("" : "+l"(grec), "+r"(dbits), "+f"(e2));
+            // (through a shuffle: ptxas re-reads plain parameters from the
+            // constant bank inside the loop, but cannot rematerialise a SHFL)
+            const tt_oct_rec *grec =
+                reinterpret_cast<const tt_oct_rec *>(__shfl_sync(TT_FULL, reinterpret_cast<long long>(g_rec), 0));
+            const int dbits = __shfl_sync(TT_FULL, dsq_bits, 0);
+            const float e2 = __shfl_sync(TT_FULL, eps2, 0);
             const float2 e22 = make_float2(e2, e2);
+
             for (;;) {
 #pragma unroll 1
                 for (int k = 0; k < kFlush; ++k) {
                     // lockstep: one warp-uniform address, served by L1 (top levels
                     // included -- they are also at [0, top) of the global array);
                     // measured 2.7% faster than the smem/global select here
-                    const float4 g = __ldg(reinterpret_cast<const float4 *>(&grec[cur].gx));
-                    const int4 t = __ldg(reinterpret_cast<const int4 *>(&grec[cur].first_child));
+                    float4 g;
+                    int4 t;
+                    ldg_rec256(grec + cur, g, t);
                     if (STATS) ++steps;
                     const int lvl = t.w;
                     const float dl = EXP_DSQ ? dsq_at(dbits, lvl) : s_dsq[lvl];
@@ -228,7 +232,8 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
                     cur = __any_sync(TT_FULL, o0 || o1) ? t.x : t.y;
                     if (cur == TT_END) break;
                 }
-                // fp32 partials -> fp64 (warp-uniform cadence)
+                // fp32 partials -> fp64 (warp-uniform cadence); the fp64 sums
+                // live in shared memory (12 registers freed for the hot loop)
                 bd[0].acc.X += (double)ax.x;
                 bd[0].acc.Y += (double)ay.x;
                 bd[0].acc.Z += (double)az.x;

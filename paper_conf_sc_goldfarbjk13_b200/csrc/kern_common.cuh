@@ -273,6 +273,15 @@ __device__ __forceinline__ float rsqrt_ftz(float x) {
     return y;
 }
 
+// One 32-byte node record (one DRAM sector) in a single 256-bit load
+// (ld.global.nc.v8, SASS LDG.E.ENL2.256 on sm_100): half the load
+// instructions of two 128-bit loads.  p must be 32-B aligned.
+__device__ __forceinline__ void ldg_rec256(const void *p, float4 &g, int4 &t) {
+    asm("ld.global.nc.v8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+        : "=f"(g.x), "=f"(g.y), "=f"(g.z), "=f"(g.w), "=r"(t.x), "=r"(t.y), "=r"(t.z), "=r"(t.w)
+        : "l"(p));
+}
+
 // L1 prefetch of a global line (the next nodes of a walk are known one step
 // ahead: both children are in the current record).
 __device__ __forceinline__ void prefetch_l1(const void *p) {
