@@ -223,10 +223,13 @@ typedef struct tt_stats {
 
 typedef struct tt_traverse_opts {
     int32_t mode;            /* tt_mode                                          */
-    int32_t auto_min_depth;  /* AUTO: lockstep iff the warp's points share a tree
-                                path of at least this many levels (0 = always,
+    int32_t auto_min_depth;  /* AUTO: T, the tree level of the per-warp coherence
+                                test -- lockstep iff the warp's points, in launch
+                                order, change their level-T cell (oct: 2^T grid
+                                cell of the root cube; kd / vp: T-level descent
+                                path) fewer than 8 times (0 = always lockstep,
                                 >= 64 = never); -1 = kernel default, measured on
-                                B200: BH 6, kNN 4, VP 4, PC never
+                                B200: BH 3, kNN 4, VP 4, PC never
                                 (10k-point PC is latency-bound: independent wins) */
     const uint32_t *order;   /* [n] device, nullable: lane j of the launch processes
                                 point order[j] (e.g. perm from tt_sort_points);

@@ -76,22 +76,6 @@ struct Body {
     Acc acc;
 };
 
-// 63-bit octant path of a body through the root cube (fp64 comparisons, R8a).
-__device__ __forceinline__ unsigned long long oct_path(float4 b, const double c0[3], double side, int levels) {
-    double c[3] = {c0[0], c0[1], c0[2]};
-    unsigned long long code = 0;
-    for (int l = 0; l < levels; ++l) {
-        double h = side * 0.25;
-        int o = ((double)b.x >= c[0]) | (((double)b.y >= c[1]) << 1) | (((double)b.z >= c[2]) << 2);
-        code = (code << 3) | (unsigned)o;
-        c[0] += (o & 1) ? h : -h;
-        c[1] += (o & 2) ? h : -h;
-        c[2] += (o & 4) ? h : -h;
-        side *= 0.5;
-    }
-    return code;
-}
-
 template <bool STATS, bool EXP_DSQ>
 __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
     extern __shared__ __align__(128) unsigned char smem[];
@@ -143,22 +127,41 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
 
         bool lock = P.c.mode != TT_MODE_INDEPENDENT;
         if (P.c.mode == TT_MODE_AUTO && P.c.auto_min_depth > 0) {
-            const int lv = min(P.c.auto_min_depth, 21);
-            // common octant-path prefix over all kBPL*32 bodies of the tile
-            const unsigned long long c0 = oct_path(bd[0].b, P.c.root_center, P.c.root_side, lv);
-            const int leader = __ffs(__ballot_sync(TT_FULL, bd[0].valid)) - 1;
-            const unsigned long long lead = __shfl_sync(TT_FULL, c0, leader);
-            unsigned long long acc_or = 0;
+            // Coherence of the tile (reading R19): walk its kBPL*32 bodies in
+            // launch order and count how often the level-T octree cell changes
+            // (T = auto_min_depth, cells from 21-bit fixed-point coordinates in
+            // the root cube).  A sorted tile is a Morton-contiguous run: a few
+            // changes even where it straddles a cell face; an unsorted tile
+            // changes at almost every body.  Lockstep iff fewer than
+            // kAutoMaxChanges.  (A common-prefix test sent the few sorted tiles
+            // that straddle a top-level face to independent mode, ~2x slower
+            // per tile, and those set the kernel's tail.)  A heuristic only:
+            // results do not depend on the mode.
+            const int T = min(P.c.auto_min_depth, 10);  // (>= 64: never lockstep, below)
+            const float lo_x = (float)(P.c.root_center[0] - 0.5 * P.c.root_side);
+            const float lo_y = (float)(P.c.root_center[1] - 0.5 * P.c.root_side);
+            const float lo_z = (float)(P.c.root_center[2] - 0.5 * P.c.root_side);
+            const float sc = (float)((double)(1 << T) / P.c.root_side);
+            const int cmax = (1 << T) - 1;
+            unsigned cell[kBPL];
 #pragma unroll
             for (int j = 0; j < kBPL; ++j) {
-                const unsigned long long cj = j == 0 ? c0 : oct_path(bd[j].b, P.c.root_center, P.c.root_side, lv);
-                if (bd[j].valid) acc_or |= cj ^ lead;
+                const unsigned cx = (unsigned)min(max(__float2int_rd((bd[j].b.x - lo_x) * sc), 0), cmax);
+                const unsigned cy = (unsigned)min(max(__float2int_rd((bd[j].b.y - lo_y) * sc), 0), cmax);
+                const unsigned cz = (unsigned)min(max(__float2int_rd((bd[j].b.z - lo_z) * sc), 0), cmax);
+                cell[j] = (cx << (2 * T)) | (cy << T) | cz;
             }
-            const unsigned hi = __reduce_or_sync(TT_FULL, (unsigned)(acc_or >> 32));
-            const unsigned lo = __reduce_or_sync(TT_FULL, (unsigned)acc_or);
-            const unsigned long long x = ((unsigned long long)hi << 32) | lo;
-            const int common = x == 0 ? lv : (__clzll((long long)x) - (64 - 3 * lv)) / 3;
-            lock = common >= P.c.auto_min_depth;
+            int changes = 0;
+#pragma unroll
+            for (int j = 0; j < kBPL; ++j) {
+                // predecessor in launch order: lane-1 of the same row, or the
+                // last lane of the previous row
+                const unsigned up = __shfl_up_sync(TT_FULL, cell[j], 1);
+                const unsigned prev_row = j > 0 ? __shfl_sync(TT_FULL, cell[j > 0 ? j - 1 : 0], 31) : cell[j];
+                const unsigned prev = lane > 0 ? up : prev_row;
+                changes += __popc(__ballot_sync(TT_FULL, bd[j].valid && cell[j] != prev));
+            }
+            lock = P.c.auto_min_depth < 64 && changes < kAutoMaxChanges;
         }
 
         unsigned fetches = 0, steps = 0;

@@ -303,6 +303,17 @@ __device__ __forceinline__ int warp_common_levels(unsigned long long code, unsig
     return lead_zero / bits;
 }
 
+// Per-warp coherence for the AUTO mode choice (reading R19): the number of
+// launch-order neighbours (lane-1, lane) whose top-level path codes differ.
+// A sorted tile is a run of consecutive leaves: a few changes even where it
+// straddles a top-level split; an unsorted tile changes at almost every lane.
+// (Invalid lanes only occur at the ragged end of the last tile.)
+constexpr int kAutoMaxChanges = 8;
+__device__ __forceinline__ int warp_key_changes(unsigned long long key, bool valid) {
+    const unsigned long long up = __shfl_up_sync(TT_FULL, key, 1);
+    return __popc(__ballot_sync(TT_FULL, valid && (threadIdx.x & 31) > 0 && key != up));
+}
+
 __device__ __forceinline__ unsigned warp_sum(unsigned v) { return __reduce_add_sync(TT_FULL, v); }
 
 // Stats writer for the warp tile (lane 0).

@@ -175,7 +175,7 @@ __global__ void __launch_bounds__(kBlock) knn_kernel(const tt_knn_params P, int 
                 cur = left ? t.x : t.y;
                 ++lv;
             }
-            lock = warp_common_levels(code << (maxl - lv), vmask, 1, maxl) >= P.c.auto_min_depth;
+            lock = P.c.auto_min_depth == 0 || warp_key_changes(code << (maxl - lv), valid) < kAutoMaxChanges;
         }
 
         KBest<KT> kb;

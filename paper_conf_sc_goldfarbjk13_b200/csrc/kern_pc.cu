@@ -98,8 +98,7 @@ __global__ void __launch_bounds__(kBlock) pc_kernel(const tt_pc_params P) {
                 cur = left ? t.x : t.y;
                 ++lv;
             }
-            const int common = warp_common_levels(code << (maxl - lv), vmask, 1, maxl);
-            lock = common >= P.c.auto_min_depth;
+            lock = P.c.auto_min_depth < 64 && warp_key_changes(code << (maxl - lv), valid) < kAutoMaxChanges;
         }
 
         unsigned count = 0, visits = 0, fetches = 0, steps = 0;

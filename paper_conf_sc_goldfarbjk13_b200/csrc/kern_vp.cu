@@ -132,7 +132,7 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
                 cur = nx;
                 ++lv;
             }
-            lock = warp_common_levels(code << (maxl - lv), vmask, 1, maxl) >= P.c.auto_min_depth;
+            lock = P.c.auto_min_depth == 0 || warp_key_changes(code << (maxl - lv), valid) < kAutoMaxChanges;
         }
 
         float best_d = POS_INF, tau = POS_INF;

@@ -38,7 +38,7 @@ bool dim_supported(int d) { return (d >= 1 && d <= 8) || d == 16; }
 
 // Default AUTO thresholds (levels of common tree path for lockstep), see
 // tt_traverse_opts.auto_min_depth and DESIGN.md §4.5.
-constexpr int kAutoBH = 6, kAutoPC = 255, kAutoKNN = 4, kAutoVP = 4;
+constexpr int kAutoBH = 3, kAutoPC = 255, kAutoKNN = 4, kAutoVP = 4;
 
 // Shared-memory budgets for the staged top levels, per kernel (bytes/node):
 // the budget trades staged levels against occupancy.

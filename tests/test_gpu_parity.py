@@ -472,6 +472,34 @@ def test_recursive_baseline_matches_oracle(bh_small, knn_small, vp_small, pc_set
     assert np.array_equal(idx.cpu().numpy(), refv.out[0]) and np.array_equal(d2.cpu().numpy(), refv.out[1])
 
 
+# ------------------------------------------------ per-warp mode choice (a2)
+def test_auto_mode_choice_follows_coherence(bh_small, knn_small, vp_small):
+    """AUTO (reading R19): sorted tiles run lockstep (even those straddling a
+    top-level split), unsorted tiles run independent -- and results equal the
+    lockstep run's (BH: up to the fp64 flush cadence)."""
+    def frac(st, n, tile):  # over full tiles (a ragged last tile has few lanes to disagree)
+        return (st.warp_mode.cpu().numpy()[:n // tile] == 1).mean()
+    b, ot, ref, tree = bh_small
+    bd = dev(b)
+    for sorted_, want in ((True, 1.0), (False, 0.0)):
+        order = P.tt_sort_points(tree, bd) if sorted_ else None
+        st = P.Stats.alloc(len(b), "cuda")
+        P.tt_traverse_bh(tree, bd, 0.5, 0.05, order=order, stats=st)
+        # 20k bodies: a few sorted tiles in the sparse outskirts span many
+        # level-3 cells and count as incoherent (99.9% lockstep at 1M)
+        assert abs(frac(st, len(b), 32 * P._lib.BH_POINTS_PER_LANE) - want) <= 0.03
+    for (p, q, otk, treek), call in ((knn_small, lambda t, x, **kw: P.tt_traverse_knn(t, x, 8, **kw)),
+                                     (vp_small, lambda t, x, **kw: P.tt_traverse_vp(t, x, **kw))):
+        qd = dev(q)
+        for sorted_, want in ((True, 1.0), (False, 0.0)):
+            order = P.tt_sort_points(treek, qd) if sorted_ else None
+            st = P.Stats.alloc(len(q), "cuda")
+            idx, d2 = call(treek, qd, order=order, stats=st)
+            il, dl = call(treek, qd, order=order, mode="lockstep")
+            assert torch.equal(idx, il) and torch.equal(d2, dl)
+            assert abs(frac(st, len(q), 32) - want) <= 0.01, (sorted_, frac(st, len(q), 32))
+
+
 # ------------------------------------ explicit rope-stack variant (NEXT-3)
 @pytest.mark.parametrize("mode", MODES)
 @pytest.mark.parametrize("sorted_", [False, True])
