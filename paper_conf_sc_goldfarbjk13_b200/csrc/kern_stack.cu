@@ -306,6 +306,7 @@ int launch_with_stack(Kern kern, const Params &p, const tt_launch_cfg &cfg) {
     int2 *gstack = nullptr;
     const cudaStream_t s = (cudaStream_t)cfg.stream;
     if (p.c.mode == TT_MODE_INDEPENDENT || (p.c.mode == TT_MODE_AUTO && std::is_same<Params, tt_pc_params>::value)) {
+        tt_keep_pool_memory();
         e = cudaMallocAsync((void **)&gstack, sizeof(int2) * (size_t)cap * (size_t)grid * kBlock, s);
         if (e != cudaSuccess) return (int)e;
     }

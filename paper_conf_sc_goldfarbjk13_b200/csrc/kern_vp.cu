@@ -20,8 +20,10 @@
 //     set (§4.3, tie -> inside first).
 //   N mode, INDEPENDENT launches: per-lane {parent << 1 | side, d}; the child
 //     and radius come from the parent's 16-B header at pop.
-//   N mode inside an AUTO launch (rare warps): per-lane {parent << 1 | side}
-//     only; d is recomputed from the parent's vantage point at pop.
+//   N mode inside an AUTO launch: per-lane {parent << 1 | side} in shared
+//     memory, d in a per-thread interleaved global scratch [cap][threads]
+//     (coalesced, L1/L2-resident; recomputing d from the parent's vantage
+//     point instead made unsorted AUTO launches 870 vs 616 ms at 1M).
 // The narrow layout halves the shared-memory stack of AUTO/LOCKSTEP launches,
 // which the SM gives back to L1 for the (L2-resident) tree.
 #include "kern_common.cuh"
@@ -67,7 +69,7 @@ __device__ __forceinline__ int child_args(int4 t, int side, float d, float &lb, 
 }
 
 template <int DIM, bool STATS>
-__global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int cap) {
+__global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int cap, float *g_d) {
     extern __shared__ __align__(128) unsigned char smem[];
     constexpr int DP = (DIM + 3) & ~3;
     uint64_t *bar = reinterpret_cast<uint64_t *>(smem);
@@ -83,6 +85,7 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
     const bool wide = P.c.mode == TT_MODE_INDEPENDENT;
+    const size_t gtid = blockIdx.x * (size_t)blockDim.x + threadIdx.x, gstride = (size_t)gridDim.x * blockDim.x;
     // per-warp region (vp_stack_bytes): wide: ent[cap][32], d[cap][32];
     // narrow: d (or N-mode ent)[cap][32], then int4 l_e[cap]
     unsigned char *wreg = s_stack + (size_t)warp * vp_stack_bytes(cap, wide);
@@ -163,6 +166,7 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
                     if (second != TT_END) {
                         n_ent[sp * 32 + lane] = (cur << 1) | (first_side ^ 1);
                         if (wide) n_d[sp * 32 + lane] = d;
+                        else g_d[(size_t)sp * gstride + gtid] = d;
                         ++sp;
                     }
                     const int first = child_args(t, first_side, d, lb, sc);
@@ -175,14 +179,7 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
                     --sp;
                     const int e = n_ent[sp * 32 + lane];
                     float d;
-                    if (wide) {
-                        d = n_d[sp * 32 + lane];
-                    } else {  // same operands and operations as at push
-                        int4 tp;
-                        float v[DIM];
-                        ld_node<DIM>(s_rec, s_vpt, g_rec, g_vpt, DP, top, e >> 1, tp, v);
-                        d = __fsqrt_rn(pinned_d2<DIM>(q, v));
-                    }
+                    d = wide ? n_d[sp * 32 + lane] : g_d[(size_t)sp * gstride + gtid];
                     cur = child_args(hdr(e >> 1), e & 1, d, lb, sc);
                 } else {
                     cur = TT_END;
@@ -287,8 +284,18 @@ int launch(const tt_vp_params &p, const tt_launch_cfg &cfg) {
     const long long need = (ntiles + kWarps - 1) / kWarps;
     if (grid > need) grid = need;
     if (grid < 1) grid = 1;
-    kern<<<(unsigned)grid, kBlock, smem, (cudaStream_t)cfg.stream>>>(p, cap);
-    return (int)cudaGetLastError();
+    // AUTO: d of the independent warps' stack entries (see the header comment)
+    float *g_d = nullptr;
+    const cudaStream_t s = (cudaStream_t)cfg.stream;
+    if (p.c.mode == TT_MODE_AUTO) {
+        tt_keep_pool_memory();
+        e = cudaMallocAsync((void **)&g_d, sizeof(float) * (size_t)cap * (size_t)grid * kBlock, s);
+        if (e != cudaSuccess) return (int)e;
+    }
+    kern<<<(unsigned)grid, kBlock, smem, s>>>(p, cap, g_d);
+    e = cudaGetLastError();
+    if (g_d) cudaFreeAsync(g_d, s);
+    return (int)e;
 }
 
 template <int DIM>
