@@ -603,7 +603,8 @@ def run_ours(args, rank, world, local_rank):
     if cnt and cnt.get("src_sha256") == kernel_sha256(name):
         inst = cnt["warp_inst_per_point"] * m
         issue_peak = nsm * 4 * sm_mhz * 1e6 / 1e9  # warp instructions per ns -> G/s
-        roofline = {"bound": "issue", "achieved": round(inst / (kms / 1e3) / 1e9, 1), "peak": round(issue_peak, 1),
+        roofline = {"bound": "alu", "roof": "warp-instruction issue (ALU, LSU and branch instructions all issue here)",
+                    "achieved": round(inst / (kms / 1e3) / 1e9, 1), "peak": round(issue_peak, 1),
                     "unit": "Gwarp-inst/s", "frac": round(inst / (kms / 1e3) / 1e9 / issue_peak, 4),
                     "inst_per_launch": int(inst),
                     "achieved_def": f"ncu smsp__inst_executed of this kernel source ({cnt['round']}) / live kernel time",
