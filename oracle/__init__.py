@@ -16,6 +16,8 @@ Parity status of each function:
   bh                               pinned: theta=0 == O(n^2) direct sum, two-body closed form
   knn                              pinned: brute-force partial sort on (d2, id)
   vp                               pinned: brute-force argmin on (d2, id)
+  build_nn / nn (NEXT-3, R21)      pinned: brute-force argmin on (d2, id), == kNN k=1 == VP;
+                                   builder: median/split/partition invariants
   sort_keys                        pinned: Morton/preorder invariants, bijection
   *_lockstep, unguided_warp_union  pinned: results == independent walks; fetches >= max lane
                                    visits; absolute fetch counts parity unpinned
@@ -63,6 +65,8 @@ def lib():
         L.or_build_oct.argtypes = [P, I64]
         L.or_build_vp.restype = P
         L.or_build_vp.argtypes = [P, I64, I, I]
+        L.or_build_nn.restype = P
+        L.or_build_nn.argtypes = [P, I64, I, I]
         L.or_build_generic.restype = P
         L.or_build_generic.argtypes = [I, P, P, I]
         L.or_free.argtypes = [P]
@@ -84,6 +88,8 @@ def lib():
         L.or_unguided_warp_union.argtypes = [P, P, I64, I, I, F, P, I]
         L.or_knn_lockstep.argtypes = [P, P, I64, I, I, P, P, P, P, I]
         L.or_vp_lockstep.argtypes = [P, P, I64, I, P, P, P, P, I]
+        L.or_nn.argtypes = [P, P, I64, I, P, P, P, P, I]
+        L.or_nn_lockstep.argtypes = [P, P, I64, I, P, P, P, P, I]
         L.or_max_threads.restype = I
         _lib = L
     return _lib
@@ -163,6 +169,13 @@ def build_vp(pts: np.ndarray) -> Tree:
     return Tree(lib().or_build_vp(_p(pts), n, d, d), "vp", pts)
 
 
+def build_nn(pts: np.ndarray) -> Tree:
+    """Point-per-node kd-tree of the paper's NN benchmark (reading R21)."""
+    pts = _f32(pts)
+    n, d = pts.shape
+    return Tree(lib().or_build_nn(_p(pts), n, d, d), "nn", pts)
+
+
 def build_generic(children: list[list[int]], root: int = 0) -> Tree:
     """Hand-given tree: children[v] = ordered child labels of node v."""
     ptr = np.zeros(len(children) + 1, dtype=np.int32)
@@ -237,6 +250,19 @@ def vp(tree: Tree, q: np.ndarray, threads=None, stats=False) -> Result:
     return Result((idx, d2), v, h)
 
 
+def nn(tree: Tree, q: np.ndarray, threads=None, stats=False) -> Result:
+    """Nearest neighbour over the R21 point-per-node kd-tree (Fig.5 pattern)."""
+    q = _f32(q)
+    m = len(q)
+    idx = np.empty(m, np.int64)
+    d2 = np.empty(m, np.float32)
+    v = np.empty(m, np.int64) if stats else None
+    h = np.empty(m, np.uint64) if stats else None
+    rc = lib().or_nn(tree._h, _p(q), m, q.shape[1], _p(idx), _p(d2), _p(v), _p(h), _threads(threads))
+    assert rc == 0
+    return Result((idx, d2), v, h)
+
+
 def sort_keys(tree: Tree, q: np.ndarray, threads=None) -> np.ndarray:
     q = _f32(q)
     keys = np.empty(len(q), np.uint64)
@@ -283,6 +309,19 @@ def vp_lockstep(tree: Tree, q: np.ndarray, threads=None):
     lv = np.empty(m, np.int64)
     wf = np.empty((m + 31) // 32, np.int64)
     rc = lib().or_vp_lockstep(tree._h, _p(q), m, q.shape[1], _p(idx), _p(d2), _p(lv), _p(wf),
+                              _threads(threads))
+    assert rc == 0
+    return idx, d2, lv, wf
+
+
+def nn_lockstep(tree: Tree, q: np.ndarray, threads=None):
+    q = _f32(q)
+    m = len(q)
+    idx = np.empty(m, np.int64)
+    d2 = np.empty(m, np.float32)
+    lv = np.empty(m, np.int64)
+    wf = np.empty((m + 31) // 32, np.int64)
+    rc = lib().or_nn_lockstep(tree._h, _p(q), m, q.shape[1], _p(idx), _p(d2), _p(lv), _p(wf),
                               _threads(threads))
     assert rc == 0
     return idx, d2, lv, wf

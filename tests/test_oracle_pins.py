@@ -395,3 +395,85 @@ def test_guided_lockstep_results_equal_independent():
     idx, d2 = oracle.vp(vt, q16).out
     li, ld, lv, wf = oracle.vp_lockstep(vt, q16)
     assert np.array_equal(li, idx) and np.array_equal(ld, d2)
+
+
+# ------------------------------------------------ NN kd-tree (NEXT-3, R21)
+@pytest.mark.parametrize("n,dim", [(1500, 3), (2001, 7), (64, 16), (1, 4), (2, 2)])
+def test_nn_build_invariants(n, dim):
+    """Point-per-node kd-tree (the paper's NN; build rule R21):
+    preorder/ropes, every point at exactly one node, the node's point is the
+    median of its set on (x[dim], id) along the largest-extent dimension."""
+    p = ttgen.gaussian_mixture(n, dim, seed=15, components=3)
+    if n > 100:
+        p[50:60] = p[3]  # exact duplicates: ties on x[dim] broken by id
+    t = oracle.build_nn(p)
+    _check_preorder_skip(t)
+    order = t.tree_order()
+    assert np.array_equal(np.sort(order), np.arange(n))
+    assert t.n_nodes == n
+    pb, pcn = t.i64(oracle.F_PBEGIN), t.i64(oracle.F_PCOUNT)
+    sd, split, me = t.i64(oracle.F_SPLITDIM), t.f32(oracle.F_SPLIT), t.i64(oracle.F_VP)
+    ch = t.children()
+    for v in range(t.n_nodes):
+        ids = order[pb[v]:pb[v] + pcn[v]]
+        assert ids[0] == me[v]  # the node's own point first, then its subtrees
+        if len(ids) == 1:
+            assert sd[v] == -1 and ch[v, 0] == -1 and ch[v, 1] == -1
+            continue
+        ext = (p[ids].max(0) - p[ids].min(0)).astype(np.float32)
+        assert sd[v] == int(np.argmax(ext))  # largest extent, lowest dim on ties
+        d = sd[v]
+        srt = sorted(ids, key=lambda i: (p[i, d], i))
+        m = len(ids) // 2
+        assert srt[m] == me[v] and split[v] == p[me[v], d]
+        left = order[pb[ch[v, 0]]:pb[ch[v, 0]] + pcn[ch[v, 0]]] if ch[v, 0] >= 0 else []
+        right = order[pb[ch[v, 1]]:pb[ch[v, 1]] + pcn[ch[v, 1]]] if ch[v, 1] >= 0 else []
+        assert sorted(left) == sorted(srt[:m]) and sorted(right) == sorted(srt[m + 1:])
+        assert all(p[i, d] <= split[v] for i in left) and all(p[i, d] >= split[v] for i in right)
+
+
+def test_nn_vs_bruteforce_knn1_and_vp():
+    """NN = argmin (d2, id) (the plain definition); the same
+    answer as kNN with k = 1 and as the vantage-point tree (three different
+    trees and pruning rules)."""
+    for dim, seed in ((7, 53), (16, 54), (3, 55)):
+        p = ttgen.gaussian_mixture(2500, dim, seed=seed, components=8)
+        p[400:404] = p[9]
+        q = np.concatenate([ttgen.gaussian_mixture(400, dim, seed=seed + 100, components=8), p[:60]])
+        t = oracle.build_nn(p)
+        r = oracle.nn(t, q, stats=True)
+        idx, d2 = r.out
+        bidx, bd2 = brute.nn(q, p)
+        assert np.array_equal(idx, bidx) and np.array_equal(d2, bd2)
+        kidx, kd2 = oracle.knn(oracle.build_kd(p, 8), q, 1).out
+        assert np.array_equal(kidx[:, 0], idx) and np.array_equal(kd2[:, 0], d2)
+        vidx, vd2 = oracle.vp(oracle.build_vp(p), q).out
+        assert np.array_equal(vidx, idx) and np.array_equal(vd2, d2)
+        assert r.visits.max() <= t.n_nodes and r.visits.min() >= 1
+        if dim == 3:  # pruning works: far fewer tests than nodes in low dimension
+            assert r.visits.mean() < 0.1 * t.n_nodes
+
+
+def test_nn_visits_order_invariant_and_lockstep_results():
+    """N-mode visit counts and the order hash do not depend on the point order
+    (P:L1154-1202 N rows); lockstep with majority vote gives the same results
+    (P:L847-849)."""
+    p = ttgen.gaussian_mixture(3000, 7, seed=56, components=6)
+    q = ttgen.gaussian_mixture(900, 7, seed=57, components=6)
+    t = oracle.build_nn(p)
+    r = oracle.nn(t, q, stats=True)
+    perm = ttgen.permutation(len(q), 58)
+    r2 = oracle.nn(t, q[perm], stats=True)
+    assert np.array_equal(r2.visits, r.visits[perm]) and np.array_equal(r2.hash, r.hash[perm])
+    keys = oracle.sort_keys(t, q)
+    sp = oracle.sort_perm(t, q)
+    assert np.array_equal(np.sort(sp), np.arange(len(q))) and np.all(np.diff(keys[sp].astype(np.float64)) >= 0)
+    for qq in (q, q[sp]):
+        idx, d2 = oracle.nn(t, qq).out
+        li, ld, lv, wf = oracle.nn_lockstep(t, qq)
+        assert np.array_equal(li, idx) and np.array_equal(ld, d2)
+        assert np.all(wf >= 1) and np.all(wf <= lv.reshape(-1) .sum() + 1)
+    # sorting makes lockstep warps cheaper (Table 2, P:L2260)
+    wf_s = oracle.nn_lockstep(t, q[sp])[3].mean()
+    wf_u = oracle.nn_lockstep(t, q)[3].mean()
+    assert wf_s < wf_u
