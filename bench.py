@@ -38,8 +38,8 @@ import ttgen  # noqa: E402
 
 METRIC = "points traversed/sec and node visits/sec at 1/2/4/8 B200; % HBM peak"
 # algorithmic bytes per useful visit of each kernel's packed layout
-BYTES_PER_VISIT = {"bh": 32, "pc": 48, "knn": 96, "vp": 80}
-BYTES_PER_POINT_IO = {"bh": 32, "pc": 20, "knn": 28 + 64, "vp": 64 + 8}
+BYTES_PER_VISIT = {"bh": 32, "pc": 48, "knn": 96, "vp": 80, "nn": 48}
+BYTES_PER_POINT_IO = {"bh": 32, "pc": 20, "knn": 28 + 64, "vp": 64 + 8, "nn": 28 + 8}
 L2_FLUSH_BYTES = 512 << 20  # > 126 MB L2
 
 
@@ -49,7 +49,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--workload", choices=["bh", "knn", "vp", "pc", "bh16m", "knn16m", "bhsteps"], default="bh",
+    ap.add_argument("--workload", choices=["bh", "knn", "vp", "pc", "nn", "bh16m", "knn16m", "bhsteps"], default="bh",
                     help="bh/knn/vp/pc: configs[0..3] (weak scaling, M points per rank); "
                          "bh16m/knn16m: configs[4] (16M points split over the ranks, strong scaling); "
                          "bhsteps: full BH time steps (GPU build + sort + force + leapfrog), bodies sharded over the ranks (strong scaling)")
@@ -96,6 +96,13 @@ def make_workload(name: str, world: int, per_rank: int = 0):
         data = ttgen.gaussian_mixture(c["n"], c["dim"], c["seed"])
         q = ttgen.gaussian_mixture(m * world, c["dim"], c["qseed"])
         return dict(cfg=c, workload="knn_1m_7d", data=data, queries=q, m=m, n_data=c["n"])
+    if name == "nn":  # NEXT-3: the paper's NN benchmark on configs[2]'s inputs
+        c = dict(ttgen.CONFIGS["knn_1m_7d"])
+        m = per_rank or c["m"]
+        data = ttgen.gaussian_mixture(c["n"], c["dim"], c["seed"])
+        q = ttgen.gaussian_mixture(m * world, c["dim"], c["qseed"])
+        return dict(cfg=c, workload="nn_1m_7d (point-per-node kd-tree, configs[2] inputs)", data=data, queries=q,
+                    m=m, n_data=c["n"])
     if name == "vp":
         c = dict(ttgen.CONFIGS["vp_1m_16d"])
         m = per_rank or c["m"]
@@ -115,6 +122,8 @@ def host_tree(P, name, w):
         return P.build_oct(w["data"])
     if name == "vp":
         return P.build_vp(w["data"])
+    if name == "nn":
+        return P.build_nn(w["data"])
     return P.build_kd(w["data"], c["leaf"])
 
 
@@ -221,7 +230,7 @@ def load_counts(workload: str, mode: str):
         return None
 
 
-KERNEL_SOURCE = {"bh": "kern_bh.cu", "pc": "kern_pc.cu", "knn": "kern_knn.cu", "vp": "kern_vp.cu"}
+KERNEL_SOURCE = {"bh": "kern_bh.cu", "pc": "kern_pc.cu", "knn": "kern_knn.cu", "vp": "kern_vp.cu", "nn": "kern_nn.cu"}
 
 
 def kernel_sha256(workload: str) -> str:
@@ -255,7 +264,7 @@ def oracle_baseline(name, w, budget_points=None):
     q = w["queries"]
     m = len(q)
     # sample sized for ~10-30 s of CPU work: every frac-th query
-    target = {"bh": 500_000, "knn": 125_000, "vp": 2_000, "pc": 10_000}[name]
+    target = {"bh": 500_000, "knn": 125_000, "vp": 2_000, "pc": 10_000, "nn": 125_000}[name]
     frac = max(1, m // target)
     idx = np.arange(0, m, frac)
     if budget_points:
@@ -273,6 +282,10 @@ def oracle_baseline(name, w, budget_points=None):
         t = oracle.build_vp(w["data"])
         t0 = time.perf_counter()
         oracle.vp(t, q[idx], threads=threads)
+    elif name == "nn":
+        t = oracle.build_nn(w["data"])
+        t0 = time.perf_counter()
+        oracle.nn(t, q[idx], threads=threads)
     else:
         t = oracle.build_kd(w["data"], c["leaf"])
         t0 = time.perf_counter()
@@ -374,6 +387,8 @@ def run_ours(args, rank, world, local_rank):
 
     # a0: tree (rank 0 builds; NCCL broadcast for N > 1) -- timed separately
     t0 = time.perf_counter()
+    if args.device_build and name == "nn":
+        raise SystemExit("--device-build: no GPU builder for the NN point-per-node kd-tree (host build only)")
     if args.device_build:
         # every rank builds the identical tree from the identical points (NEXT-1)
         data_dev = torch.from_numpy(np.ascontiguousarray(w["data"])).to(device)
@@ -407,7 +422,7 @@ def run_ours(args, rank, world, local_rank):
     elif name == "knn":
         out = (torch.zeros((n_all, c["k"]), dtype=torch.int32, device=device),
                torch.zeros((n_all, c["k"]), dtype=torch.float32, device=device))
-    elif name == "vp":
+    elif name in ("vp", "nn"):
         out = (torch.zeros(n_all, dtype=torch.int32, device=device),
                torch.zeros(n_all, dtype=torch.float32, device=device))
     else:
@@ -432,6 +447,9 @@ def run_ours(args, rank, world, local_rank):
         elif name == "vp":
             P.tt_traverse_vp(tree, pts, out_idx=res[0], out_d2=res[1], order=order, mode=args.mode,
                              auto_min_depth=args.auto_min_depth, stats=stats, variant=args.variant)
+        elif name == "nn":
+            P.tt_traverse_nn(tree, pts, out_idx=res[0], out_d2=res[1], order=order, mode=args.mode,
+                             auto_min_depth=args.auto_min_depth, stats=stats)
         else:
             P.tt_traverse_pc(tree, pts, c["radius"], out=res, order=order, mode=args.mode,
                              auto_min_depth=args.auto_min_depth, stats=stats, variant=args.variant)
@@ -518,7 +536,7 @@ def run_ours(args, rank, world, local_rank):
             res_dev = (torch.empty((m, c["k"]), dtype=torch.int32, device=device),
                        torch.empty((m, c["k"]), dtype=torch.float32, device=device))
             res_host = tuple(torch.empty(r.shape, dtype=r.dtype).pin_memory() for r in res_dev)
-        elif name == "vp":
+        elif name in ("vp", "nn"):
             res_dev = (torch.empty(m, dtype=torch.int32, device=device),
                        torch.empty(m, dtype=torch.float32, device=device))
             res_host = tuple(torch.empty(r.shape, dtype=r.dtype).pin_memory() for r in res_dev)
@@ -541,8 +559,9 @@ def run_ours(args, rank, world, local_rank):
                                   mode=args.mode)
                 for h_, d_ in zip(res_host, res_dev):
                     h_.copy_(d_, non_blocking=True)
-            elif name == "vp":
-                P.tt_traverse_vp(tree, q_dev, out_idx=res_dev[0], out_d2=res_dev[1], order=perm, mode=args.mode)
+            elif name in ("vp", "nn"):
+                (P.tt_traverse_vp if name == "vp" else P.tt_traverse_nn)(
+                    tree, q_dev, out_idx=res_dev[0], out_d2=res_dev[1], order=perm, mode=args.mode)
                 for h_, d_ in zip(res_host, res_dev):
                     h_.copy_(d_, non_blocking=True)
             else:
@@ -580,7 +599,7 @@ def run_ours(args, rank, world, local_rank):
     bpv = BYTES_PER_VISIT[name]
     alg_bytes = visits * bpv + m * BYTES_PER_POINT_IO[name]  # per launch on rank 0
     achieved = alg_bytes / (kms / 1e3) / 1e9
-    kernel_name = {"bh": "bh_kernel", "pc": "pc_kernel", "knn": "knn_kernel", "vp": "vp_kernel"}[name]
+    kernel_name = {"bh": "bh_kernel", "pc": "pc_kernel", "knn": "knn_kernel", "vp": "vp_kernel", "nn": "nn_kernel"}[name]
     cnt = load_counts(name, args.mode) if not args.unsorted and args.variant == "autoropes" else None
     clocks = clk.summary()
     sm_mhz = clocks.get("sm_mhz") or float(peaks.get("sm_max_mhz", 1965.0))

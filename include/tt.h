@@ -55,7 +55,8 @@ typedef enum tt_status {
 typedef enum tt_kind {
     TT_KIND_OCT = 1, /* Barnes-Hut oct-tree of bodies     */
     TT_KIND_KD = 2,  /* kd-tree              */
-    TT_KIND_VP = 3   /* vantage-point tree [27]                    */
+    TT_KIND_VP = 3,  /* vantage-point tree [27]                    */
+    TT_KIND_NN = 4   /* point-per-node kd-tree of the NN benchmark */
 } tt_kind;
 
 typedef enum tt_mode {
@@ -71,9 +72,11 @@ typedef void *tt_stream; /* cudaStream_t */
 #define TT_MAX_HEIGHT 48      /* rope-stack capacity bound (levels)            */
 #define TT_MAX_DIM 16         /* point dimensionality supported by the kernels */
 #define TT_MAX_K 32           /* kNN k supported by the kernels                */
+#ifndef TT_BH_POINTS_PER_LANE
 #define TT_BH_POINTS_PER_LANE 2 /* a BH warp tile holds 32*2 = 64 bodies (2 per
                                    lane); its tt_stats warp_* entry covers 64
                                    points (other kernels: 32 points, 1 per lane) */
+#endif
 
 /* ------------------------------------------------------------------------ */
 /* Host-side tree construction (build rules: DESIGN.md R3, R8a, R9, R12).   */
@@ -89,6 +92,10 @@ tt_status tt_build_kd(const float *pts, int64_t n, int32_t dim, int32_t ld, int3
 /* bodies: n rows of (x, y, z, mass). */
 tt_status tt_build_oct(const float *bodies, int64_t n, tt_host_tree **out);
 tt_status tt_build_vp(const float *pts, int64_t n, int32_t dim, int32_t ld, tt_host_tree **out);
+/* NEXT-3 (R21): point-per-node kd-tree -- each node holds the median of its
+ * set on (x[dim], id) along the largest-extent dimension (lowest on ties);
+ * left = the points before it, right = the points after it.              */
+tt_status tt_build_nn(const float *pts, int64_t n, int32_t dim, int32_t ld, tt_host_tree **out);
 void tt_host_tree_free(tt_host_tree *t);
 
 /* Canonical tree description, all arrays in preorder (host memory).  Node
@@ -106,17 +113,18 @@ typedef struct tt_tree_desc {
     const int32_t *level;       /* [n_nodes]                                      */
     const int32_t *pbegin;      /* [n_nodes] first tree-order point of subtree    */
     const int32_t *pcount;      /* [n_nodes] points in subtree                    */
-    /* KD */
+    /* KD (and NN: the split of the node's own point)                        */
     const int32_t *split_dim;   /* [n_nodes] -1 for a leaf                        */
     const float *split;         /* [n_nodes]                                      */
     const float *lo, *hi;       /* [n_nodes * dim] tight bounding boxes           */
     /* OCT */
     const float *com;           /* [n_nodes * 4] centre of mass x,y,z and mass    */
     const int32_t *body;        /* [n_nodes] OCT: body id of a leaf, -1 for a cell;
-                                   VP: id of the node's vantage point            */
+                                   VP: id of the node's vantage point;
+                                   NN: id of the node's own point                */
     double root_center[3];
     double root_side;
-    /* VP */
+    /* VP (NN: in_child = left, out_child = right)                          */
     const int32_t *in_child;    /* [n_nodes] inside child or -1                   */
     const int32_t *out_child;   /* [n_nodes] outside child or -1                  */
     const float *r_in_max;      /* [n_nodes] max distance vp -> inside points     */
@@ -185,7 +193,8 @@ tt_status tt_tree_get_info(const tt_tree *t, tt_tree_info *out);
 /* a1: point sort (§4.4).  Key = where the point's descent of the
  * tree by the build's split rule ends, in tree (preorder) order: kd -> the
  * leaf's first tree-order point; oct -> 63-bit octant path (Morton order,
- * equal to the preorder of leaves); vp -> 2-bit-per-level path code.  A
+ * equal to the preorder of leaves); vp -> 2-bit-per-level path code; nn ->
+ * the same code of the left-iff-x[dim]<split descent.  A
  * stable radix sort of (key, index) gives perm: perm[j] = original index of
  * the j-th point in tree order (ties by index).  pts: device, n rows of `ld`
  * floats (OCT: ld >= 4 or 3).  keys_out (nullable): the keys, in input order.
@@ -202,7 +211,7 @@ tt_status tt_sort_points(const tt_tree *t, const float *pts, int64_t n, int32_t 
  * from one greedy descent: kd -> largest pinned d2 to the points of the leaf
  * the split rule reaches; vp -> smallest distance to a vantage point on the
  * inside-iff-d<=r_in path; tile = the largest over its points.  Oct trees:
- * a plain copy (BH tiles are near-uniform, §4.6).  Traversal results never
+ * and NN trees: a plain copy (BH tiles are near-uniform, §4.6).  Traversal results never
  * depend on the order, only the schedule does.  pts: device, n rows of `ld`
  * floats (the points perm_in indexes); perm_in/perm_out: device [n], may be
  * the same buffer.  Temporary device memory is stream-ordered.            */
@@ -283,6 +292,15 @@ tt_status tt_traverse_knn(const tt_tree *t, const float *q, int64_t n, int32_t l
 
 /* Vantage-point-tree nearest neighbour ([27]): argmin (d2, id). */
 tt_status tt_traverse_vp(const tt_tree *t, const float *q, int64_t n, int32_t ld, int32_t *idx_out,
+                         float *d2_out, const tt_traverse_opts *opts, tt_stream s);
+
+/* NEXT-3: nearest neighbour over the point-per-node kd-tree of the paper's NN
+ * benchmark (tt_build_nn, reading R21): argmin (d2, id), the
+ * same answer as tt_traverse_knn with k = 1 and tt_traverse_vp.  Fig.5
+ * pattern: truncate iff the node's bound > best d2; update with the node's
+ * point; near = q[dim] < split ? left : right; far child bound =
+ * max(bound, rn(rn(q[dim] - split)^2)).  AUTO default threshold 4.       */
+tt_status tt_traverse_nn(const tt_tree *t, const float *q, int64_t n, int32_t ld, int32_t *idx_out,
                          float *d2_out, const tt_traverse_opts *opts, tt_stream s);
 
 /* NEXT-4: one kick-drift update of a Barnes-Hut time step (leapfrog KDK is

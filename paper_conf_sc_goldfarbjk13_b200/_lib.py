@@ -15,13 +15,13 @@ LIB_PATH = os.path.join(HERE, "libtt.so")
 TT_OK = 0
 STATUS = {0: "TT_OK", -1: "TT_ERR_INVALID_ARG", -2: "TT_ERR_CUDA", -3: "TT_ERR_OOM",
           -4: "TT_ERR_TREE_TOO_DEEP", -5: "TT_ERR_KIND_MISMATCH", -6: "TT_ERR_UNSUPPORTED"}
-KIND_OCT, KIND_KD, KIND_VP = 1, 2, 3
+KIND_OCT, KIND_KD, KIND_VP, KIND_NN = 1, 2, 3, 4
 MODE = {"auto": 0, "lockstep": 1, "L": 1, "independent": 2, "N": 2}
 MEM_HOST, MEM_DEVICE = 0, 1
 VARIANT = {"autoropes": 0, "recursive": 1, "stack": 2}
 MAX_HEIGHT, MAX_DIM, MAX_K = 48, 16, 32
 BH_POINTS_PER_LANE = 2
-TILE_POINTS = {"oct": 32 * BH_POINTS_PER_LANE, "kd": 32, "vp": 32}  # points per warp tile (tt_stats warp_*)
+TILE_POINTS = {"oct": 32 * BH_POINTS_PER_LANE, "kd": 32, "vp": 32, "nn": 32}  # points per warp tile (tt_stats warp_*)
 
 
 class TTError(RuntimeError):
@@ -74,6 +74,7 @@ SIGNATURES = {
     "tt_build_kd": (I32, [P, I64, I32, I32, I32, P]),
     "tt_build_oct": (I32, [P, I64, P]),
     "tt_build_vp": (I32, [P, I64, I32, I32, P]),
+    "tt_build_nn": (I32, [P, I64, I32, I32, P]),
     "tt_host_tree_free": (None, [P]),
     "tt_host_tree_desc": (I32, [P, P]),
     "tt_tree_pack_size": (I32, [P, P]),
@@ -94,6 +95,7 @@ SIGNATURES = {
     "tt_traverse_pc": (I32, [P, P, I64, I32, F, P, P, P]),
     "tt_traverse_knn": (I32, [P, P, I64, I32, I32, P, P, P, P]),
     "tt_traverse_vp": (I32, [P, P, I64, I32, P, P, P, P]),
+    "tt_traverse_nn": (I32, [P, P, I64, I32, P, P, P, P]),
     "tt_status_string": (C.c_char_p, [I32]),
     "tt_last_cuda_error": (I32, []),
     "tt_build_info": (C.c_char_p, []),

@@ -1,7 +1,7 @@
 // host_build.cpp -- host tree builders producing the canonical left-biased
 // linearisation (preorder, first child first, rope = index after the subtree;
 // P:L1063-1067, Fig.2).  Build rules are the DESIGN.md readings
-// R3 (kd), R8a/R9 (oct), R12 (vp).  Compiled with -ffp-contract=off so the
+// R3 (kd), R8a/R9 (oct), R12 (vp), R21 (nn).  Compiled with -ffp-contract=off so the
 // fp32 distance used by the vp build is the pinned R0 sequence.
 //
 // Each builder partitions one index array in place: a node owns a contiguous
@@ -210,6 +210,63 @@ void vp_rec(tt_host_tree &t, int32_t b, int32_t e, int lvl, std::vector<float> &
     t.skip[v] = (int32_t)t.level.size();
 }
 
+// ------------------------------------------------------------------ nn (R21)
+// Point-per-node kd-tree (the paper's NN benchmark): the node
+// holds the median of its set on (x[dim], id) along the largest-extent
+// dimension; left = the elements before it, right = those after it.  The
+// node's point goes first in its range so subtrees stay contiguous.
+void nn_rec(tt_host_tree &t, int32_t b, int32_t e, int lvl) {
+    const int D = t.dim;
+    int32_t v = new_node(t, lvl, b, e);
+    const int32_t n = e - b;
+    if (n == 1) {
+        t.body[v] = t.ids[b];
+        t.skip[v] = (int32_t)t.level.size();
+        return;
+    }
+    float lo[TT_MAX_DIM], hi[TT_MAX_DIM];
+    for (int d = 0; d < D; ++d) {
+        lo[d] = std::numeric_limits<float>::infinity();
+        hi[d] = -std::numeric_limits<float>::infinity();
+    }
+    for (int32_t i = b; i < e; ++i) {
+        const float *p = &t.points[(size_t)t.ids[i] * D];
+        for (int d = 0; d < D; ++d) {
+            lo[d] = std::min(lo[d], p[d]);
+            hi[d] = std::max(hi[d], p[d]);
+        }
+    }
+    int sd = 0;
+    float ext = hi[0] - lo[0];
+    for (int d = 1; d < D; ++d) {
+        float x = hi[d] - lo[d];
+        if (x > ext) { ext = x; sd = d; }
+    }
+    const float *P = t.points.data();
+    auto less = [P, D, sd](int32_t a, int32_t c) {
+        float xa = P[(size_t)a * D + sd], xc = P[(size_t)c * D + sd];
+        return xa < xc || (xa == xc && a < c);
+    };
+    const int32_t m = n / 2;
+    std::nth_element(t.ids.begin() + b, t.ids.begin() + b + m, t.ids.begin() + e, less);
+    // the left elements are those before position b+m; move the median to b
+    std::rotate(t.ids.begin() + b, t.ids.begin() + b + m, t.ids.begin() + b + m + 1);
+    const int32_t me = t.ids[b];
+    t.body[v] = me;
+    t.split_dim[v] = sd;
+    t.split[v] = P[(size_t)me * D + sd];
+    if (m > 0) {
+        t.in_child[v] = (int32_t)t.level.size();
+        nn_rec(t, b + 1, b + 1 + m, lvl + 1);
+    }
+    if (n - m - 1 > 0) {
+        t.out_child[v] = (int32_t)t.level.size();
+        nn_rec(t, b + 1 + m, e, lvl + 1);
+    }
+    t.first_child[v] = t.in_child[v] >= 0 ? t.in_child[v] : t.out_child[v];
+    t.skip[v] = (int32_t)t.level.size();
+}
+
 template <class F>
 tt_status guarded(F &&f) {
     try {
@@ -301,6 +358,25 @@ tt_status tt_build_vp(const float *pts, int64_t n, int32_t dim, int32_t ld, tt_h
     });
 }
 
+tt_status tt_build_nn(const float *pts, int64_t n, int32_t dim, int32_t ld, tt_host_tree **out) {
+    if (!pts || !out || n <= 0 || n > INT32_MAX / 2 || dim <= 0 || dim > TT_MAX_DIM || ld < dim)
+        return TT_ERR_INVALID_ARG;
+    return guarded([&] {
+        auto *t = new tt_host_tree();
+        t->kind = TT_KIND_NN;
+        t->dim = dim;
+        t->n_points = n;
+        t->points.resize((size_t)n * dim);
+        for (int64_t i = 0; i < n; ++i)
+            std::memcpy(&t->points[(size_t)i * dim], pts + (size_t)i * ld, sizeof(float) * dim);
+        t->ids.resize((size_t)n);
+        for (int64_t i = 0; i < n; ++i) t->ids[i] = (int32_t)i;
+        nn_rec(*t, 0, (int32_t)n, 0);
+        *out = t;
+        return TT_OK;
+    });
+}
+
 void tt_host_tree_free(tt_host_tree *t) { delete t; }
 
 tt_status tt_host_tree_desc(const tt_host_tree *t, tt_tree_desc *d) {
@@ -329,6 +405,12 @@ tt_status tt_host_tree_desc(const tt_host_tree *t, tt_tree_desc *d) {
         d->body = t->body.data();
         for (int i = 0; i < 3; ++i) d->root_center[i] = t->root_center[i];
         d->root_side = t->root_side;
+    } else if (t->kind == TT_KIND_NN) {
+        d->body = t->body.data();  // the node's point id
+        d->split_dim = t->split_dim.data();
+        d->split = t->split.data();
+        d->in_child = t->in_child.data();    // left
+        d->out_child = t->out_child.data();  // right
     } else {
         d->body = t->body.data();  // vantage point id per node
         d->in_child = t->in_child.data();

@@ -172,18 +172,27 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
             // FADD2 / FMUL2 / FFMA2 for both bodies, each half rounded exactly
             // like the scalar op (rn(g - b) = rn(g + (-b)): negation is exact),
             // so results are bit-identical to the scalar form.
-            static_assert(kBPL == 2, "packed lockstep loop is written for body pairs");
+            static_assert(kBPL % 2 == 0, "packed lockstep loop is written for body pairs");
+            constexpr int NP = kBPL / 2;
             // negated coordinate pairs, formed once per tile: rn(-0 + (-b)) = -b
             // exactly; the opaque -0 addend keeps ptxas from folding this into a
             // negate modifier that re-assembles the pairs every step
             const float nz = opaque_neg_zero(n);  // -0, see sqr2_rn
             const float2 nz2 = make_float2(nz, nz);
-            const float2 nbx = add2_rn(nz2, make_float2(-bd[0].b.x, -bd[1].b.x));
-            const float2 nby = add2_rn(nz2, make_float2(-bd[0].b.y, -bd[1].b.y));
-            const float2 nbz = add2_rn(nz2, make_float2(-bd[0].b.z, -bd[1].b.z));
-            const int self0 = bd[0].self, self1 = bd[1].self;
-            int w0 = bd[0].wait, w1 = bd[1].wait;
-            float2 ax = make_float2(0.f, 0.f), ay = ax, az = ax;
+            float2 nbx[NP], nby[NP], nbz[NP], ax[NP], ay[NP], az[NP];
+            int self[kBPL], w[kBPL];
+#pragma unroll
+            for (int p = 0; p < NP; ++p) {
+                nbx[p] = add2_rn(nz2, make_float2(-bd[2 * p].b.x, -bd[2 * p + 1].b.x));
+                nby[p] = add2_rn(nz2, make_float2(-bd[2 * p].b.y, -bd[2 * p + 1].b.y));
+                nbz[p] = add2_rn(nz2, make_float2(-bd[2 * p].b.z, -bd[2 * p + 1].b.z));
+                ax[p] = ay[p] = az[p] = make_float2(0.f, 0.f);
+            }
+#pragma unroll
+            for (int j = 0; j < kBPL; ++j) {
+                self[j] = bd[j].self;
+                w[j] = bd[j].wait;
+            }
             int cur = 0;
             // kernel parameters pinned in registers for the hot loop (otherwise
             // re-read from the constant bank every iteration)
@@ -207,43 +216,51 @@ __global__ void __launch_bounds__(kBlock) bh_kernel(const tt_bh_params P) {
                     if (STATS) ++steps;
                     const int lvl = t.w;
                     const float dl = EXP_DSQ ? dsq_at(dbits, lvl) : s_dsq[lvl];
-                    const float2 dx = add2_rn(make_float2(g.x, g.x), nbx);
-                    const float2 dy = add2_rn(make_float2(g.y, g.y), nby);
-                    const float2 dz = add2_rn(make_float2(g.z, g.z), nbz);
-                    // rn(rn(rn(dx^2) + rn(dy^2)) + rn(dz^2)): the pinned order (R0)
-                    const float2 drsq = add2_rn(add2_rn(sqr2_rn(dx, nz), sqr2_rn(dy, nz)), sqr2_rn(dz, nz));
-                    const bool a0 = lvl <= w0, a1 = lvl <= w1;
                     const bool cell = t.x >= 0;
-                    const bool o0 = a0 && cell && drsq.x < dl;
-                    const bool o1 = a1 && cell && drsq.y < dl;
-                    if (STATS) {
-                        bd[0].visits += a0;
-                        bd[1].visits += a1;
+                    bool any_open = false;
+#pragma unroll
+                    for (int p = 0; p < NP; ++p) {
+                        const float2 dx = add2_rn(make_float2(g.x, g.x), nbx[p]);
+                        const float2 dy = add2_rn(make_float2(g.y, g.y), nby[p]);
+                        const float2 dz = add2_rn(make_float2(g.z, g.z), nbz[p]);
+                        // rn(rn(rn(dx^2) + rn(dy^2)) + rn(dz^2)): the pinned order (R0)
+                        const float2 drsq = add2_rn(add2_rn(sqr2_rn(dx, nz), sqr2_rn(dy, nz)), sqr2_rn(dz, nz));
+                        const bool a0 = lvl <= w[2 * p], a1 = lvl <= w[2 * p + 1];
+                        const bool o0 = a0 && cell && drsq.x < dl;
+                        const bool o1 = a1 && cell && drsq.y < dl;
+                        if (STATS) {
+                            bd[2 * p].visits += a0;
+                            bd[2 * p + 1].visits += a1;
+                        }
+                        // active ? (open ? follow : wait at lvl) : keep -- as a min
+                        // (an inactive lane has lvl > wait)
+                        w[2 * p] = o0 ? INT_MAX : min(w[2 * p], lvl);
+                        w[2 * p + 1] = o1 ? INT_MAX : min(w[2 * p + 1], lvl);
+                        // branch-free update (some lane almost always interacts)
+                        const float2 mw = make_float2(a0 && !o0 && t.z != self[2 * p] ? g.w : 0.f,
+                                                      a1 && !o1 && t.z != self[2 * p + 1] ? g.w : 0.f);
+                        const float2 r = add2_rn(drsq, e22);
+                        const float2 inv = make_float2(rsqrt_ftz(r.x), rsqrt_ftz(r.y));
+                        const float2 f = mul2_rn(mul2_rn(mw, mul2_rn(inv, inv)), inv);
+                        ax[p] = fma2_rn(f, dx, ax[p]);
+                        ay[p] = fma2_rn(f, dy, ay[p]);
+                        az[p] = fma2_rn(f, dz, az[p]);
+                        any_open = any_open || o0 || o1;
                     }
-                    // active ? (open ? follow : wait at lvl) : keep -- as a min
-                    // (an inactive lane has lvl > wait)
-                    w0 = o0 ? INT_MAX : min(w0, lvl);
-                    w1 = o1 ? INT_MAX : min(w1, lvl);
-                    // branch-free update (some lane almost always interacts)
-                    const float2 mw = make_float2(a0 && !o0 && t.z != self0 ? g.w : 0.f, a1 && !o1 && t.z != self1 ? g.w : 0.f);
-                    const float2 r = add2_rn(drsq, e22);
-                    const float2 inv = make_float2(rsqrt_ftz(r.x), rsqrt_ftz(r.y));
-                    const float2 f = mul2_rn(mul2_rn(mw, mul2_rn(inv, inv)), inv);
-                    ax = fma2_rn(f, dx, ax);
-                    ay = fma2_rn(f, dy, ay);
-                    az = fma2_rn(f, dz, az);
-                    cur = __any_sync(TT_FULL, o0 || o1) ? t.x : t.y;
+                    cur = __any_sync(TT_FULL, any_open) ? t.x : t.y;
                     if (cur == TT_END) break;
                 }
-                // fp32 partials -> fp64 (warp-uniform cadence); the fp64 sums
-                // live in shared memory (12 registers freed for the hot loop)
-                bd[0].acc.X += (double)ax.x;
-                bd[0].acc.Y += (double)ay.x;
-                bd[0].acc.Z += (double)az.x;
-                bd[1].acc.X += (double)ax.y;
-                bd[1].acc.Y += (double)ay.y;
-                bd[1].acc.Z += (double)az.y;
-                ax = ay = az = make_float2(0.f, 0.f);
+                // fp32 partials -> fp64 (warp-uniform cadence)
+#pragma unroll
+                for (int p = 0; p < NP; ++p) {
+                    bd[2 * p].acc.X += (double)ax[p].x;
+                    bd[2 * p].acc.Y += (double)ay[p].x;
+                    bd[2 * p].acc.Z += (double)az[p].x;
+                    bd[2 * p + 1].acc.X += (double)ax[p].y;
+                    bd[2 * p + 1].acc.Y += (double)ay[p].y;
+                    bd[2 * p + 1].acc.Z += (double)az[p].y;
+                    ax[p] = ay[p] = az[p] = make_float2(0.f, 0.f);
+                }
                 if (cur == TT_END) break;
             }
             fetches = steps;

@@ -12,7 +12,9 @@
 //        radius when the leaf holds >= k points: the ball the search must
 //        cover);
 //   vp : the smallest distance to a vantage point on the inside-iff-d<=r_in
-//        path (the tau the search starts pruning with).
+//        path (the tau the search starts pruning with);
+//   nn : the smallest pinned d2 to a node point on the left-iff-x<split
+//        path (likewise).
 // tile key = the largest estimate of its points (a lockstep warp runs as long
 // as its most expensive lane).  Whole tiles move; the points inside a tile
 // and the ragged last tile stay where they are, so the similarity of the
@@ -66,6 +68,21 @@ __device__ __forceinline__ float vp_cost(const tt_vp_rec *rec, const float *vpt,
     return best;
 }
 
+template <int DIM>
+__device__ __forceinline__ float nn_cost(const tt_nn_rec *rec, const float *vpt, int dp, const float (&q)[DIM]) {
+    int cur = 0;
+    float best = __int_as_float(0x7f800000);
+    for (int l = 0; l < TT_MAX_HEIGHT + 2 && cur >= 0; ++l) {
+        const int4 t = __ldg(reinterpret_cast<const int4 *>(rec + cur));
+        float v[DIM];
+        load_row_nc<DIM>(v, vpt + (size_t)cur * dp);
+        best = fminf(best, pinned_d2<DIM>(q, v));
+        if (t.w < 0) break;
+        cur = select_dim<DIM>(q, t.w) < __int_as_float(t.z) ? t.x : t.y;
+    }
+    return best;
+}
+
 // one warp per tile: key = bits of the largest (non-negative) estimate
 template <int DIM>
 __global__ void tile_cost_kernel(int kind, const void *rec, const float *tpts, const float *vpt, int dp,
@@ -80,8 +97,9 @@ __global__ void tile_cost_kernel(int kind, const void *rec, const float *tpts, c
             if (pos >= n) break;
             float q[DIM];
             load_query<DIM>(q, pts, perm[pos], ld);
-            const float e = kind == TT_KIND_KD ? kd_cost<DIM>(static_cast<const tt_kd_rec *>(rec), tpts, dp, q)
-                                               : vp_cost<DIM>(static_cast<const tt_vp_rec *>(rec), vpt, dp, q);
+            const float e = kind == TT_KIND_KD   ? kd_cost<DIM>(static_cast<const tt_kd_rec *>(rec), tpts, dp, q)
+                            : kind == TT_KIND_NN ? nn_cost<DIM>(static_cast<const tt_nn_rec *>(rec), vpt, dp, q)
+                                                 : vp_cost<DIM>(static_cast<const tt_vp_rec *>(rec), vpt, dp, q);
             c = fmaxf(c, e);
         }
         // non-negative floats order like their bit patterns (+inf included)

@@ -8,7 +8,9 @@
 //   oct: 63-bit octant path through the root cube (fp64 comparisons exactly as
 //        the build partitions bodies) = Morton order = preorder of leaves;
 //   vp : 2-bit-per-level code (inside = 01, outside = 10, end = 00) of the
-//        inside-iff-d<=r_in_max descent; a node sorts before its subtree.
+//        inside-iff-d<=r_in_max descent; a node sorts before its subtree;
+//   nn : the same code (left = 01, right = 10) of the left-iff-x[dim]<split
+//        descent of the point-per-node kd-tree.
 // A stable LSD radix sort of (key, index) then yields perm (ties by index).
 // The key kernel is ours; the radix sort is CUB's DeviceRadixSort (a library
 // sort primitive, like a library GEMM).
@@ -87,6 +89,26 @@ __global__ void vp_keys(const tt_vp_rec *rec, const float *vpt, int dp, const fl
     }
 }
 
+template <int DIM>
+__global__ void nn_keys(const tt_nn_rec *rec, const float *pts, long long n, int ld, unsigned long long *keys) {
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
+        float q[DIM];
+        load_query<DIM>(q, pts, i, ld);
+        int cur = 0;
+        unsigned long long code = 0;
+        for (int l = 0; l < 31; ++l) {
+            const int4 t = __ldg(reinterpret_cast<const int4 *>(rec + cur));
+            if (t.w < 0) break;
+            const bool left = select_dim<DIM>(q, t.w) < __int_as_float(t.z);
+            const int nx = left ? t.x : t.y;
+            if (nx < 0) break;
+            code |= (unsigned long long)(left ? 1 : 2) << (62 - 2 * l);
+            cur = nx;
+        }
+        keys[i] = code;
+    }
+}
+
 int grid_for(long long n) {
     long long g = (n + 255) / 256;
     if (g > 148 * 16) g = 148 * 16;
@@ -98,6 +120,8 @@ void launch_keys(const tt_tree *t, const float *pts, long long n, int ld, unsign
                  cudaStream_t s) {
     if (t->hdr.kind == TT_KIND_KD)
         kd_keys<DIM><<<grid_for(n), 256, 0, s>>>(static_cast<const tt_kd_rec *>(t->dev.rec), pts, n, ld, keys);
+    else if (t->hdr.kind == TT_KIND_NN)
+        nn_keys<DIM><<<grid_for(n), 256, 0, s>>>(static_cast<const tt_nn_rec *>(t->dev.rec), pts, n, ld, keys);
     else
         vp_keys<DIM><<<grid_for(n), 256, 0, s>>>(static_cast<const tt_vp_rec *>(t->dev.rec), t->dev.vpt, t->hdr.dp,
                                                 pts, n, ld, keys);

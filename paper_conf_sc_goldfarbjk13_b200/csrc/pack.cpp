@@ -28,12 +28,13 @@ int dim_padded(int dim) { return (dim + 3) & ~3; }
 int stage_bytes_per_node(int kind, int dp) {
     if (kind == TT_KIND_OCT) return 32;
     if (kind == TT_KIND_KD) return 32 + 8 * dp;
-    return 16 + 4 * dp;
+    return 16 + 4 * dp;  // VP, NN
 }
 
 int validate(const tt_tree_desc *d) {
     if (!d) return TT_ERR_INVALID_ARG;
-    if (d->kind != TT_KIND_OCT && d->kind != TT_KIND_KD && d->kind != TT_KIND_VP) return TT_ERR_INVALID_ARG;
+    if (d->kind != TT_KIND_OCT && d->kind != TT_KIND_KD && d->kind != TT_KIND_VP && d->kind != TT_KIND_NN)
+        return TT_ERR_INVALID_ARG;
     if (d->n_nodes <= 0 || d->n_nodes > INT32_MAX - 1 || d->n_points <= 0 || d->n_points > INT32_MAX - 1)
         return TT_ERR_INVALID_ARG;
     if (d->dim <= 0) return TT_ERR_INVALID_ARG;
@@ -48,6 +49,9 @@ int validate(const tt_tree_desc *d) {
     if (d->kind == TT_KIND_VP &&
         (!d->body || !d->in_child || !d->out_child || !d->r_in_max || !d->r_out_min || !d->points))
         return TT_ERR_INVALID_ARG;
+    if (d->kind == TT_KIND_NN &&
+        (!d->body || !d->in_child || !d->out_child || !d->split || !d->split_dim || !d->points))
+        return TT_ERR_INVALID_ARG;
     const int64_t N = d->n_nodes;
     for (int64_t v = 0; v < N; ++v) {
         if (d->skip[v] <= v || d->skip[v] > N) return TT_ERR_INVALID_ARG;
@@ -59,9 +63,13 @@ int validate(const tt_tree_desc *d) {
             if (d->split_dim[v] >= d->dim) return TT_ERR_INVALID_ARG;
             if (d->first_child[v] >= 0 && d->skip[d->first_child[v]] >= d->skip[v]) return TT_ERR_INVALID_ARG;
         }
-        if (d->kind == TT_KIND_VP) {
+        if (d->kind == TT_KIND_VP || d->kind == TT_KIND_NN) {
             if (d->body[v] < 0 || d->body[v] >= d->n_points) return TT_ERR_INVALID_ARG;
             if (d->in_child[v] >= N || d->out_child[v] >= N) return TT_ERR_INVALID_ARG;
+        }
+        if (d->kind == TT_KIND_NN) {
+            const bool inner = d->in_child[v] >= 0 || d->out_child[v] >= 0;
+            if (inner != (d->split_dim[v] >= 0) || d->split_dim[v] >= d->dim) return TT_ERR_INVALID_ARG;
         }
         if (d->kind == TT_KIND_OCT && d->body[v] >= d->n_points) return TT_ERR_INVALID_ARG;
         if (d->pbegin[v] < 0 || d->pcount[v] < 0 || (int64_t)d->pbegin[v] + d->pcount[v] > d->n_points)
@@ -100,7 +108,7 @@ void plan(const tt_tree_desc *d, tt_blob_header &h, std::vector<int32_t> *newidx
     }
     h.top_levels = L;
     h.top_count = (int32_t)acc;
-    h.rec_bytes = d->kind == TT_KIND_VP ? 16 : 32;
+    h.rec_bytes = (d->kind == TT_KIND_VP || d->kind == TT_KIND_NN) ? 16 : 32;
     uint64_t off = align256(sizeof(tt_blob_header));
     h.off_rec = off;
     off = align256(off + (uint64_t)d->n_nodes * h.rec_bytes);
@@ -113,7 +121,7 @@ void plan(const tt_tree_desc *d, tt_blob_header &h, std::vector<int32_t> *newidx
         off = align256(off + (uint64_t)d->n_points * sizeof(int32_t));
         h.off_cbox = off;
         off = align256(off + (uint64_t)d->n_nodes * 4 * h.dp * sizeof(float));
-    } else if (d->kind == TT_KIND_VP) {
+    } else if (d->kind == TT_KIND_VP || d->kind == TT_KIND_NN) {
         h.off_vpt = off;
         off = align256(off + (uint64_t)d->n_nodes * h.dp * sizeof(float));
         h.off_pid = off;
@@ -215,6 +223,20 @@ int tt_pack_impl(const tt_tree_desc *d, void *blob, size_t bytes) {
             const int32_t id = d->tree_order[j];
             pid[j] = id;
             std::memcpy(pts + (size_t)j * h.dp, d->points + (size_t)id * d->dim, sizeof(float) * d->dim);
+        }
+    } else if (d->kind == TT_KIND_NN) {
+        auto *rec = reinterpret_cast<tt_nn_rec *>(base + h.off_rec);
+        auto *vpt = reinterpret_cast<float *>(base + h.off_vpt);
+        auto *pid = reinterpret_cast<int32_t *>(base + h.off_pid);
+        for (int64_t v = 0; v < N; ++v) {
+            const int32_t nv = nx[(size_t)v];
+            tt_nn_rec &r = rec[nv];
+            r.left = map(d->in_child[v]);
+            r.right = map(d->out_child[v]);
+            r.split = d->split[v];
+            r.dim = d->split_dim[v];
+            pid[nv] = d->body[v];
+            std::memcpy(vpt + (size_t)nv * h.dp, d->points + (size_t)d->body[v] * d->dim, sizeof(float) * d->dim);
         }
     } else {
         auto *rec = reinterpret_cast<tt_vp_rec *>(base + h.off_rec);

@@ -38,11 +38,11 @@ bool dim_supported(int d) { return (d >= 1 && d <= 8) || d == 16; }
 
 // Default AUTO thresholds (levels of common tree path for lockstep), see
 // tt_traverse_opts.auto_min_depth and DESIGN.md §4.5.
-constexpr int kAutoBH = 3, kAutoPC = 255, kAutoKNN = 4, kAutoVP = 4;
+constexpr int kAutoBH = 3, kAutoPC = 255, kAutoKNN = 4, kAutoVP = 4, kAutoNN = 4;
 
 // Shared-memory budgets for the staged top levels, per kernel (bytes/node):
 // the budget trades staged levels against occupancy.
-constexpr int kTopBH = 32 * 1024, kTopPC = 32 * 1024, kTopKNN = 16 * 1024, kTopVP = 4 * 1024;
+constexpr int kTopBH = 32 * 1024, kTopPC = 32 * 1024, kTopKNN = 16 * 1024, kTopVP = 4 * 1024, kTopNN = 8 * 1024;
 
 tt_status setup_common(const tt_tree *t, int kind, int64_t n, const tt_traverse_opts *o, int default_amd,
                        int stage_bytes_per_node, int stage_budget, tt_common_params &c, tt_launch_cfg &cfg,
@@ -345,6 +345,7 @@ tt_status tt_traverse_bh(const tt_tree *t, const float *bodies, const int32_t *s
 
 tt_status tt_traverse_pc(const tt_tree *t, const float *q, int64_t n, int32_t ld, float radius, uint32_t *count_out,
                          const tt_traverse_opts *opts, tt_stream s) {
+    if (!t) return TT_ERR_INVALID_ARG;  // (the staging size below reads t->hdr)
     tt_pc_params p;
     tt_launch_cfg cfg;
     tt_status st = setup_common(t, TT_KIND_KD, n, opts, kAutoPC, 32 + 8 * t->hdr.dp, kTopPC, p.c, cfg, s);
@@ -367,6 +368,7 @@ tt_status tt_traverse_pc(const tt_tree *t, const float *q, int64_t n, int32_t ld
 
 tt_status tt_traverse_knn(const tt_tree *t, const float *q, int64_t n, int32_t ld, int32_t k, int32_t *idx_out,
                           float *d2_out, const tt_traverse_opts *opts, tt_stream s) {
+    if (!t) return TT_ERR_INVALID_ARG;  // (the staging size below reads t->hdr)
     tt_knn_params p;
     tt_launch_cfg cfg;
     tt_status st = setup_common(t, TT_KIND_KD, n, opts, kAutoKNN, 32 + 16 * t->hdr.dp, kTopKNN, p.c, cfg, s);
@@ -391,6 +393,7 @@ tt_status tt_traverse_knn(const tt_tree *t, const float *q, int64_t n, int32_t l
 
 tt_status tt_traverse_vp(const tt_tree *t, const float *q, int64_t n, int32_t ld, int32_t *idx_out, float *d2_out,
                          const tt_traverse_opts *opts, tt_stream s) {
+    if (!t) return TT_ERR_INVALID_ARG;  // (the staging size below reads t->hdr)
     tt_vp_params p;
     tt_launch_cfg cfg;
     tt_status st = setup_common(t, TT_KIND_VP, n, opts, kAutoVP, 16 + 4 * t->hdr.dp, kTopVP, p.c, cfg, s);
@@ -408,6 +411,27 @@ tt_status tt_traverse_vp(const tt_tree *t, const float *q, int64_t n, int32_t ld
     if (cfg.variant == TT_VARIANT_STACK) return TT_ERR_UNSUPPORTED;  // guided kernels already keep rope stacks
     return finish_launch(cfg.variant == TT_VARIANT_RECURSIVE ? tt_launch_vp_recursive(p, t->hdr.dim, cfg)
                                                             : tt_launch_vp(p, t->hdr.dim, cfg));
+}
+
+tt_status tt_traverse_nn(const tt_tree *t, const float *q, int64_t n, int32_t ld, int32_t *idx_out, float *d2_out,
+                         const tt_traverse_opts *opts, tt_stream s) {
+    if (!t) return TT_ERR_INVALID_ARG;  // (the staging size below reads t->hdr)
+    tt_nn_params p;
+    tt_launch_cfg cfg;
+    tt_status st = setup_common(t, TT_KIND_NN, n, opts, kAutoNN, 16 + 4 * t->hdr.dp, kTopNN, p.c, cfg, s);
+    if (st != TT_OK) return st;
+    if (ld < t->hdr.dim) return TT_ERR_INVALID_ARG;
+    if (!dim_supported(t->hdr.dim)) return TT_ERR_UNSUPPORTED;
+    if (cfg.variant != TT_VARIANT_AUTOROPES) return TT_ERR_UNSUPPORTED;  // no recursive / stack variant for NN
+    if (n == 0) return TT_OK;
+    if (!q || !idx_out || !d2_out) return TT_ERR_INVALID_ARG;
+    st = have_device();
+    if (st != TT_OK) return st;
+    p.q = q;
+    p.ld = ld;
+    p.idx = idx_out;
+    p.d2 = d2_out;
+    return finish_launch(tt_launch_nn(p, t->hdr.dim, cfg));
 }
 
 tt_status tt_kick_drift(float *bodies, float *vel, const float *acc, int64_t n, float dt_kick, float dt_drift,

@@ -28,6 +28,8 @@
 //      + box[2*dp] floats (lo[dp], hi[dp]) in a separate array
 // VP:  t = {in | -1, out | -1, r_in_max (float bits), r_out_min (float bits)}
 //      + vpt[dp] vantage coordinates and pid (vantage point's original id)
+// NN:  t = {left | -1, right | -1, split (float bits), split_dim | -1}
+//      + vpt[dp] the node's point and pid (its original id)
 // ---------------------------------------------------------------------------
 struct alignas(16) tt_oct_rec {
     float gx, gy, gz, gm;
@@ -44,7 +46,13 @@ struct alignas(16) tt_vp_rec {
 };
 static_assert(sizeof(tt_oct_rec) == 32, "oct record = one 32-B sector");
 static_assert(sizeof(tt_kd_rec) == 32, "kd record = one 32-B sector");
+struct alignas(16) tt_nn_rec {
+    int32_t left, right;
+    float split;
+    int32_t dim;
+};
 static_assert(sizeof(tt_vp_rec) == 16, "vp header = one 128-bit group");
+static_assert(sizeof(tt_nn_rec) == 16, "nn header = one 128-bit group");
 
 // Blob = header + sections, every section 256-byte aligned, offsets relative to
 // the blob start (position independent: the blob can be broadcast as bytes).
@@ -68,8 +76,8 @@ struct tt_dev_tree {
     const void *rec;      // records, top nodes first
     const float *box;     // KD: [n_nodes][2*dp]
     const float *pts;     // KD: [n_points][dp] tree order
-    const int32_t *pid;   // KD: [n_points]; VP: [n_nodes]
-    const float *vpt;     // VP: [n_nodes][dp]
+    const int32_t *pid;   // KD: [n_points]; VP, NN: [n_nodes]
+    const float *vpt;     // VP, NN: [n_nodes][dp] the node's point
     const float *cbox;    // KD: [n_nodes][2][2*dp] boxes of the two children
 };
 
@@ -123,6 +131,9 @@ struct tt_vp_params {
     float *d2;
 };
 
+// NN: same argument block as VP
+typedef tt_vp_params tt_nn_params;
+
 // Host-side handle.
 struct tt_tree {
     tt_blob_header hdr;
@@ -144,6 +155,7 @@ int tt_launch_bh(const tt_bh_params &p, const tt_launch_cfg &cfg);
 int tt_launch_pc(const tt_pc_params &p, int dim, const tt_launch_cfg &cfg);
 int tt_launch_knn(const tt_knn_params &p, int dim, const tt_launch_cfg &cfg);
 int tt_launch_vp(const tt_vp_params &p, int dim, const tt_launch_cfg &cfg);
+int tt_launch_nn(const tt_nn_params &p, int dim, const tt_launch_cfg &cfg);
 // naive recursive baseline (kern_recursive.cu)
 int tt_launch_bh_recursive(const tt_bh_params &p, const tt_launch_cfg &cfg);
 int tt_launch_pc_recursive(const tt_pc_params &p, int dim, const tt_launch_cfg &cfg);

@@ -22,9 +22,9 @@ from ._lib import TTError, check
 
 __all__ = [
     "HostTree", "Tree", "Stats", "TTError",
-    "build_kd", "build_oct", "build_vp", "tt_tree_pack", "tt_tree_from_blob", "tt_tree_upload",
+    "build_kd", "build_oct", "build_vp", "build_nn", "tt_tree_pack", "tt_tree_from_blob", "tt_tree_upload",
     "tt_build_oct_device", "tt_build_kd_device", "tt_build_vp_device", "tt_tree_download",
-    "tt_sort_points", "tt_schedule_tiles", "tt_traverse_bh", "tt_traverse_pc", "tt_traverse_knn", "tt_traverse_vp",
+    "tt_sort_points", "tt_schedule_tiles", "tt_traverse_bh", "tt_traverse_pc", "tt_traverse_knn", "tt_traverse_vp", "tt_traverse_nn",
     "build_info",
 ]
 
@@ -54,7 +54,7 @@ class HostTree:
         self._keep = keepalive
         self.desc = L.tt_tree_desc()
         check(L.load().tt_host_tree_desc(self._h, C.byref(self.desc)), "tt_host_tree_desc")
-        self.kind = {1: "oct", 2: "kd", 3: "vp"}[self.desc.kind]
+        self.kind = {1: "oct", 2: "kd", 3: "vp", 4: "nn"}[self.desc.kind]
         self.dim = self.desc.dim
         self.height = self.desc.height
         self.n_nodes = self.desc.n_nodes
@@ -128,6 +128,14 @@ def build_vp(pts: np.ndarray) -> HostTree:
     return HostTree(h)
 
 
+def build_nn(pts: np.ndarray) -> HostTree:
+    """NEXT-3: point-per-node kd-tree of the paper's NN benchmark (R21)."""
+    a = _host_points(pts)
+    h = C.c_void_p()
+    check(L.load().tt_build_nn(_np_ptr(a), a.shape[0], a.shape[1], a.shape[1], C.byref(h)), "tt_build_nn")
+    return HostTree(h)
+
+
 def tt_tree_pack(host: HostTree) -> np.ndarray:
     """a0 on the host: the position-independent device blob (uint8 array)."""
     lib = L.load()
@@ -146,7 +154,7 @@ class Tree:
         self._h = handle
         info = L.tt_tree_info()
         check(L.load().tt_tree_get_info(self._h, C.byref(info)), "tt_tree_get_info")
-        self.kind = {1: "oct", 2: "kd", 3: "vp"}[info.kind]
+        self.kind = {1: "oct", 2: "kd", 3: "vp", 4: "nn"}[info.kind]
         self.dim = info.dim
         self.height = info.height
         self.n_nodes = info.n_nodes
@@ -377,5 +385,22 @@ def tt_traverse_vp(tree: Tree, q: torch.Tensor, out_idx: torch.Tensor | None = N
     o, keep = _opts(mode, auto_min_depth, order, stats, n, variant)
     check(L.load().tt_traverse_vp(tree._h, q.data_ptr(), _lanes(order, n), q.stride(0), out_idx.data_ptr(), out_d2.data_ptr(),
                                   C.byref(o), C.c_void_p(_stream_handle(stream))), "tt_traverse_vp")
+    del keep
+    return out_idx, out_d2
+
+
+def tt_traverse_nn(tree: Tree, q: torch.Tensor, out_idx: torch.Tensor | None = None,
+                   out_d2: torch.Tensor | None = None, order: torch.Tensor | None = None, mode="auto",
+                   auto_min_depth: int | None = None, stats: Stats | None = None, stream=None):
+    """NEXT-3: nearest neighbour over the point-per-node kd-tree (tt_build_nn)."""
+    _dev(q, torch.float32, "q", tree.dim)
+    n = q.shape[0]
+    if out_idx is None:
+        out_idx = torch.empty(n, dtype=torch.int32, device=q.device)
+    if out_d2 is None:
+        out_d2 = torch.empty(n, dtype=torch.float32, device=q.device)
+    o, keep = _opts(mode, auto_min_depth, order, stats, n, "autoropes")
+    check(L.load().tt_traverse_nn(tree._h, q.data_ptr(), _lanes(order, n), q.stride(0), out_idx.data_ptr(),
+                                  out_d2.data_ptr(), C.byref(o), C.c_void_p(_stream_handle(stream))), "tt_traverse_nn")
     del keep
     return out_idx, out_d2

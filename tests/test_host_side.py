@@ -83,6 +83,55 @@ def test_vp_builder_matches_oracle():
     assert np.array_equal(h.array("skip"), o.i64(oracle.F_SKIP))
 
 
+@pytest.mark.parametrize("n,dim", [(3001, 7), (1, 3), (2, 16), (700, 2)])
+def test_nn_builder_matches_oracle(n, dim):
+    """NEXT-3 point-per-node kd-tree (R21): libtt's builder vs the oracle's."""
+    p = ttgen.gaussian_mixture(n, dim, seed=105, components=4)
+    if n > 100:
+        p[20:25] = p[60]
+    h, o = P.build_nn(p), oracle.build_nn(p)
+    assert h.kind == "nn" and h.n_nodes == o.n_nodes == n and h.height == o.height
+    assert np.array_equal(h.array("body"), o.i64(oracle.F_VP))
+    assert np.array_equal(h.array("split_dim"), o.i64(oracle.F_SPLITDIM))
+    sd = o.i64(oracle.F_SPLITDIM) >= 0
+    assert np.array_equal(h.array("split")[sd], o.f32(oracle.F_SPLIT)[sd])
+    ch = o.children()
+    assert np.array_equal(h.array("in_child"), ch[:, 0])
+    assert np.array_equal(h.array("out_child"), ch[:, 1])
+    assert np.array_equal(h.array("skip"), o.i64(oracle.F_SKIP))
+    assert np.array_equal(h.array("level"), o.i64(oracle.F_LEVEL))
+    assert np.array_equal(h.array("tree_order"), o.tree_order())
+
+
+def test_nn_blob_records_and_points():
+    p = ttgen.gaussian_mixture(2500, 7, seed=106, components=4)
+    h = P.build_nn(p)
+    blob = h.pack()
+    hd = {k: (int(v) if np.ndim(v) == 0 else v) for k, v in
+          zip(HDR.names, np.frombuffer(blob[:HDR.itemsize].tobytes(), HDR)[0])}
+    assert hd["kind"] == 4 and hd["rec_bytes"] == 16 and hd["dp"] == 8 and hd["n_nodes"] == 2500
+    N = h.n_nodes
+    rec = np.frombuffer(blob[hd["off_rec"]:hd["off_rec"] + 16 * N].tobytes(),
+                        dtype=[("l", "<i4"), ("r", "<i4"), ("split", "<f4"), ("dim", "<i4")])
+    pts = np.frombuffer(blob[hd["off_vpt"]:hd["off_vpt"] + 32 * N].tobytes(), "<f4").reshape(N, 8)
+    pid = np.frombuffer(blob[hd["off_pid"]:hd["off_pid"] + 4 * N].tobytes(), "<i4")
+    assert np.array_equal(np.sort(pid), np.arange(N))
+    assert np.array_equal(pts[:, :7], p[pid]) and np.all(pts[:, 7] == 0)
+    # walk the device numbering from the root: every subtree satisfies the split rule
+    stack, seen = [0], 0
+    while stack:
+        v = stack.pop()
+        seen += 1
+        for c, side in ((rec["l"][v], 0), (rec["r"][v], 1)):
+            if c < 0:
+                continue
+            assert rec["dim"][v] >= 0
+            d = rec["dim"][v]
+            assert (p[pid[c], d] <= rec["split"][v]) if side == 0 else (p[pid[c], d] >= rec["split"][v])
+            stack.append(c)
+    assert seen == N
+
+
 # ------------------------------------------------------------- blob layout
 HDR = np.dtype([("magic", "<u4"), ("version", "<u4"), ("kind", "<i4"), ("dim", "<i4"), ("dp", "<i4"),
                 ("height", "<i4"), ("leaf_size", "<i4"), ("top_levels", "<i4"), ("top_count", "<i4"),
