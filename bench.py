@@ -61,6 +61,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--points-per-rank", type=int, default=0, help="override M (testing)")
     ap.add_argument("--auto-min-depth", type=int, default=None, help="AUTO-mode threshold (default: kernel's)")
+    ap.add_argument("--switch-below", type=int, default=0,
+                    help="kNN: dynamic L->N switch when fewer lanes are active (NEXT-3; 0 = never)")
     ap.add_argument("--device-build", action="store_true",
                     help="build the tree on the GPU (tt_build_oct_device / tt_build_kd_device) instead of host "
                          "build + upload")
@@ -443,7 +445,8 @@ def run_ours(args, rank, world, local_rank):
                              variant=args.variant)
         elif name == "knn":
             P.tt_traverse_knn(tree, pts, c["k"], out_idx=res[0], out_d2=res[1], order=order, mode=args.mode,
-                              auto_min_depth=args.auto_min_depth, stats=stats, variant=args.variant)
+                              auto_min_depth=args.auto_min_depth, stats=stats, variant=args.variant,
+                              switch_below=args.switch_below)
         elif name == "vp":
             P.tt_traverse_vp(tree, pts, out_idx=res[0], out_d2=res[1], order=order, mode=args.mode,
                              auto_min_depth=args.auto_min_depth, stats=stats, variant=args.variant)
@@ -647,6 +650,7 @@ def run_ours(args, rank, world, local_rank):
         "config": {"workload": w["workload"], "points_per_rank": m, "global_points": n_all,
                    "tree_points": w["n_data"], "mode": args.mode, "sorted": not args.unsorted,
                    "tile_schedule": "longest-first" if lpt else "in-order",
+                   **({"switch_below": args.switch_below} if args.switch_below else {}),
                    "auto_min_depth": args.auto_min_depth, "variant": args.variant,
                    "parallelism": f"dp{world} (points sharded, tree replicated)",
                    "l2": "flushed between timed steps (512 MiB write)",

@@ -93,8 +93,9 @@ tt_status tt_build_kd(const float *pts, int64_t n, int32_t dim, int32_t ld, int3
 tt_status tt_build_oct(const float *bodies, int64_t n, tt_host_tree **out);
 tt_status tt_build_vp(const float *pts, int64_t n, int32_t dim, int32_t ld, tt_host_tree **out);
 /* NEXT-3 (R21): point-per-node kd-tree -- each node holds the median of its
- * set on (x[dim], id) along the largest-extent dimension (lowest on ties);
- * left = the points before it, right = the points after it.              */
+ * set on (x[dim], id) along the largest-extent dimension (lowest on ties)
+ * and the tight box of its subtree; left = the points before it, right =
+ * the points after it.                                                    */
 tt_status tt_build_nn(const float *pts, int64_t n, int32_t dim, int32_t ld, tt_host_tree **out);
 void tt_host_tree_free(tt_host_tree *t);
 
@@ -116,7 +117,7 @@ typedef struct tt_tree_desc {
     /* KD (and NN: the split of the node's own point)                        */
     const int32_t *split_dim;   /* [n_nodes] -1 for a leaf                        */
     const float *split;         /* [n_nodes]                                      */
-    const float *lo, *hi;       /* [n_nodes * dim] tight bounding boxes           */
+    const float *lo, *hi;       /* [n_nodes * dim] tight bounding boxes (KD, NN)  */
     /* OCT */
     const float *com;           /* [n_nodes * 4] centre of mass x,y,z and mass    */
     const int32_t *body;        /* [n_nodes] OCT: body id of a leaf, -1 for a cell;
@@ -227,7 +228,8 @@ typedef struct tt_stats {
                                 (lockstep: one per step; independent: per lane);
                                 T = 32 points per tile (BH: 32*TT_BH_POINTS_PER_LANE) */
     uint32_t *warp_steps;    /* [ceil(n/T)] loop iterations of the warp          */
-    uint8_t *warp_mode;      /* [ceil(n/T)] 1 = lockstep, 2 = independent       */
+    uint8_t *warp_mode;      /* [ceil(n/T)] 1 = lockstep, 2 = independent,
+                                3 = lockstep switched to independent          */
 } tt_stats;
 
 typedef struct tt_traverse_opts {
@@ -258,6 +260,15 @@ typedef struct tt_traverse_opts {
                                 stack per warp in shared memory;
                                 AUTO = BH lockstep, PC independent; 32-point
                                 warp tiles                                     */
+    int32_t switch_below;    /* NEXT-3 dynamic L->N switching (kNN only, else
+                                must be 0): a lockstep warp whose active lanes at
+                                a node number fewer than this converts its warp
+                                rope stack into per-lane stacks (each lane keeps
+                                the entries whose mask holds it, in order) and
+                                finishes the tile independently; tt_stats
+                                warp_mode = 3 for such tiles.  0 = never (default);
+                                33 = at the root (= independent).  Results never
+                                depend on it.                                   */
 } tt_traverse_opts;
 
 typedef enum tt_variant {
@@ -297,9 +308,9 @@ tt_status tt_traverse_vp(const tt_tree *t, const float *q, int64_t n, int32_t ld
 /* NEXT-3: nearest neighbour over the point-per-node kd-tree of the paper's NN
  * benchmark (tt_build_nn, reading R21): argmin (d2, id), the
  * same answer as tt_traverse_knn with k = 1 and tt_traverse_vp.  Fig.5
- * pattern: truncate iff the node's bound > best d2; update with the node's
- * point; near = q[dim] < split ? left : right; far child bound =
- * max(bound, rn(rn(q[dim] - split)^2)).  AUTO default threshold 4.       */
+ * pattern: truncate iff the pinned distance to the node's tight box > best
+ * d2; update with the node's point; near = q[dim] < split ? left : right,
+ * visited first.  AUTO default threshold 4.                              */
 tt_status tt_traverse_nn(const tt_tree *t, const float *q, int64_t n, int32_t ld, int32_t *idx_out,
                          float *d2_out, const tt_traverse_opts *opts, tt_stream s);
 

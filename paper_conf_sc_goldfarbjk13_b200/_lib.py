@@ -65,7 +65,7 @@ class tt_stats(C.Structure):
 class tt_traverse_opts(C.Structure):
     _fields_ = [("mode", C.c_int32), ("auto_min_depth", C.c_int32), ("order", C.c_void_p),
                 ("stats", C.c_void_p), ("block_threads", C.c_int32), ("ctas_per_sm", C.c_int32),
-                ("variant", C.c_int32)]
+                ("variant", C.c_int32), ("switch_below", C.c_int32)]
 
 
 # name -> (restype, argtypes); every function declared in include/tt.h

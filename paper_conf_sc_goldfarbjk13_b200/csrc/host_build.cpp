@@ -214,16 +214,12 @@ void vp_rec(tt_host_tree &t, int32_t b, int32_t e, int lvl, std::vector<float> &
 // Point-per-node kd-tree (the paper's NN benchmark): the node
 // holds the median of its set on (x[dim], id) along the largest-extent
 // dimension; left = the elements before it, right = those after it.  The
-// node's point goes first in its range so subtrees stay contiguous.
+// node's point goes first in its range so subtrees stay contiguous.  Every
+// node keeps the tight box of its subtree (the truncation test, R21).
 void nn_rec(tt_host_tree &t, int32_t b, int32_t e, int lvl) {
     const int D = t.dim;
     int32_t v = new_node(t, lvl, b, e);
     const int32_t n = e - b;
-    if (n == 1) {
-        t.body[v] = t.ids[b];
-        t.skip[v] = (int32_t)t.level.size();
-        return;
-    }
     float lo[TT_MAX_DIM], hi[TT_MAX_DIM];
     for (int d = 0; d < D; ++d) {
         lo[d] = std::numeric_limits<float>::infinity();
@@ -235,6 +231,13 @@ void nn_rec(tt_host_tree &t, int32_t b, int32_t e, int lvl) {
             lo[d] = std::min(lo[d], p[d]);
             hi[d] = std::max(hi[d], p[d]);
         }
+    }
+    t.lo.insert(t.lo.end(), lo, lo + D);  // tight box of the subtree (can_correlate)
+    t.hi.insert(t.hi.end(), hi, hi + D);
+    if (n == 1) {
+        t.body[v] = t.ids[b];
+        t.skip[v] = (int32_t)t.level.size();
+        return;
     }
     int sd = 0;
     float ext = hi[0] - lo[0];
@@ -411,6 +414,8 @@ tt_status tt_host_tree_desc(const tt_host_tree *t, tt_tree_desc *d) {
         d->split = t->split.data();
         d->in_child = t->in_child.data();    // left
         d->out_child = t->out_child.data();  // right
+        d->lo = t->lo.data();                // tight subtree boxes
+        d->hi = t->hi.data();
     } else {
         d->body = t->body.data();  // vantage point id per node
         d->in_child = t->in_child.data();

@@ -318,11 +318,11 @@ __device__ __forceinline__ unsigned warp_sum(unsigned v) { return __reduce_add_s
 
 // Stats writer for the warp tile (lane 0).
 __device__ __forceinline__ void write_warp_stats(const tt_common_params &c, long long tile, unsigned fetches,
-                                                 unsigned steps, bool lock) {
+                                                 unsigned steps, bool lock, bool switched = false) {
     if ((threadIdx.x & 31) == 0) {
         if (c.st_warp_fetches) c.st_warp_fetches[tile] = fetches;
         if (c.st_warp_steps) c.st_warp_steps[tile] = steps;
-        if (c.st_warp_mode) c.st_warp_mode[tile] = lock ? 1 : 2;
+        if (c.st_warp_mode) c.st_warp_mode[tile] = switched ? 3 : lock ? 1 : 2;
     }
 }
 

@@ -139,7 +139,7 @@ __global__ void __launch_bounds__(kBlock) knn_kernel(const tt_knn_params P, int 
     //   L: lb[cap][32], node[cap], mask[cap] (warp-uniform part owned by lane 0)
     unsigned char *wreg = s_stack + (size_t)warp * cap * 32 * 8;
     int *n_node = reinterpret_cast<int *>(wreg);
-    float *n_lb = reinterpret_cast<float *>(wreg + (size_t)cap * 32 * 4);
+    float *n_lbs = reinterpret_cast<float *>(wreg + (size_t)cap * 32 * 4);
     float *l_lb = reinterpret_cast<float *>(wreg);
     int *l_node = reinterpret_cast<int *>(wreg + (size_t)cap * 32 * 4);
     unsigned *l_mask = reinterpret_cast<unsigned *>(l_node + cap);
@@ -181,46 +181,19 @@ __global__ void __launch_bounds__(kBlock) knn_kernel(const tt_knn_params P, int 
         KBest<KT> kb;
         kb.init(k);
         unsigned visits = 0, fetches = 0, steps = 0;
-        if (!lock) {
-            int sp = 0;
-            int cur = valid ? 0 : TT_END;
-            float lb = 0.f;  // the root is never pruned: the list starts empty
-            while (cur != TT_END) {
-                if (STATS) ++visits;
-                if (!(kb.worst() < INF && lb > kb.worst())) {  // can_correlate
-                    int4 t, u;
-                    ld_rec(s_rec, g_rec, top, cur, t, u);
-                    if (t.x < 0) {
-                        leaf_update<DIM, KT>(P, u.z, u.w, DP, q, kb);
-                    } else {
-                        float lbl, lbr;
-                        child_lbs<DIM>(s_cbox, g_cbox, DP, top, cur, q, lbl, lbr);
-                        const bool left_near = select_dim<DIM>(q, u.y) < __int_as_float(u.x);
-                        n_node[sp * 32 + lane] = left_near ? t.y : t.x;  // push far with its bound
-                        n_lb[sp * 32 + lane] = left_near ? lbr : lbl;
-                        ++sp;
-                        cur = left_near ? t.x : t.y;                     // visit near
-                        lb = left_near ? lbl : lbr;
-                        continue;
-                    }
-                }
-                if (sp > 0) {
-                    --sp;
-                    cur = n_node[sp * 32 + lane];
-                    lb = n_lb[sp * 32 + lane];
-                } else {
-                    cur = TT_END;
-                }
-            }
-            if (STATS) {
-                fetches = warp_sum(visits);
-                steps = __reduce_max_sync(TT_FULL, visits);
-            }
-        } else {
+        // independent-walk state: the whole tile (N mode), or the rest of it
+        // after a dynamic L->N switch
+        int n_sp = 0;
+        int n_cur = valid ? 0 : TT_END;
+        float n_lb = 0.f;  // the root is never pruned: the list starts empty
+        bool run_n = !lock;
+        unsigned l_fetches = 0, l_steps = 0;
+        if (lock) {
             int sp = 0;
             int cur = 0;
             unsigned mask = vmask;
             float lb = 0.f;
+            const int switch_below = P.c.switch_below;
             for (;;) {
                 const bool in = (mask >> lane) & 1u;
                 if (STATS) {
@@ -229,6 +202,55 @@ __global__ void __launch_bounds__(kBlock) knn_kernel(const tt_knn_params P, int 
                 }
                 const bool active = in && !(kb.worst() < INF && lb > kb.worst());
                 const unsigned act = __ballot_sync(TT_FULL, active);
+                if (act && __popc(act) < switch_below) {
+                    // NEXT-3 dynamic L->N switch: each lane's rope stack is the
+                    // warp entries whose mask holds it, in order (a lockstep
+                    // lane visits exactly those), with its own bound.  The
+                    // warp-uniform halves are read lane-distributed first; a
+                    // lane's writes then only touch its own column of lb[][]
+                    // (row j <= i, already consumed) and the node/mask region
+                    // (already read).
+                    int en0 = 0, en1 = 0;
+                    unsigned em0 = 0, em1 = 0;
+                    if (lane < sp) {
+                        en0 = l_node[lane];
+                        em0 = l_mask[lane];
+                    }
+                    if (lane + 32 < sp) {
+                        en1 = l_node[lane + 32];
+                        em1 = l_mask[lane + 32];
+                    }
+                    __syncwarp();
+                    int j = 0;
+                    for (int i = 0; i < sp; ++i) {
+                        const int e_node = __shfl_sync(TT_FULL, i < 32 ? en0 : en1, i & 31);
+                        const unsigned e_mask = __shfl_sync(TT_FULL, i < 32 ? em0 : em1, i & 31);
+                        if ((e_mask >> lane) & 1u) {
+                            const float v = l_lb[i * 32 + lane];
+                            n_node[j * 32 + lane] = e_node;
+                            n_lbs[j * 32 + lane] = v;
+                            ++j;
+                        }
+                    }
+                    n_sp = j;
+                    // lanes of the mask resume at `cur` (the N loop re-takes its
+                    // truncation test, so it is not counted twice); the others
+                    // pop their own stack
+                    if (in) {
+                        n_cur = cur;
+                        n_lb = lb;
+                        if (STATS) --visits;
+                    } else if (n_sp > 0) {
+                        --n_sp;
+                        n_cur = n_node[n_sp * 32 + lane];
+                        n_lb = n_lbs[n_sp * 32 + lane];
+                    } else {
+                        n_cur = TT_END;
+                    }
+                    if (STATS) --steps;
+                    run_n = true;
+                    break;
+                }
                 if (act) {
                     if (STATS) ++fetches;
                     int4 t, u;
@@ -266,6 +288,47 @@ __global__ void __launch_bounds__(kBlock) knn_kernel(const tt_knn_params P, int 
                 mask = __shfl_sync(TT_FULL, e_mask, 0);
                 lb = l_lb[sp * 32 + lane];
             }
+            l_fetches = fetches;
+            l_steps = steps;
+        }
+        if (run_n) {
+            const unsigned v0 = visits;
+            int sp = n_sp;
+            int cur = n_cur;
+            float lb = n_lb;
+            while (cur != TT_END) {
+                if (STATS) ++visits;
+                if (!(kb.worst() < INF && lb > kb.worst())) {  // can_correlate
+                    int4 t, u;
+                    ld_rec(s_rec, g_rec, top, cur, t, u);
+                    if (t.x < 0) {
+                        leaf_update<DIM, KT>(P, u.z, u.w, DP, q, kb);
+                    } else {
+                        float lbl, lbr;
+                        child_lbs<DIM>(s_cbox, g_cbox, DP, top, cur, q, lbl, lbr);
+                        const bool left_near = select_dim<DIM>(q, u.y) < __int_as_float(u.x);
+                        n_node[sp * 32 + lane] = left_near ? t.y : t.x;  // push far with its bound
+                        n_lbs[sp * 32 + lane] = left_near ? lbr : lbl;
+                        ++sp;
+                        cur = left_near ? t.x : t.y;                     // visit near
+                        lb = left_near ? lbl : lbr;
+                        continue;
+                    }
+                }
+                if (sp > 0) {
+                    --sp;
+                    cur = n_node[sp * 32 + lane];
+                    lb = n_lbs[sp * 32 + lane];
+                } else {
+                    cur = TT_END;
+                }
+            }
+            if (STATS) {
+                // N part: every lane visit is a fetch; a switched tile adds its
+                // lockstep fetches / steps
+                fetches = l_fetches + warp_sum(visits - v0);
+                steps = l_steps + __reduce_max_sync(TT_FULL, visits - v0);
+            }
         }
         if (valid) {
 #pragma unroll
@@ -279,7 +342,7 @@ __global__ void __launch_bounds__(kBlock) knn_kernel(const tt_knn_params P, int 
             }
             if (STATS && P.c.st_visits) P.c.st_visits[pid] = visits;
         }
-        if (STATS) write_warp_stats(P.c, tile, fetches, steps, lock);
+        if (STATS) write_warp_stats(P.c, tile, fetches, steps, lock, lock && run_n);
         __syncwarp();
     }
     cta_finish(P.c.counter);

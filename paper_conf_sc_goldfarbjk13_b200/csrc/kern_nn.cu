@@ -5,17 +5,17 @@
 //
 // Fig.5 pattern with the update at every node (each node holds a
 // data point, Fig.1 line 9 before the children):
-//   truncate iff lb > best d2 (strict: an equal distance can still win on id);
+//   truncate iff boxd2(q, node's tight subtree box) > best d2 (can_correlate,
+//     as R5a; strict: an equal distance can still win on id);
 //   update with the node's point by (d2, id);
-//   near = q[dim] < split ? left : right (R5);
-//   near child keeps lb, far child gets max(lb, rn(rn(q[dim] - split)^2)).
-// The bound travels on the rope stack with the node as Fig.7's non-invariant
-// argument.  Stacks as in kern_knn.cu:
-//   independent (N): per-lane {node, lb}, lane-interleaved [depth][32] in
+//   near = q[dim] < split ? left : right (R5), visited first.
+// The test needs no argument from the parent, so rope-stack entries are bare
+// node indices:
+//   independent (N): per-lane stacks, lane-interleaved [depth][32] int32 in
 //     shared memory (bank = lane);
-//   lockstep (L): per-warp {node, mask} owned by lane 0 + per-lane lb
-//     (P:L1015-1023); the call set is reduced by a majority vote of the active
-//     lanes (§4.3, tie -> left first, R6).
+//   lockstep (L): one {node, mask} stack per warp owned by lane 0
+//     (P:L1015-1023); the call set is reduced by a majority vote of the
+//     active lanes (§4.3, tie -> left first, R6).
 #include "kern_common.cuh"
 
 namespace {
@@ -26,6 +26,22 @@ constexpr int kBlock = 256;
 constexpr int kWarps = kBlock / 32;
 constexpr int kSmemHdr = 128;
 
+// the node's tight box distance (can_correlate)
+template <int DIM>
+__device__ __forceinline__ float node_boxd2(const float *s_box, const float *g_box, int dp, int top, int cur,
+                                            const float (&q)[DIM]) {
+    float lo[DIM], hi[DIM];
+    if (cur < top) {
+        load_row_smem<DIM>(lo, s_box + (size_t)cur * 2 * dp);
+        load_row_smem<DIM>(hi, s_box + (size_t)cur * 2 * dp + dp);
+    } else {
+        load_row_nc<DIM>(lo, g_box + (size_t)cur * 2 * dp);
+        load_row_nc<DIM>(hi, g_box + (size_t)cur * 2 * dp + dp);
+    }
+    return pinned_boxd2<DIM>(q, lo, hi);
+}
+
+// record and point of node `cur`
 template <int DIM>
 __device__ __forceinline__ void ld_node(const unsigned char *s_rec, const float *s_pt, const tt_nn_rec *g_rec,
                                         const float *g_pt, int dp, int top, int cur, int4 &t, float (&v)[DIM]) {
@@ -45,23 +61,25 @@ __global__ void __launch_bounds__(kBlock) nn_kernel(const tt_nn_params P, int ca
     uint64_t *bar = reinterpret_cast<uint64_t *>(smem);
     const int top = P.c.top_count;
     unsigned char *s_rec = smem + kSmemHdr;
-    float *s_pt = reinterpret_cast<float *>(s_rec + (size_t)top * 16);
+    float *s_box = reinterpret_cast<float *>(s_rec + (size_t)top * 16);
+    float *s_pt = s_box + (size_t)top * 2 * DP;
     unsigned char *s_stack = reinterpret_cast<unsigned char *>(s_pt + (size_t)top * DP);
     const tt_nn_rec *g_rec = static_cast<const tt_nn_rec *>(P.c.tree.rec);
+    const float *g_box = P.c.tree.box;
     const float *g_pt = P.c.tree.vpt;
-    StageChunk ch[2] = {{s_rec, g_rec, (unsigned)top * 16u}, {s_pt, g_pt, (unsigned)top * 4u * DP}};
+    StageChunk ch[3] = {{s_rec, g_rec, (unsigned)top * 16u},
+                        {s_box, g_box, (unsigned)top * 8u * DP},
+                        {s_pt, g_pt, (unsigned)top * 4u * DP}};
     stage_top(bar, ch);
 
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
-    // per-warp region of cap*32*8 bytes:
-    //   N: node[cap][32], lb[cap][32]        (per-lane stacks, lane-interleaved)
-    //   L: lb[cap][32], node[cap], mask[cap] (warp-uniform part owned by lane 0)
-    unsigned char *wreg = s_stack + (size_t)warp * cap * 32 * 8;
+    // per-warp region of cap*32*4 bytes:
+    //   N: node[cap][32]          (per-lane stacks, lane-interleaved)
+    //   L: node[cap], mask[cap]   (warp-uniform, owned by lane 0)
+    unsigned char *wreg = s_stack + (size_t)warp * cap * 32 * 4;
     int *n_node = reinterpret_cast<int *>(wreg);
-    float *n_lb = reinterpret_cast<float *>(wreg + (size_t)cap * 32 * 4);
-    float *l_lb = reinterpret_cast<float *>(wreg);
-    int *l_node = reinterpret_cast<int *>(wreg + (size_t)cap * 32 * 4);
+    int *l_node = reinterpret_cast<int *>(wreg);
     unsigned *l_mask = reinterpret_cast<unsigned *>(l_node + cap);
     const long long n = P.c.n;
     const long long ntiles = (n + 31) >> 5;
@@ -105,10 +123,9 @@ __global__ void __launch_bounds__(kBlock) nn_kernel(const tt_nn_params P, int ca
         if (!lock) {
             int sp = 0;
             int cur = valid ? 0 : TT_END;
-            float lb = 0.f;  // the root is never pruned: best starts at +inf
             while (cur != TT_END) {
                 if (STATS) ++visits;
-                if (!(lb > best_d)) {
+                if (!(node_boxd2<DIM>(s_box, g_box, DP, top, cur, q) > best_d)) {
                     int4 t;
                     float v[DIM];
                     ld_node<DIM>(s_rec, s_pt, g_rec, g_pt, DP, top, cur, t, v);
@@ -121,30 +138,16 @@ __global__ void __launch_bounds__(kBlock) nn_kernel(const tt_nn_params P, int ca
                         }
                     }
                     if (t.w >= 0) {
-                        const float qd = select_dim<DIM>(q, t.w);
-                        const float split = __int_as_float(t.z);
-                        const bool left_near = qd < split;
-                        const float diff = __fsub_rn(qd, split);
-                        const float far_lb = fmaxf(lb, __fmul_rn(diff, diff));
+                        const bool left_near = select_dim<DIM>(q, t.w) < __int_as_float(t.z);
                         const int nearc = left_near ? t.x : t.y, farc = left_near ? t.y : t.x;
-                        if (farc != TT_END) {
-                            n_node[sp * 32 + lane] = farc;
-                            n_lb[sp * 32 + lane] = far_lb;
-                            ++sp;
-                        }
+                        if (farc != TT_END) n_node[sp++ * 32 + lane] = farc;
                         if (nearc != TT_END) {
                             cur = nearc;
                             continue;
                         }
                     }
                 }
-                if (sp > 0) {
-                    --sp;
-                    cur = n_node[sp * 32 + lane];
-                    lb = n_lb[sp * 32 + lane];
-                } else {
-                    cur = TT_END;
-                }
+                cur = sp > 0 ? n_node[--sp * 32 + lane] : TT_END;
             }
             if (STATS) {
                 fetches = warp_sum(visits);
@@ -154,14 +157,14 @@ __global__ void __launch_bounds__(kBlock) nn_kernel(const tt_nn_params P, int ca
             int sp = 0;
             int cur = 0;
             unsigned mask = vmask;
-            float lb = 0.f;
             for (;;) {
                 const bool in = (mask >> lane) & 1u;
                 if (STATS) {
                     ++steps;
                     visits += in;
                 }
-                const bool active = in && !(lb > best_d);
+                // one warp-uniform box fetch, tested by every lane of the mask
+                const bool active = in && !(node_boxd2<DIM>(s_box, g_box, DP, top, cur, q) > best_d);
                 const unsigned act = __ballot_sync(TT_FULL, active);
                 if (act) {
                     if (STATS) ++fetches;
@@ -179,29 +182,19 @@ __global__ void __launch_bounds__(kBlock) nn_kernel(const tt_nn_params P, int ca
                         }
                     }
                     if (t.w >= 0) {
-                        const float qd = select_dim<DIM>(q, t.w);
-                        const float split = __int_as_float(t.z);
-                        const bool left_near = qd < split;
-                        const float diff = __fsub_rn(qd, split);
-                        const float far_lb = fmaxf(lb, __fmul_rn(diff, diff));
+                        const bool left_near = select_dim<DIM>(q, t.w) < __int_as_float(t.z);
                         const int votes = __popc(__ballot_sync(TT_FULL, active && left_near));
                         const bool left_first = 2 * votes >= __popc(act);
                         const int first = left_first ? t.x : t.y, second = left_first ? t.y : t.x;
-                        // the lane's bound for a child: lb if it is the lane's near
-                        // child, else far_lb
-                        const float lb_first = (left_first == left_near) ? lb : far_lb;
-                        const float lb_second = (left_first == left_near) ? far_lb : lb;
                         if (second != TT_END) {
                             if (lane == 0) {  // push second (warp-uniform entry)
                                 l_node[sp] = second;
                                 l_mask[sp] = act;
                             }
-                            l_lb[sp * 32 + lane] = lb_second;
                             ++sp;
                         }
                         if (first != TT_END) {
                             cur = first;
-                            lb = lb_first;
                             mask = act;
                             continue;
                         }
@@ -218,7 +211,6 @@ __global__ void __launch_bounds__(kBlock) nn_kernel(const tt_nn_params P, int ca
                 }
                 cur = __shfl_sync(TT_FULL, e_node, 0);
                 mask = __shfl_sync(TT_FULL, e_mask, 0);
-                lb = l_lb[sp * 32 + lane];
             }
         }
         if (valid) {
@@ -236,7 +228,7 @@ template <int DIM, bool STATS>
 int launch(const tt_nn_params &p, const tt_launch_cfg &cfg) {
     constexpr int DP = (DIM + 3) & ~3;
     const int cap = p.c.height + 2;
-    const size_t smem = kSmemHdr + (size_t)p.c.top_count * (16 + 4 * DP) + (size_t)kWarps * cap * 32 * 8;
+    const size_t smem = kSmemHdr + (size_t)p.c.top_count * (16 + 12 * DP) + (size_t)kWarps * cap * 32 * 4;
     auto kern = nn_kernel<DIM, STATS>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return (int)e;

@@ -28,7 +28,8 @@ int dim_padded(int dim) { return (dim + 3) & ~3; }
 int stage_bytes_per_node(int kind, int dp) {
     if (kind == TT_KIND_OCT) return 32;
     if (kind == TT_KIND_KD) return 32 + 8 * dp;
-    return 16 + 4 * dp;  // VP, NN
+    if (kind == TT_KIND_NN) return 16 + 12 * dp;  // record + box + point
+    return 16 + 4 * dp;                            // VP
 }
 
 int validate(const tt_tree_desc *d) {
@@ -50,7 +51,8 @@ int validate(const tt_tree_desc *d) {
         (!d->body || !d->in_child || !d->out_child || !d->r_in_max || !d->r_out_min || !d->points))
         return TT_ERR_INVALID_ARG;
     if (d->kind == TT_KIND_NN &&
-        (!d->body || !d->in_child || !d->out_child || !d->split || !d->split_dim || !d->points))
+        (!d->body || !d->in_child || !d->out_child || !d->split || !d->split_dim || !d->points || !d->lo ||
+         !d->hi))
         return TT_ERR_INVALID_ARG;
     const int64_t N = d->n_nodes;
     for (int64_t v = 0; v < N; ++v) {
@@ -122,6 +124,10 @@ void plan(const tt_tree_desc *d, tt_blob_header &h, std::vector<int32_t> *newidx
         h.off_cbox = off;
         off = align256(off + (uint64_t)d->n_nodes * 4 * h.dp * sizeof(float));
     } else if (d->kind == TT_KIND_VP || d->kind == TT_KIND_NN) {
+        if (d->kind == TT_KIND_NN) {
+            h.off_box = off;
+            off = align256(off + (uint64_t)d->n_nodes * 2 * h.dp * sizeof(float));
+        }
         h.off_vpt = off;
         off = align256(off + (uint64_t)d->n_nodes * h.dp * sizeof(float));
         h.off_pid = off;
@@ -226,6 +232,7 @@ int tt_pack_impl(const tt_tree_desc *d, void *blob, size_t bytes) {
         }
     } else if (d->kind == TT_KIND_NN) {
         auto *rec = reinterpret_cast<tt_nn_rec *>(base + h.off_rec);
+        auto *box = reinterpret_cast<float *>(base + h.off_box);
         auto *vpt = reinterpret_cast<float *>(base + h.off_vpt);
         auto *pid = reinterpret_cast<int32_t *>(base + h.off_pid);
         for (int64_t v = 0; v < N; ++v) {
@@ -235,6 +242,11 @@ int tt_pack_impl(const tt_tree_desc *d, void *blob, size_t bytes) {
             r.right = map(d->out_child[v]);
             r.split = d->split[v];
             r.dim = d->split_dim[v];
+            float *bx = box + (size_t)nv * 2 * h.dp;
+            for (int k = 0; k < d->dim; ++k) {
+                bx[k] = d->lo[v * d->dim + k];
+                bx[h.dp + k] = d->hi[v * d->dim + k];
+            }
             pid[nv] = d->body[v];
             std::memcpy(vpt + (size_t)nv * h.dp, d->points + (size_t)d->body[v] * d->dim, sizeof(float) * d->dim);
         }

@@ -46,7 +46,7 @@ constexpr int kTopBH = 32 * 1024, kTopPC = 32 * 1024, kTopKNN = 16 * 1024, kTopV
 
 tt_status setup_common(const tt_tree *t, int kind, int64_t n, const tt_traverse_opts *o, int default_amd,
                        int stage_bytes_per_node, int stage_budget, tt_common_params &c, tt_launch_cfg &cfg,
-                       tt_stream s) {
+                       tt_stream s, bool allow_switch = false) {
     if (!t) return TT_ERR_INVALID_ARG;
     if (t->hdr.kind != kind) return TT_ERR_KIND_MISMATCH;
     if (n < 0 || n > (int64_t)0xffffffffu * 32) return TT_ERR_INVALID_ARG;
@@ -83,6 +83,10 @@ tt_status setup_common(const tt_tree *t, int kind, int64_t n, const tt_traverse_
             return TT_ERR_INVALID_ARG;
         if (o->variant == TT_VARIANT_RECURSIVE && o->mode == TT_MODE_LOCKSTEP) return TT_ERR_UNSUPPORTED;
         cfg.variant = o->variant;
+        if (o->switch_below < 0 || o->switch_below > 33) return TT_ERR_INVALID_ARG;
+        if (o->switch_below != 0 && (!allow_switch || o->variant != TT_VARIANT_AUTOROPES))
+            return TT_ERR_UNSUPPORTED;  // kNN autoropes only
+        c.switch_below = o->switch_below;
     }
     unsigned slot = __atomic_fetch_add(&const_cast<tt_tree *>(t)->slot_next, 1u, __ATOMIC_RELAXED) % TT_COUNTER_SLOTS;
     c.counter = t->d_counters + 2 * slot;
@@ -371,7 +375,7 @@ tt_status tt_traverse_knn(const tt_tree *t, const float *q, int64_t n, int32_t l
     if (!t) return TT_ERR_INVALID_ARG;  // (the staging size below reads t->hdr)
     tt_knn_params p;
     tt_launch_cfg cfg;
-    tt_status st = setup_common(t, TT_KIND_KD, n, opts, kAutoKNN, 32 + 16 * t->hdr.dp, kTopKNN, p.c, cfg, s);
+    tt_status st = setup_common(t, TT_KIND_KD, n, opts, kAutoKNN, 32 + 16 * t->hdr.dp, kTopKNN, p.c, cfg, s, true);
     if (st != TT_OK) return st;
     if (k < 1) return TT_ERR_INVALID_ARG;
     if (k > TT_MAX_K) return TT_ERR_UNSUPPORTED;
@@ -418,7 +422,7 @@ tt_status tt_traverse_nn(const tt_tree *t, const float *q, int64_t n, int32_t ld
     if (!t) return TT_ERR_INVALID_ARG;  // (the staging size below reads t->hdr)
     tt_nn_params p;
     tt_launch_cfg cfg;
-    tt_status st = setup_common(t, TT_KIND_NN, n, opts, kAutoNN, 16 + 4 * t->hdr.dp, kTopNN, p.c, cfg, s);
+    tt_status st = setup_common(t, TT_KIND_NN, n, opts, kAutoNN, 16 + 12 * t->hdr.dp, kTopNN, p.c, cfg, s);
     if (st != TT_OK) return st;
     if (ld < t->hdr.dim) return TT_ERR_INVALID_ARG;
     if (!dim_supported(t->hdr.dim)) return TT_ERR_UNSUPPORTED;

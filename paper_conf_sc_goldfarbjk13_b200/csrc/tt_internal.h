@@ -29,7 +29,7 @@
 // VP:  t = {in | -1, out | -1, r_in_max (float bits), r_out_min (float bits)}
 //      + vpt[dp] vantage coordinates and pid (vantage point's original id)
 // NN:  t = {left | -1, right | -1, split (float bits), split_dim | -1}
-//      + vpt[dp] the node's point and pid (its original id)
+//      + box[2*dp] tight subtree box, vpt[dp] the node's point, pid (its id)
 // ---------------------------------------------------------------------------
 struct alignas(16) tt_oct_rec {
     float gx, gy, gz, gm;
@@ -74,7 +74,7 @@ struct tt_blob_header {
 struct tt_dev_tree {
     const tt_blob_header *hdr_dev;
     const void *rec;      // records, top nodes first
-    const float *box;     // KD: [n_nodes][2*dp]
+    const float *box;     // KD, NN: [n_nodes][2*dp]
     const float *pts;     // KD: [n_points][dp] tree order
     const int32_t *pid;   // KD: [n_points]; VP, NN: [n_nodes]
     const float *vpt;     // VP, NN: [n_nodes][dp] the node's point
@@ -91,6 +91,7 @@ struct tt_common_params {
     const uint32_t *order; // nullable
     int32_t mode;          // tt_mode
     int32_t auto_min_depth;
+    int32_t switch_below;  // dynamic L->N switching threshold (kNN), 0 = never
     uint32_t *counter;     // [2] tile scheduler: next tile, finished CTAs
     // stats (nullable)
     uint32_t *st_visits, *st_warp_fetches, *st_warp_steps;

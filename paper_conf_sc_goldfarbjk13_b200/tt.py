@@ -267,9 +267,10 @@ def _lanes(order, n):
     return n if order is None else order.numel()
 
 
-def _opts(mode, auto_min_depth, order, stats, n, variant="autoropes"):
+def _opts(mode, auto_min_depth, order, stats, n, variant="autoropes", switch_below=0):
     o = L.tt_traverse_opts()
     o.variant = L.VARIANT[variant]
+    o.switch_below = int(switch_below)
     o.mode = L.MODE[mode] if isinstance(mode, str) else int(mode)
     o.auto_min_depth = -1 if auto_min_depth is None else int(auto_min_depth)
     keep = []
@@ -357,14 +358,14 @@ def tt_traverse_pc(tree: Tree, q: torch.Tensor, radius: float, out: torch.Tensor
 def tt_traverse_knn(tree: Tree, q: torch.Tensor, k: int, out_idx: torch.Tensor | None = None,
                     out_d2: torch.Tensor | None = None, order: torch.Tensor | None = None, mode="auto",
                     auto_min_depth: int | None = None, stats: Stats | None = None, stream=None,
-                    variant: str = "autoropes"):
+                    variant: str = "autoropes", switch_below: int = 0):
     _dev(q, torch.float32, "q", tree.dim)
     n = q.shape[0]
     if out_idx is None:
         out_idx = torch.empty((n, k), dtype=torch.int32, device=q.device)
     if out_d2 is None:
         out_d2 = torch.empty((n, k), dtype=torch.float32, device=q.device)
-    o, keep = _opts(mode, auto_min_depth, order, stats, n, variant)
+    o, keep = _opts(mode, auto_min_depth, order, stats, n, variant, switch_below)
     check(L.load().tt_traverse_knn(tree._h, q.data_ptr(), _lanes(order, n), q.stride(0), int(k), out_idx.data_ptr(),
                                    out_d2.data_ptr(), C.byref(o), C.c_void_p(_stream_handle(stream))),
           "tt_traverse_knn")

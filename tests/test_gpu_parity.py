@@ -650,3 +650,31 @@ def test_gpu_vp_build_is_byte_identical_to_host_pack(n, dim):
     assert gpu_blob.size == host_blob.size
     diff = np.nonzero(gpu_blob != host_blob)[0]
     assert diff.size == 0, f"{diff.size} bytes differ, first at {diff[:8]}"
+
+
+# ------------------------------------------------ NEXT-3 dynamic L->N switch
+@pytest.mark.parametrize("sorted_", [False, True])
+def test_knn_dynamic_switch_results_exact(knn_small, sorted_):
+    """Dynamic L->N switching (tt_traverse_opts.switch_below) never changes
+    results; switch_below = 33 switches every tile at the root,
+    so lane visits are exactly the independent walk's (autoropes order), and
+    switch_below = 0 is plain lockstep (the Fig.8 simulation)."""
+    p, q, ot, tree = knn_small
+    qd = dev(q)
+    order = P.tt_sort_points(tree, qd) if sorted_ else None
+    ref = oracle.knn(ot, q, 8, stats=True)
+    for a in (0, 2, 5, 12, 24, 33):
+        st = P.Stats.alloc(len(q), "cuda")
+        idx, d2 = P.tt_traverse_knn(tree, qd, 8, order=order, mode="lockstep", stats=st, switch_below=a)
+        assert np.array_equal(idx.cpu().numpy(), ref.out[0]) and np.array_equal(d2.cpu().numpy(), ref.out[1]), a
+        wm = st.warp_mode.cpu().numpy()
+        if a == 33:
+            assert np.all(wm == 3)
+            assert np.array_equal(st.visits.cpu().numpy(), ref.visits)
+        if a == 0:
+            assert np.all(wm == 1)
+            o = order.cpu().numpy() if sorted_ else np.arange(len(q))
+            li, ld, lv, wf = oracle.knn_lockstep(ot, q[o], 8)
+            assert np.array_equal(st.warp_fetches.cpu().numpy(), wf)
+    with pytest.raises(P.TTError):
+        P.tt_traverse_knn(tree, qd, 8, switch_below=34)

@@ -101,6 +101,8 @@ def test_nn_builder_matches_oracle(n, dim):
     assert np.array_equal(h.array("skip"), o.i64(oracle.F_SKIP))
     assert np.array_equal(h.array("level"), o.i64(oracle.F_LEVEL))
     assert np.array_equal(h.array("tree_order"), o.tree_order())
+    assert np.array_equal(h.array("lo"), o.f32(oracle.F_LO, dim).reshape(-1, dim))
+    assert np.array_equal(h.array("hi"), o.f32(oracle.F_HI, dim).reshape(-1, dim))
 
 
 def test_nn_blob_records_and_points():
@@ -117,18 +119,27 @@ def test_nn_blob_records_and_points():
     pid = np.frombuffer(blob[hd["off_pid"]:hd["off_pid"] + 4 * N].tobytes(), "<i4")
     assert np.array_equal(np.sort(pid), np.arange(N))
     assert np.array_equal(pts[:, :7], p[pid]) and np.all(pts[:, 7] == 0)
-    # walk the device numbering from the root: every subtree satisfies the split rule
-    stack, seen = [0], 0
-    while stack:
-        v = stack.pop()
-        seen += 1
+    box = np.frombuffer(blob[hd["off_box"]:hd["off_box"] + 64 * N].tobytes(), "<f4").reshape(N, 2, 8)
+    # subtree point sets from the device numbering; every node's box is their
+    # tight box and every child satisfies the node's split rule
+    def subtree(v):
+        out, st = [], [v]
+        while st:
+            u = st.pop()
+            out.append(u)
+            st += [c for c in (rec["l"][u], rec["r"][u]) if c >= 0]
+        return out
+    seen = 0
+    for v in range(N):
+        ids = pid[subtree(v)]
+        assert np.array_equal(box[v, 0, :7], p[ids].min(0)) and np.array_equal(box[v, 1, :7], p[ids].max(0))
         for c, side in ((rec["l"][v], 0), (rec["r"][v], 1)):
             if c < 0:
                 continue
-            assert rec["dim"][v] >= 0
             d = rec["dim"][v]
+            assert d >= 0
             assert (p[pid[c], d] <= rec["split"][v]) if side == 0 else (p[pid[c], d] >= rec["split"][v])
-            stack.append(c)
+        seen += 1
     assert seen == N
 
 
