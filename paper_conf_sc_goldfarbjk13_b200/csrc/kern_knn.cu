@@ -118,8 +118,19 @@ __device__ __forceinline__ void leaf_update(const tt_knn_params &P, int pb, int 
     }
 }
 
+#ifndef TT_KNN_MINB
+#define TT_KNN_MINB 4
+#endif
+// per-warp rope-stack bytes: INDEPENDENT launches keep {node, lb} per lane in
+// shared memory ("wide"); AUTO / LOCKSTEP launches keep per-lane lb + the
+// warp-uniform {node, mask} ("narrow"), and their independent warps put the
+// lb half of a lane entry in a per-thread interleaved global scratch.
+__host__ __device__ constexpr size_t knn_stack_bytes(int cap, bool wide) {
+    return wide ? (size_t)cap * 32 * 8 : (size_t)cap * (32 * 4 + 8);
+}
+
 template <int DIM, int KT, bool STATS>
-__global__ void __launch_bounds__(kBlock) knn_kernel(const tt_knn_params P, int cap) {
+__global__ void __launch_bounds__(kBlock, TT_KNN_MINB) knn_kernel(const tt_knn_params P, int cap, float *g_lb) {
     extern __shared__ __align__(128) unsigned char smem[];
     constexpr int DP = (DIM + 3) & ~3;
     uint64_t *bar = reinterpret_cast<uint64_t *>(smem);
@@ -137,9 +148,14 @@ __global__ void __launch_bounds__(kBlock) knn_kernel(const tt_knn_params P, int 
     // per-warp region of cap*32*8 bytes:
     //   N: node[cap][32], lb[cap][32]       (per-lane stacks, lane-interleaved)
     //   L: lb[cap][32], node[cap], mask[cap] (warp-uniform part owned by lane 0)
-    unsigned char *wreg = s_stack + (size_t)warp * cap * 32 * 8;
+    const bool wide = g_lb == nullptr;
+    unsigned char *wreg = s_stack + (size_t)warp * knn_stack_bytes(cap, wide);
     int *n_node = reinterpret_cast<int *>(wreg);
-    float *n_lbs = reinterpret_cast<float *>(wreg + (size_t)cap * 32 * 4);
+    // lb half of the independent stacks: shared (wide) or global scratch
+    const size_t gtid = blockIdx.x * (size_t)blockDim.x + threadIdx.x, gstride = (size_t)gridDim.x * blockDim.x;
+    float *n_lbs = wide ? reinterpret_cast<float *>(wreg + (size_t)cap * 32 * 4) : g_lb + gtid;
+    const size_t lbs_stride = wide ? 32 : gstride;
+    const int lbs_lane = wide ? lane : 0;
     float *l_lb = reinterpret_cast<float *>(wreg);
     int *l_node = reinterpret_cast<int *>(wreg + (size_t)cap * 32 * 4);
     unsigned *l_mask = reinterpret_cast<unsigned *>(l_node + cap);
@@ -228,7 +244,7 @@ __global__ void __launch_bounds__(kBlock) knn_kernel(const tt_knn_params P, int 
                         if ((e_mask >> lane) & 1u) {
                             const float v = l_lb[i * 32 + lane];
                             n_node[j * 32 + lane] = e_node;
-                            n_lbs[j * 32 + lane] = v;
+                            n_lbs[j * lbs_stride + lbs_lane] = v;
                             ++j;
                         }
                     }
@@ -243,7 +259,7 @@ __global__ void __launch_bounds__(kBlock) knn_kernel(const tt_knn_params P, int 
                     } else if (n_sp > 0) {
                         --n_sp;
                         n_cur = n_node[n_sp * 32 + lane];
-                        n_lb = n_lbs[n_sp * 32 + lane];
+                        n_lb = n_lbs[n_sp * lbs_stride + lbs_lane];
                     } else {
                         n_cur = TT_END;
                     }
@@ -308,7 +324,7 @@ __global__ void __launch_bounds__(kBlock) knn_kernel(const tt_knn_params P, int 
                         child_lbs<DIM>(s_cbox, g_cbox, DP, top, cur, q, lbl, lbr);
                         const bool left_near = select_dim<DIM>(q, u.y) < __int_as_float(u.x);
                         n_node[sp * 32 + lane] = left_near ? t.y : t.x;  // push far with its bound
-                        n_lbs[sp * 32 + lane] = left_near ? lbr : lbl;
+                        n_lbs[sp * lbs_stride + lbs_lane] = left_near ? lbr : lbl;
                         ++sp;
                         cur = left_near ? t.x : t.y;                     // visit near
                         lb = left_near ? lbl : lbr;
@@ -318,7 +334,7 @@ __global__ void __launch_bounds__(kBlock) knn_kernel(const tt_knn_params P, int 
                 if (sp > 0) {
                     --sp;
                     cur = n_node[sp * 32 + lane];
-                    lb = n_lbs[sp * 32 + lane];
+                    lb = n_lbs[sp * lbs_stride + lbs_lane];
                 } else {
                     cur = TT_END;
                 }
@@ -352,7 +368,8 @@ template <int DIM, int KT, bool STATS>
 int launch(const tt_knn_params &p, const tt_launch_cfg &cfg) {
     constexpr int DP = (DIM + 3) & ~3;
     const int cap = p.c.height + 2;
-    const size_t smem = kSmemHdr + (size_t)p.c.top_count * (32 + 16 * DP) + (size_t)kWarps * cap * 32 * 8;
+    const bool wide = p.c.mode == TT_MODE_INDEPENDENT;
+    const size_t smem = kSmemHdr + (size_t)p.c.top_count * (32 + 16 * DP) + (size_t)kWarps * knn_stack_bytes(cap, wide);
     auto kern = knn_kernel<DIM, KT, STATS>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return (int)e;
@@ -368,8 +385,17 @@ int launch(const tt_knn_params &p, const tt_launch_cfg &cfg) {
     const long long need = (ntiles + kWarps - 1) / kWarps;
     if (grid > need) grid = need;
     if (grid < 1) grid = 1;
-    kern<<<(unsigned)grid, kBlock, smem, (cudaStream_t)cfg.stream>>>(p, cap);
-    return (int)cudaGetLastError();
+    float *g_lb = nullptr;
+    const cudaStream_t s = (cudaStream_t)cfg.stream;
+    if (!wide) {
+        tt_keep_pool_memory();
+        e = cudaMallocAsync((void **)&g_lb, sizeof(float) * (size_t)cap * (size_t)grid * kBlock, s);
+        if (e != cudaSuccess) return (int)e;
+    }
+    kern<<<(unsigned)grid, kBlock, smem, s>>>(p, cap, g_lb);
+    e = cudaGetLastError();
+    if (g_lb) cudaFreeAsync(g_lb, s);
+    return (int)e;
 }
 
 template <int DIM, int KT>

@@ -62,6 +62,7 @@ tt_status setup_common(const tt_tree *t, int kind, int64_t n, const tt_traverse_
     c.root_side = t->hdr.root_side;
     cfg.block_threads = 256;
     cfg.ctas_per_sm = 0;
+    if (const char *ev = std::getenv("TT_CTAS_PER_SM")) cfg.ctas_per_sm = std::atoi(ev);  // tuning sweeps only
     cfg.stream = s;
     cfg.variant = TT_VARIANT_AUTOROPES;
     if (o) {
@@ -77,7 +78,7 @@ tt_status setup_common(const tt_tree *t, int kind, int64_t n, const tt_traverse_
         }
         if (o->block_threads != 0 && o->block_threads != 256) return TT_ERR_UNSUPPORTED;
         if (o->ctas_per_sm < 0) return TT_ERR_INVALID_ARG;
-        cfg.ctas_per_sm = o->ctas_per_sm;
+        if (o->ctas_per_sm > 0) cfg.ctas_per_sm = o->ctas_per_sm;
         if (o->variant != TT_VARIANT_AUTOROPES && o->variant != TT_VARIANT_RECURSIVE &&
             o->variant != TT_VARIANT_STACK)
             return TT_ERR_INVALID_ARG;

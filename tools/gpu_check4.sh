@@ -1,0 +1,6 @@
+#!/bin/bash
+mkdir -p gpurun_out
+timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.txt 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.txt
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.txt 2>&1; echo "smoke rc=$?" >> gpurun_out/smoke.txt
+timeout 600 python tools/tile_costs.py bh knn > gpurun_out/tile_costs.txt 2>&1
+tail -3 gpurun_out/pytest_gpu.txt; cat gpurun_out/smoke.txt gpurun_out/tile_costs.txt
