@@ -5,7 +5,7 @@ set -x
 mkdir -p gpurun_out
 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/launches_bh.csv \
     python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e > /dev/null 2>&1
-for spec in "bh auto 1000000" "pc auto 10000" "knn auto 1000000" "vp auto 1000000" "vp independent 1000000" "knn independent 1000000"; do
+for spec in "bh auto 1000000" "pc auto 10000" "knn auto 1000000" "vp auto 1000000" "vp independent 1000000" "knn independent 1000000" "nn auto 1000000"; do
   set -- $spec
   w=$1; m=$2; n=$3
   ncu --set full --clock-control none --import-source on -k regex:${w}_kernel -s 1 -c 1 \
