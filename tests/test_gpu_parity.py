@@ -451,6 +451,29 @@ def test_bh_config5_16m_sampled():
     assert err.max() <= BH_TOL
 
 
+@pytest.mark.slow
+def test_knn_config5_16m_sampled():
+    """configs[4]: kNN k=8, 16,777,216 queries over 16,777,216 7-D mixture
+    points, in the launch configuration bench.py times (device-built tree,
+    sort + longest-first schedule, AUTO); sampled queries bit-exact against
+    brute force over all 16M points (the plain definition, R4)."""
+    c = ttgen.CONFIGS["knn_16m_7d"]
+    p = ttgen.gaussian_mixture(c["n"], c["dim"], c["seed"])
+    q = ttgen.gaussian_mixture(c["m"], c["dim"], c["qseed"])
+    pd, qd = dev(p), dev(q)
+    tree = P.tt_build_kd_device(pd, c["leaf"])
+    perm = P.tt_schedule_tiles(tree, qd, P.tt_sort_points(tree, qd))
+    idx, d2 = P.tt_traverse_knn(tree, qd, c["k"], order=perm)
+    sample = np.random.default_rng(4).choice(len(q), 24, replace=False)
+    gi, gd = idx.cpu().numpy(), d2.cpu().numpy()
+    for i in sample:
+        D = _pinned_d2(q[i][None, :], p)  # the plain definition over all points
+        kth = np.partition(D, c["k"] - 1)[c["k"] - 1]
+        cand = np.nonzero(D <= kth)[0]
+        best = cand[np.lexsort((cand, D[cand]))][: c["k"]]  # (d2, id) order
+        assert np.array_equal(gi[i], best) and np.array_equal(gd[i], D[best])
+
+
 # ------------------------------------------------ recursive baseline (NEXT-2)
 def test_recursive_baseline_matches_oracle(bh_small, knn_small, vp_small, pc_setup):
     """The naive recursive GPU baseline computes the same results
