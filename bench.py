@@ -415,6 +415,15 @@ def run_ours(args, rank, world, local_rank):
     build_where = "device (tt_build_*_device)" if args.device_build else "host (tt_build_*)"
 
     q_all = torch.from_numpy(np.ascontiguousarray(w["queries"])).to(device)
+    ids_all = None
+    if world > 1 and not args.unsorted:
+        # Spatial decomposition (data placement, before the timed region, as a
+        # time-stepping code keeps its bodies -- DESIGN.md §9): rank r owns a
+        # contiguous range of the global tree order, so its warps are as
+        # coherent as on one GPU.  Each step still sorts the rank's own shard.
+        gperm = P.tt_sort_points(tree, q_all).long()
+        q_all = q_all[gperm].contiguous()
+        ids_all = gperm.to(torch.int32)
     q_shard = q_all[lo:hi]
     n_all = len(w["queries"])
     stream = torch.cuda.current_stream()
@@ -436,7 +445,9 @@ def run_ours(args, rank, world, local_rank):
         return tuple(x[lo:hi] for x in o) if isinstance(o, tuple) else o[lo:hi]
 
     out_shard = views(out)
-    self_ids = torch.arange(lo, hi, dtype=torch.int32, device=device) if name == "bh" else None
+    self_ids = None
+    if name == "bh":  # the bodies' ids in the tree (original indices)
+        self_ids = ids_all[lo:hi] if ids_all is not None else torch.arange(lo, hi, dtype=torch.int32, device=device)
 
     def traverse(pts, res, order, stats=None):
         if name == "bh":
@@ -529,7 +540,7 @@ def run_ours(args, rank, world, local_rank):
     # e2e through the public API with host buffers (pinned), copies inside
     e2e = None
     if not args.no_e2e:
-        q_host = torch.from_numpy(np.ascontiguousarray(w["queries"][lo:hi])).pin_memory()
+        q_host = q_shard.cpu().pin_memory()
         q_dev = torch.empty_like(q_host, device=device)
         res_host = None
         if name == "bh":
@@ -652,7 +663,8 @@ def run_ours(args, rank, world, local_rank):
                    "tile_schedule": "longest-first" if lpt else "in-order",
                    **({"switch_below": args.switch_below} if args.switch_below else {}),
                    "auto_min_depth": args.auto_min_depth, "variant": args.variant,
-                   "parallelism": f"dp{world} (points sharded, tree replicated)",
+                   "parallelism": f"dp{world} (points sharded by global tree order, tree replicated)"
+                   if world > 1 and not args.unsorted else f"dp{world} (points sharded, tree replicated)",
                    "l2": "flushed between timed steps (512 MiB write)",
                    "params": {k: v for k, v in c.items() if k not in ("kind",)}},
         "node_visits_per_sec": visits_tot / (kms / 1e3),
