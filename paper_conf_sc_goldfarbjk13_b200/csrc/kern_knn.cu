@@ -228,6 +228,7 @@ __global__ void __launch_bounds__(kBlock, TT_KNN_MINB) knn_kernel(const tt_knn_p
                     // (already read).
                     int en0 = 0, en1 = 0;
                     unsigned em0 = 0, em1 = 0;
+                    __syncwarp();  // lane 0's pushes visible to every lane
                     if (lane < sp) {
                         en0 = l_node[lane];
                         em0 = l_mask[lane];
