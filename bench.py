@@ -59,6 +59,7 @@ def parse():
                     help="skip tt_schedule_tiles (longest-first tile order after the sort; kd/vp trees)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-chase", action="store_true", help="skip the live L2-latency (tt_diag_chase) roof")
     ap.add_argument("--points-per-rank", type=int, default=0, help="override M (testing)")
     ap.add_argument("--auto-min-depth", type=int, default=None, help="AUTO-mode threshold (default: kernel's)")
     ap.add_argument("--switch-below", type=int, default=0,
@@ -249,6 +250,28 @@ def kernel_sha256(workload: str) -> str:
         h.update(os.path.basename(f).encode())
         h.update(open(f, "rb").read())
     return h.hexdigest()
+
+
+def chase_ceiling(P, nrec: int, device, per_lane: bool, steps: int = 3000) -> float:
+    """Dependent record loads per second of a pure chase (tt_diag_chase):
+    the walk's latency ceiling.  Median of 3 timed launches after 1 warm-up."""
+    import torch
+    rec = P.chase_records(int(nrec), device)
+    nsm = torch.cuda.get_device_properties(device).multi_processor_count
+    chains = nsm * 4 * 256 if per_lane else nsm * 4 * 8
+    n = steps // 8 if per_lane else steps
+    s = torch.cuda.current_stream()
+    P.tt_diag_chase(rec, n, per_lane)
+    ts = []
+    for _ in range(3):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(s)
+        P.tt_diag_chase(rec, n, per_lane)
+        b.record(s)
+        torch.cuda.synchronize()
+        ts.append(a.elapsed_time(b) / 1e3)
+    del rec
+    return chains * n / statistics.median(ts)
 
 
 def measured_peaks():
@@ -646,6 +669,22 @@ def run_ours(args, rank, world, local_rank):
     else:
         roofline = {**hbm_eff, **common, "issue": None,
                     "note": "no ncu instruction count for this kernel source: HBM-effective roofline only"}
+    # L2-latency roof (live): a lockstep step is one 32-B record load whose
+    # address comes from the previous record; tt_diag_chase runs that pure
+    # dependent chase over as many records as the tree has nodes, with the
+    # traversal kernels' launch shape.  Independent-mode launches compare
+    # lane visits with the per-lane chase.
+    if args.variant == "autoropes" and not args.no_chase:
+        per_lane = lock_frac < 0.5
+        peak_steps = chase_ceiling(P, tree.n_nodes, device, per_lane)
+        ach = (visits if per_lane else wf) / (kms / 1e3)
+        roofline["chase"] = {
+            "bound": "l2-latency", "achieved": round(ach / 1e9, 3), "peak": round(peak_steps / 1e9, 3),
+            "unit": "G dependent record loads/s", "frac": round(ach / peak_steps, 4),
+            "achieved_def": ("lane visits" if per_lane else "lockstep warp fetches (tt_stats)") + " / kernel time",
+            "peak_def": f"tt_diag_chase over {tree.n_nodes} random-cycle 32-B records, "
+                        + ("one chain per lane" if per_lane else "one chain per warp (uniform loads)")
+                        + ", 4 x 256-thread CTAs per SM, measured live"}
     cpu = None
     if world == 1 and not args.no_cpu_baseline:
         try:

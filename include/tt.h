@@ -337,6 +337,20 @@ tt_status tt_kick_drift_permuted(const float *bodies, const float *vel, const fl
                                  float *vel_out, int32_t *ids_out, tt_stream s);
 
 /* ------------------------------------------------------------------------ */
+/* Diagnostics (not part of the method; SURVEY §8(d) "diagnostic ceilings").
+ * The dependent-load ceiling of a tree walk: every warp (per_lane = 0, the
+ * lockstep access: one warp-uniform 32-B record per step) or every lane
+ * (per_lane = 1, independent walks) follows its own chain through `nrec`
+ * 32-byte records for `steps` steps, with the traversal kernels' launch shape
+ * (256-thread CTAs, <= 4 per SM or ctas_per_sm).  records: device, 32-B
+ * aligned; the int32 at byte offset 16 of record i is the index of the next
+ * record (0 <= next < nrec).  sink: device uint32 (written only to keep the
+ * loads).  Asynchronous on `s`; the caller times it.  Errors:
+ * TT_ERR_INVALID_ARG, TT_ERR_CUDA.                                        */
+tt_status tt_diag_chase(const void *records, int64_t nrec, int32_t per_lane, int64_t steps, int32_t ctas_per_sm,
+                        uint32_t *sink, tt_stream s);
+
+/* ------------------------------------------------------------------------ */
 const char *tt_status_string(tt_status s);
 /* Last CUDA error code seen by the library (cudaError_t as int), 0 if none. */
 int32_t tt_last_cuda_error(void);

@@ -96,6 +96,7 @@ SIGNATURES = {
     "tt_traverse_knn": (I32, [P, P, I64, I32, I32, P, P, P, P]),
     "tt_traverse_vp": (I32, [P, P, I64, I32, P, P, P, P]),
     "tt_traverse_nn": (I32, [P, P, I64, I32, P, P, P, P]),
+    "tt_diag_chase": (I32, [P, I64, I32, I64, I32, P, P]),
     "tt_status_string": (C.c_char_p, [I32]),
     "tt_last_cuda_error": (I32, []),
     "tt_build_info": (C.c_char_p, []),

@@ -1,0 +1,62 @@
+// kern_diag.cu -- roofline diagnostics for a gather-bound tree walk (SURVEY
+// §8(d) "diagnostic ceilings"), sm_100a.  Not part of the method.
+//
+// A lockstep traversal step is one 32-B record load whose address comes from
+// the previous record (first child or rope), i.e. a dependent pointer chase
+// through an L2-resident array.  tt_diag_chase measures that ceiling on the
+// machine: every warp follows its own random cycle through `nrec` 32-B
+// records with the kernels' launch shape (persistent CTAs of 256 threads,
+// occupancy-many per SM) and the kernels' load (one ld.global.nc.v8 per
+// step):
+//   per_lane = 0: the 32 lanes of a warp load the same record (lockstep:
+//                 one request, one sector, broadcast);
+//   per_lane = 1: every lane follows its own chain (independent walks: 32
+//                 sectors per request) -- the random-gather ceiling.
+// Steps per second = warps (or lanes) x steps / time, timed by the caller.
+#include "kern_common.cuh"
+
+namespace {
+
+using namespace tt;
+
+__device__ __forceinline__ unsigned long long mix64(unsigned long long x) {
+    x ^= x >> 33;
+    x *= 0xff51afd7ed558ccdull;
+    x ^= x >> 33;
+    x *= 0xc4ceb9fe1a85ec53ull;
+    x ^= x >> 33;
+    return x;
+}
+
+__global__ void __launch_bounds__(256, 4) chase_kernel(const unsigned char *rec, long long nrec, long long steps,
+                                                       int per_lane, unsigned *sink) {
+    const unsigned long long gtid = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x;
+    const unsigned long long who = per_lane ? gtid : (gtid >> 5);
+    int cur = (int)(mix64(who + 0x9e3779b97f4a7c15ull) % (unsigned long long)nrec);
+    unsigned acc = 0;
+#pragma unroll 1
+    for (long long s = 0; s < steps; ++s) {
+        float4 g;
+        int4 t;
+        ldg_rec256(rec + (size_t)cur * 32u, g, t);
+        cur = t.x;                        // the next record depends on this one
+        acc += (unsigned)t.y ^ __float_as_uint(g.x);
+    }
+    if (acc == 0x9e3779b9u) sink[0] = acc;  // keep the loads (practically never taken)
+}
+
+}  // namespace
+
+int tt_launch_chase(const void *rec, long long nrec, long long steps, int per_lane, int ctas_per_sm, unsigned *sink,
+                    void *stream) {
+    int dev = 0, nsm = 0, occ = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, chase_kernel, 256, 0);
+    if (e != cudaSuccess) return (int)e;
+    if (occ > 4) occ = 4;  // the traversal kernels' residency (4 x 8 warps per SM)
+    if (ctas_per_sm > 0 && ctas_per_sm < occ) occ = ctas_per_sm;
+    chase_kernel<<<(unsigned)(nsm * occ), 256, 0, (cudaStream_t)stream>>>(static_cast<const unsigned char *>(rec),
+                                                                         nrec, steps, per_lane, sink);
+    return (int)cudaGetLastError();
+}

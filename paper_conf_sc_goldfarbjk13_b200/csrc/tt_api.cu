@@ -439,6 +439,17 @@ tt_status tt_traverse_nn(const tt_tree *t, const float *q, int64_t n, int32_t ld
     return finish_launch(tt_launch_nn(p, t->hdr.dim, cfg));
 }
 
+tt_status tt_diag_chase(const void *records, int64_t nrec, int32_t per_lane, int64_t steps, int32_t ctas_per_sm,
+                        uint32_t *sink, tt_stream s) {
+    if (!records || !sink || nrec <= 0 || nrec > INT32_MAX || steps < 0 || ctas_per_sm < 0 ||
+        (per_lane != 0 && per_lane != 1) || !aligned(records, 32))
+        return TT_ERR_INVALID_ARG;
+    tt_status st = have_device();
+    if (st != TT_OK) return st;
+    const int e = tt_launch_chase(records, nrec, steps, per_lane, ctas_per_sm, sink, s);
+    return e ? cuda_fail((cudaError_t)e) : TT_OK;
+}
+
 tt_status tt_kick_drift(float *bodies, float *vel, const float *acc, int64_t n, float dt_kick, float dt_drift,
                         tt_stream s) {
     if (n < 0) return TT_ERR_INVALID_ARG;

@@ -195,6 +195,10 @@ int tt_build_kd_gpu_impl(const float *pts, long long n, int dim, int ld, int lea
 int tt_build_vp_gpu_impl(const float *pts, long long n, int dim, int ld, void *stream, tt_blob_header *hdr,
                          void **blob);
 
+// Diagnostics (kern_diag.cu): dependent 32-B record chase.
+int tt_launch_chase(const void *rec, long long nrec, long long steps, int per_lane, int ctas_per_sm, unsigned *sink,
+                    void *stream);
+
 // Default mempool keeps freed stream-ordered scratch across syncs (kern_sort.cu).
 void tt_keep_pool_memory();
 

@@ -24,7 +24,7 @@ __all__ = [
     "HostTree", "Tree", "Stats", "TTError",
     "build_kd", "build_oct", "build_vp", "build_nn", "tt_tree_pack", "tt_tree_from_blob", "tt_tree_upload",
     "tt_build_oct_device", "tt_build_kd_device", "tt_build_vp_device", "tt_tree_download",
-    "tt_sort_points", "tt_schedule_tiles", "tt_traverse_bh", "tt_traverse_pc", "tt_traverse_knn", "tt_traverse_vp", "tt_traverse_nn",
+    "tt_sort_points", "tt_schedule_tiles", "tt_traverse_bh", "tt_traverse_pc", "tt_traverse_knn", "tt_traverse_vp", "tt_traverse_nn", "chase_records", "tt_diag_chase",
     "build_info",
 ]
 
@@ -405,3 +405,26 @@ def tt_traverse_nn(tree: Tree, q: torch.Tensor, out_idx: torch.Tensor | None = N
                                   out_d2.data_ptr(), C.byref(o), C.c_void_p(_stream_handle(stream))), "tt_traverse_nn")
     del keep
     return out_idx, out_d2
+
+
+# ---------------------------------------------------------------- diagnostics
+def chase_records(nrec: int, device, seed: int = 0) -> torch.Tensor:
+    """nrec 32-B records forming one random cycle (int32 at word 4 = next
+    index), for tt_diag_chase.  Plumbing only (a permutation)."""
+    g = torch.Generator(device=device).manual_seed(seed)
+    perm = torch.randperm(nrec, device=device, generator=g, dtype=torch.int64)
+    rec = torch.zeros((nrec, 8), dtype=torch.int32, device=device)
+    rec[perm, 4] = torch.roll(perm, -1).to(torch.int32)
+    rec[:, 5] = 1
+    return rec
+
+
+def tt_diag_chase(records: torch.Tensor, steps: int, per_lane: bool = False, ctas_per_sm: int = 0,
+                  stream=None) -> None:
+    """Dependent 32-B record chase with the traversal kernels' launch shape
+    (the walk's latency ceiling; include/tt.h).  Asynchronous; time it."""
+    _dev(records, torch.int32, "records", 8)
+    sink = torch.zeros(1, dtype=torch.int32, device=records.device)
+    check(L.load().tt_diag_chase(records.data_ptr(), records.shape[0], int(bool(per_lane)), int(steps),
+                                 int(ctas_per_sm), sink.data_ptr(), C.c_void_p(_stream_handle(stream))),
+          "tt_diag_chase")

@@ -701,3 +701,20 @@ def test_knn_dynamic_switch_results_exact(knn_small, sorted_):
             assert np.array_equal(st.warp_fetches.cpu().numpy(), wf)
     with pytest.raises(P.TTError):
         P.tt_traverse_knn(tree, qd, 8, switch_below=34)
+
+
+def test_diag_chase_runs_and_checks_args():
+    """The roofline diagnostic (tt_diag_chase) runs in both access modes and
+    rejects bad arguments; the chase records form one cycle."""
+    rec = P.chase_records(1000, "cuda", seed=3)
+    nxt = rec[:, 4].cpu().numpy()
+    seen, cur = set(), 0
+    for _ in range(1000):
+        seen.add(cur)
+        cur = int(nxt[cur])
+    assert len(seen) == 1000 and cur == 0
+    for per_lane in (False, True):
+        P.tt_diag_chase(rec, 100, per_lane)
+    torch.cuda.synchronize()
+    with pytest.raises(P.TTError):
+        P.tt_diag_chase(rec[:0], 10)
