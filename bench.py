@@ -67,7 +67,7 @@ def parse():
     ap.add_argument("--device-build", action="store_true",
                     help="build the tree on the GPU (tt_build_oct_device / tt_build_kd_device) instead of host "
                          "build + upload")
-    ap.add_argument("--variant", default="autoropes", choices=["autoropes", "recursive", "stack"],
+    ap.add_argument("--variant", default="autoropes", choices=["autoropes", "recursive", "stack", "split"],
                     help="recursive = the paper's naive recursive GPU baseline (ablation, N mode); "
                          "stack = explicit rope stacks, Fig.9b (ablation, BH and PC)")
     return ap.parse_args()

@@ -259,7 +259,12 @@ typedef struct tt_traverse_opts {
                                 global memory, lockstep = one (node, mask)
                                 stack per warp in shared memory;
                                 AUTO = BH lockstep, PC independent; 32-point
-                                warp tiles                                     */
+                                warp tiles;
+                                3 = split (PC only, else TT_ERR_UNSUPPORTED):
+                                each point's walk is split by subtree over a
+                                16-lane group (for point sets too small to fill
+                                the GPU one lane per point, e.g. configs[0]);
+                                mode is ignored, stats->visits only            */
     int32_t switch_below;    /* NEXT-3 dynamic L->N switching (kNN only, else
                                 must be 0): a lockstep warp whose active lanes at
                                 a node number fewer than this converts its warp
@@ -274,7 +279,8 @@ typedef struct tt_traverse_opts {
 typedef enum tt_variant {
     TT_VARIANT_AUTOROPES = 0,
     TT_VARIANT_RECURSIVE = 1,
-    TT_VARIANT_STACK = 2
+    TT_VARIANT_STACK = 2,
+    TT_VARIANT_SPLIT = 3
 } tt_variant;
 
 /* Barnes-Hut force pass (Fig.9): bodies float4 (x,y,z,m) rows;

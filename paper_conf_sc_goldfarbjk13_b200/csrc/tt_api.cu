@@ -80,7 +80,7 @@ tt_status setup_common(const tt_tree *t, int kind, int64_t n, const tt_traverse_
         if (o->ctas_per_sm < 0) return TT_ERR_INVALID_ARG;
         if (o->ctas_per_sm > 0) cfg.ctas_per_sm = o->ctas_per_sm;
         if (o->variant != TT_VARIANT_AUTOROPES && o->variant != TT_VARIANT_RECURSIVE &&
-            o->variant != TT_VARIANT_STACK)
+            o->variant != TT_VARIANT_STACK && o->variant != TT_VARIANT_SPLIT)
             return TT_ERR_INVALID_ARG;
         if (o->variant == TT_VARIANT_RECURSIVE && o->mode == TT_MODE_LOCKSTEP) return TT_ERR_UNSUPPORTED;
         cfg.variant = o->variant;
@@ -332,6 +332,7 @@ tt_status tt_traverse_bh(const tt_tree *t, const float *bodies, const int32_t *s
     if (!bodies || !acc_out || !aligned(bodies, 16) || !aligned(acc_out, 16)) return TT_ERR_INVALID_ARG;
     st = have_device();
     if (st != TT_OK) return st;
+    if (cfg.variant == TT_VARIANT_SPLIT) return TT_ERR_UNSUPPORTED;  // PC only
     p.bodies = reinterpret_cast<const float4 *>(bodies);
     p.self_ids = self_ids;
     // dsq_root = fl32(side^2 / theta^2) in fp64 (reading R8); theta = 0 -> +inf
@@ -368,6 +369,7 @@ tt_status tt_traverse_pc(const tt_tree *t, const float *q, int64_t n, int32_t ld
     p.count = count_out;
     return finish_launch(cfg.variant == TT_VARIANT_RECURSIVE ? tt_launch_pc_recursive(p, t->hdr.dim, cfg)
                          : cfg.variant == TT_VARIANT_STACK   ? tt_launch_pc_stack(p, t->hdr.dim, cfg)
+                         : cfg.variant == TT_VARIANT_SPLIT   ? tt_launch_pc_split(p, t->hdr.dim, cfg)
                                                              : tt_launch_pc(p, t->hdr.dim, cfg));
 }
 
@@ -391,7 +393,8 @@ tt_status tt_traverse_knn(const tt_tree *t, const float *q, int64_t n, int32_t l
     p.k = k;
     p.idx = idx_out;
     p.d2 = d2_out;
-    if (cfg.variant == TT_VARIANT_STACK) return TT_ERR_UNSUPPORTED;  // guided kernels already keep rope stacks
+    if (cfg.variant == TT_VARIANT_STACK || cfg.variant == TT_VARIANT_SPLIT)
+        return TT_ERR_UNSUPPORTED;  // guided kernels already keep rope stacks; SPLIT is PC only
     return finish_launch(cfg.variant == TT_VARIANT_RECURSIVE ? tt_launch_knn_recursive(p, t->hdr.dim, cfg)
                                                             : tt_launch_knn(p, t->hdr.dim, cfg));
 }
@@ -413,7 +416,8 @@ tt_status tt_traverse_vp(const tt_tree *t, const float *q, int64_t n, int32_t ld
     p.ld = ld;
     p.idx = idx_out;
     p.d2 = d2_out;
-    if (cfg.variant == TT_VARIANT_STACK) return TT_ERR_UNSUPPORTED;  // guided kernels already keep rope stacks
+    if (cfg.variant == TT_VARIANT_STACK || cfg.variant == TT_VARIANT_SPLIT)
+        return TT_ERR_UNSUPPORTED;  // guided kernels already keep rope stacks; SPLIT is PC only
     return finish_launch(cfg.variant == TT_VARIANT_RECURSIVE ? tt_launch_vp_recursive(p, t->hdr.dim, cfg)
                                                             : tt_launch_vp(p, t->hdr.dim, cfg));
 }

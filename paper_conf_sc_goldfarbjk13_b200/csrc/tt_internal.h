@@ -165,6 +165,8 @@ int tt_launch_vp_recursive(const tt_vp_params &p, int dim, const tt_launch_cfg &
 // explicit rope-stack variant, unguided kernels (kern_stack.cu)
 int tt_launch_bh_stack(const tt_bh_params &p, const tt_launch_cfg &cfg);
 int tt_launch_pc_stack(const tt_pc_params &p, int dim, const tt_launch_cfg &cfg);
+// one point's traversal split over a 16-lane group (kern_pc_split.cu)
+int tt_launch_pc_split(const tt_pc_params &p, int dim, const tt_launch_cfg &cfg);
 int tt_launch_sort(const tt_tree *t, const float *pts, int64_t n, int32_t ld, uint32_t *perm,
                    uint64_t *keys_out, void *stream);
 int tt_launch_schedule(const tt_tree *t, const float *pts, int64_t n, int32_t ld, const uint32_t *perm_in,

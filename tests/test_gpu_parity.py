@@ -718,3 +718,34 @@ def test_diag_chase_runs_and_checks_args():
     torch.cuda.synchronize()
     with pytest.raises(P.TTError):
         P.tt_diag_chase(rec[:0], 10)
+
+
+# --------------------------------------- PC traversal split over 8-lane groups
+@pytest.mark.parametrize("sorted_", [False, True])
+def test_pc_split_variant_exact(pc_setup, sorted_):
+    """TT_VARIANT_SPLIT: every point's walk divided by subtree over 16 lanes;
+    counts and per-point visit counts equal the recursive oracle's."""
+    c, p, ot, ref, tree = pc_setup
+    pd = dev(p)
+    order = P.tt_sort_points(tree, pd) if sorted_ else None
+    st = P.Stats.alloc(len(p), "cuda")
+    cnt = P.tt_traverse_pc(tree, pd, c["radius"], order=order, stats=st, variant="split").cpu().numpy()
+    assert np.array_equal(cnt.astype(np.uint32), ref.out[0])
+    assert np.array_equal(st.visits.cpu().numpy(), ref.visits)
+
+
+def test_pc_split_small_trees_and_buckets():
+    for n, leaf in ((1, 1), (2, 1), (3, 1), (7, 1), (9, 2), (200, 4), (3001, 1)):
+        p = ttgen.uniform(n, 3, seed=500 + n)
+        q = ttgen.uniform(37, 3, seed=600 + n)
+        ot = oracle.build_kd(p, leaf)
+        tree = P.tt_tree_upload(P.build_kd(p, leaf))
+        for r in (0.05, 0.3, 2.0):
+            ref = oracle.pc(ot, q, r, stats=True)
+            st = P.Stats.alloc(len(q), "cuda")
+            cnt = P.tt_traverse_pc(tree, dev(q), r, stats=st, variant="split").cpu().numpy()
+            assert np.array_equal(cnt.astype(np.uint32), ref.out[0]), (n, leaf, r)
+            assert np.array_equal(st.visits.cpu().numpy(), ref.visits), (n, leaf, r)
+    b = ttgen.plummer(100, seed=7)
+    with pytest.raises(P.TTError):
+        P.tt_traverse_bh(P.tt_tree_upload(P.build_oct(b)), dev(b), 0.5, 0.05, variant="split")
