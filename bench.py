@@ -239,16 +239,20 @@ KERNEL_SOURCE = {"bh": "kern_bh.cu", "pc": "kern_pc.cu", "knn": "kern_knn.cu", "
 def kernel_sha256(workload: str) -> str:
     """Hash of the sources that decide the traversal kernel's instruction
     stream for `workload` (its kern_*.cu, the shared device headers and the
-    build flags); nvcc output bytes themselves are not reproducible."""
+    nvcc flags of build.py); nvcc output bytes themselves are not
+    reproducible."""
     import hashlib
     kind = workload.rstrip("0123456789m").replace("steps", "")  # bh16m -> bh, bhsteps -> bh
     pkg = os.path.join(ROOT, "paper_conf_sc_goldfarbjk13_b200")
     files = [os.path.join(pkg, "csrc", f) for f in (KERNEL_SOURCE[kind], "kern_common.cuh", "tt_internal.h")]
-    files.append(os.path.join(pkg, "build.py"))
     h = hashlib.sha256()
     for f in files:
         h.update(os.path.basename(f).encode())
         h.update(open(f, "rb").read())
+    # the compile flags of build.py (not its source list)
+    flags = [ln.strip() for ln in open(os.path.join(pkg, "build.py")).read().splitlines()
+             if "ARCH" in ln or "-O3" in ln or "-Xptxas" in ln or "-lineinfo" in ln]
+    h.update("\n".join(flags).encode())
     return h.hexdigest()
 
 
@@ -412,8 +416,6 @@ def run_ours(args, rank, world, local_rank):
 
     # a0: tree (rank 0 builds; NCCL broadcast for N > 1) -- timed separately
     t0 = time.perf_counter()
-    if args.device_build and name == "nn":
-        raise SystemExit("--device-build: no GPU builder for the NN point-per-node kd-tree (host build only)")
     if args.device_build:
         # every rank builds the identical tree from the identical points (NEXT-1)
         data_dev = torch.from_numpy(np.ascontiguousarray(w["data"])).to(device)
@@ -421,6 +423,7 @@ def run_ours(args, rank, world, local_rank):
         t0 = time.perf_counter()
         tree = (P.tt_build_oct_device(data_dev) if name == "bh"
                 else P.tt_build_vp_device(data_dev) if name == "vp"
+                else P.tt_build_nn_device(data_dev) if name == "nn"
                 else P.tt_build_kd_device(data_dev, w["cfg"]["leaf"]))
         t1 = time.perf_counter()
         del data_dev
