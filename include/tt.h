@@ -175,6 +175,10 @@ tt_status tt_build_kd_device(const float *pts, int64_t n, int32_t dim, int32_t l
 /* NEXT-1: build a vantage-point tree (reading R12) on the GPU, same contract
  * as tt_build_kd_device (bytes identical to tt_tree_pack of tt_build_vp). */
 tt_status tt_build_vp_device(const float *pts, int64_t n, int32_t dim, int32_t ld, tt_stream s, tt_tree **out);
+/* NEXT-1 for the NEXT-3 NN tree: build the point-per-node kd-tree (reading
+ * R21) on the GPU, same contract as tt_build_kd_device (bytes identical to
+ * tt_tree_pack of tt_build_nn).                                            */
+tt_status tt_build_nn_device(const float *pts, int64_t n, int32_t dim, int32_t ld, tt_stream s, tt_tree **out);
 /* Copy the packed device blob back to host memory (bytes >= device_bytes of
  * tt_tree_get_info); synchronous.  E.g. to checkpoint a tree.              */
 tt_status tt_tree_download(const tt_tree *t, void *host_blob, size_t bytes);

@@ -84,6 +84,7 @@ SIGNATURES = {
     "tt_build_oct_device": (I32, [P, I64, P, P]),
     "tt_build_kd_device": (I32, [P, I64, I32, I32, I32, P, P]),
     "tt_build_vp_device": (I32, [P, I64, I32, I32, P, P]),
+    "tt_build_nn_device": (I32, [P, I64, I32, I32, P, P]),
     "tt_tree_download": (I32, [P, P, SZ]),
     "tt_kick_drift": (I32, [P, P, P, I64, F, F, P]),
     "tt_kick_drift_permuted": (I32, [P, P, P, P, P, I64, F, F, P, P, P, P]),

@@ -12,6 +12,10 @@
 
 #include "tt_internal.h"
 
+// build_nn_gpu.cu (declared here rather than in tt_internal.h)
+int tt_build_nn_gpu_impl(const float *pts, long long n, int dim, int ld, void *stream, tt_blob_header *hdr,
+                         void **blob);
+
 namespace {
 
 std::atomic<int> g_last_cuda_error{0};
@@ -237,6 +241,24 @@ tt_status tt_build_vp_device(const float *pts, int64_t n, int32_t dim, int32_t l
     tt_blob_header h;
     void *d_blob = nullptr;
     const int e = tt_build_vp_gpu_impl(pts, n, dim, ld, s, &h, &d_blob);
+    if (e) return cuda_fail((cudaError_t)e);
+    if (h.height > TT_MAX_HEIGHT) {
+        cudaFree(d_blob);
+        return TT_ERR_TREE_TOO_DEEP;
+    }
+    st = adopt_blob(h, d_blob, (cudaStream_t)s, out);
+    if (st != TT_OK) cudaFree(d_blob);
+    return st;
+}
+
+tt_status tt_build_nn_device(const float *pts, int64_t n, int32_t dim, int32_t ld, tt_stream s, tt_tree **out) {
+    if (!pts || !out || n <= 0 || n > INT32_MAX / 2 || dim <= 0 || dim > TT_MAX_DIM || ld < dim)
+        return TT_ERR_INVALID_ARG;
+    tt_status st = have_device();
+    if (st != TT_OK) return st;
+    tt_blob_header h;
+    void *d_blob = nullptr;
+    const int e = tt_build_nn_gpu_impl(pts, n, dim, ld, s, &h, &d_blob);
     if (e) return cuda_fail((cudaError_t)e);
     if (h.height > TT_MAX_HEIGHT) {
         cudaFree(d_blob);

@@ -23,7 +23,7 @@ from ._lib import TTError, check
 __all__ = [
     "HostTree", "Tree", "Stats", "TTError",
     "build_kd", "build_oct", "build_vp", "build_nn", "tt_tree_pack", "tt_tree_from_blob", "tt_tree_upload",
-    "tt_build_oct_device", "tt_build_kd_device", "tt_build_vp_device", "tt_tree_download",
+    "tt_build_oct_device", "tt_build_kd_device", "tt_build_vp_device", "tt_build_nn_device", "tt_tree_download",
     "tt_sort_points", "tt_schedule_tiles", "tt_traverse_bh", "tt_traverse_pc", "tt_traverse_knn", "tt_traverse_vp", "tt_traverse_nn", "chase_records", "tt_diag_chase",
     "build_info",
 ]
@@ -215,6 +215,15 @@ def tt_build_kd_device(pts: torch.Tensor, leaf_size: int = 1, stream=None) -> Tr
     h = C.c_void_p()
     check(L.load().tt_build_kd_device(pts.data_ptr(), pts.shape[0], pts.shape[1], pts.stride(0), int(leaf_size),
                                       C.c_void_p(_stream_handle(stream)), C.byref(h)), "tt_build_kd_device")
+    return Tree(h)
+
+
+def tt_build_nn_device(pts: torch.Tensor, stream=None) -> Tree:
+    """Build the NN point-per-node kd-tree (R21) on the GPU from (n, dim) device points."""
+    _dev(pts, torch.float32, "pts", 1)
+    h = C.c_void_p()
+    check(L.load().tt_build_nn_device(pts.data_ptr(), pts.shape[0], pts.shape[1], pts.stride(0),
+                                      C.c_void_p(_stream_handle(stream)), C.byref(h)), "tt_build_nn_device")
     return Tree(h)
 
 

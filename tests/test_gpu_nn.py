@@ -111,3 +111,18 @@ def test_nn_1m_sampled():
     ref = oracle.nn(oracle.build_nn(p), q[sample])
     assert np.array_equal(idx.cpu().numpy()[sample], ref.out[0])
     assert np.array_equal(d2.cpu().numpy()[sample], ref.out[1])
+
+
+@pytest.mark.parametrize("n,dim", [(1, 3), (2, 3), (3, 2), (7, 7), (5_000, 16), (20_011, 7), (1_000_000, 7)])
+def test_gpu_nn_build_is_byte_identical_to_host_pack(n, dim):
+    """tt_build_nn_device writes the same blob bytes as tt_tree_pack of the
+    host builder (duplicates included: ties broken by id)."""
+    p = ttgen.gaussian_mixture(n, dim, seed=320, components=6)
+    if n > 100:
+        p[50:60] = p[7]
+    host_blob = P.build_nn(p).pack()
+    t = P.tt_build_nn_device(dev(p))
+    gpu_blob = P.tt_tree_download(t)
+    assert gpu_blob.size == host_blob.size
+    diff = np.nonzero(gpu_blob != host_blob)[0]
+    assert diff.size == 0, f"{diff.size} bytes differ, first at {diff[:8]}"
