@@ -67,7 +67,7 @@ def parse():
     ap.add_argument("--device-build", action="store_true",
                     help="build the tree on the GPU (tt_build_oct_device / tt_build_kd_device) instead of host "
                          "build + upload")
-    ap.add_argument("--variant", default="autoropes", choices=["autoropes", "recursive", "stack", "split"],
+    ap.add_argument("--variant", default="autoropes", choices=["autoropes", "recursive", "stack", "split", "groups", "ropes"],
                     help="recursive = the paper's naive recursive GPU baseline (ablation, N mode); "
                          "stack = explicit rope stacks, Fig.9b (ablation, BH and PC)")
     return ap.parse_args()
@@ -233,7 +233,7 @@ def load_counts(workload: str, mode: str):
         return None
 
 
-KERNEL_SOURCE = {"bh": "kern_bh.cu", "pc": "kern_pc.cu", "knn": "kern_knn.cu", "vp": "kern_vp.cu", "nn": "kern_nn.cu"}
+KERNEL_SOURCE = {"bh": "kern_bh_group.cu", "pc": "kern_pc.cu", "knn": "kern_knn.cu", "vp": "kern_vp.cu", "nn": "kern_nn.cu"}
 
 
 def kernel_sha256(workload: str) -> str:
@@ -524,7 +524,7 @@ def run_ours(args, rank, world, local_rank):
     traverse(q_shard, out_shard, order_buf, st)
     torch.cuda.synchronize()
     visits = int(st.visits.to(torch.int64).sum().item())
-    tile_pts = P._lib.TILE_POINTS[tree.kind] if args.variant == "autoropes" else 32
+    tile_pts = P._lib.TILE_POINTS[tree.kind] if args.variant in ("autoropes", "groups", "ropes") else 32
     tiles = -(-m // tile_pts)
     wf = int(st.warp_fetches[:tiles].to(torch.int64).sum().item())
     lock_frac = float((st.warp_mode[:tiles] == 1).float().mean().item())
@@ -639,7 +639,7 @@ def run_ours(args, rank, world, local_rank):
     bpv = BYTES_PER_VISIT[name]
     alg_bytes = visits * bpv + m * BYTES_PER_POINT_IO[name]  # per launch on rank 0
     achieved = alg_bytes / (kms / 1e3) / 1e9
-    kernel_name = {"bh": "bh_kernel", "pc": "pc_kernel", "knn": "knn_kernel", "vp": "vp_kernel", "nn": "nn_kernel"}[name]
+    kernel_name = {"bh": "bh_group_kernel", "pc": "pc_kernel", "knn": "knn_kernel", "vp": "vp_kernel", "nn": "nn_kernel"}[name]
     cnt = load_counts(name, args.mode) if not args.unsorted and args.variant == "autoropes" else None
     clocks = clk.summary()
     sm_mhz = clocks.get("sm_mhz") or float(peaks.get("sm_max_mhz", 1965.0))

@@ -252,7 +252,8 @@ typedef struct tt_traverse_opts {
     const tt_stats *stats;   /* host struct of device pointers, nullable         */
     int32_t block_threads;   /* 0 = default (256)                               */
     int32_t ctas_per_sm;     /* 0 = occupancy maximum                            */
-    int32_t variant;         /* tt_variant: 0 = autoropes (the method);
+    int32_t variant;         /* tt_variant: 0 = autoropes (the method; for BH
+                                the child-group lockstep walk, 4);
                                 1 = naive recursive baseline (P:L1084-1090,
                                 independent mode only -- LOCKSTEP is
                                 TT_ERR_UNSUPPORTED; it fills stats->visits only,
@@ -268,7 +269,16 @@ typedef struct tt_traverse_opts {
                                 each point's walk is split by subtree over a
                                 16-lane group (for point sets too small to fill
                                 the GPU one lane per point, e.g. configs[0]);
-                                mode is ignored, stats->visits only            */
+                                mode is ignored, stats->visits only;
+                                4 = groups (BH only; BH's default, 0 selects
+                                it): lockstep warps expand a whole cell per
+                                step -- its children, stored contiguously in a
+                                group array built on the first such call and
+                                kept with the tree, are loaded together and
+                                tested by every body that opened the cell;
+                                independent warps take the stackless rope walk;
+                                5 = ropes (BH only): the per-node Fig.8
+                                lockstep walk over stored ropes             */
     int32_t switch_below;    /* NEXT-3 dynamic L->N switching (kNN only, else
                                 must be 0): a lockstep warp whose active lanes at
                                 a node number fewer than this converts its warp
@@ -284,7 +294,9 @@ typedef enum tt_variant {
     TT_VARIANT_AUTOROPES = 0,
     TT_VARIANT_RECURSIVE = 1,
     TT_VARIANT_STACK = 2,
-    TT_VARIANT_SPLIT = 3
+    TT_VARIANT_SPLIT = 3,
+    TT_VARIANT_GROUPS = 4,
+    TT_VARIANT_ROPES = 5
 } tt_variant;
 
 /* Barnes-Hut force pass (Fig.9): bodies float4 (x,y,z,m) rows;

@@ -18,7 +18,7 @@ STATUS = {0: "TT_OK", -1: "TT_ERR_INVALID_ARG", -2: "TT_ERR_CUDA", -3: "TT_ERR_O
 KIND_OCT, KIND_KD, KIND_VP, KIND_NN = 1, 2, 3, 4
 MODE = {"auto": 0, "lockstep": 1, "L": 1, "independent": 2, "N": 2}
 MEM_HOST, MEM_DEVICE = 0, 1
-VARIANT = {"autoropes": 0, "recursive": 1, "stack": 2, "split": 3}
+VARIANT = {"autoropes": 0, "recursive": 1, "stack": 2, "split": 3, "groups": 4, "ropes": 5}
 MAX_HEIGHT, MAX_DIM, MAX_K = 48, 16, 32
 BH_POINTS_PER_LANE = 2
 TILE_POINTS = {"oct": 32 * BH_POINTS_PER_LANE, "kd": 32, "vp": 32, "nn": 32}  # points per warp tile (tt_stats warp_*)

@@ -14,7 +14,7 @@ BUILD = os.path.join(HERE, "_build")
 LIB = os.path.join(HERE, "libtt.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-CU = ["tt_api.cu", "kern_bh.cu", "kern_pc.cu", "kern_pc_split.cu", "kern_knn.cu", "kern_vp.cu", "kern_nn.cu", "kern_sort.cu", "kern_sched.cu", "kern_recursive.cu", "kern_stack.cu",
+CU = ["tt_api.cu", "kern_bh.cu", "kern_bh_group.cu", "kern_pc.cu", "kern_pc_split.cu", "kern_knn.cu", "kern_vp.cu", "kern_nn.cu", "kern_sort.cu", "kern_sched.cu", "kern_recursive.cu", "kern_stack.cu",
       "build_oct_gpu.cu", "build_kd_gpu.cu", "build_vp_gpu.cu", "build_nn_gpu.cu",
       "kern_integrate.cu", "kern_diag.cu"]
 CPP = ["host_build.cpp", "pack.cpp"]

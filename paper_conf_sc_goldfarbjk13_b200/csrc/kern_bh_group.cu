@@ -1,0 +1,363 @@
+// kern_bh_group.cu -- Barnes-Hut lockstep walk by child groups
+// (TT_VARIANT_GROUPS), sm_100a.
+//
+// The lockstep walk of kern_bh.cu makes one dependent L2 round trip per node
+// (next = first child or rope of the record just loaded), and that latency is
+// what binds it (0.58 of a pure pointer chase).  Here the warp
+// expands a whole cell at once: when any of its bodies opens a cell, the
+// cell's children -- stored contiguously in a group array built once per tree
+// from the preorder blob -- are loaded together (independent loads, one round
+// trip) and every active body tests each of them.  A child some body opens is
+// pushed with the ballot of the bodies that opened it (Fig.8's per-entry
+// mask, here one mask per body row of the 64-body tile).  Every body tests
+// exactly the nodes its recursive walk tests (the children of the cells it
+// opens), so per-body visit counts equal the oracle's and the warp fetches
+// equal the Fig.8 union; only the order in which a body's terms are summed
+// differs (within the 1e-4 bar: fp32 partials flushed to fp64).
+//
+// Group record (32 B, like tt_oct_rec): {com.xyz, mass} +
+// {group offset of the node's children | -1, number of children, body | -1,
+// level}; entry 0 is the root, the children of a cell are contiguous.
+#include <climits>
+#include <cfloat>
+#include <cmath>
+
+#include <cub/device/device_scan.cuh>
+
+#include "kern_common.cuh"
+
+namespace {
+
+using namespace tt;
+
+constexpr int kBlock = 256;
+constexpr int kSmemHdr = 384;          // mbarrier + dsq table (as kern_bh.cu)
+constexpr int kBPL = TT_BH_POINTS_PER_LANE;
+constexpr int kStackPerWarp = 8 * 40;  // <= 8 children pushed per level, height <= 33 (R9) + slack
+constexpr int kFlushEvery = 16;        // children between fp32 -> fp64 flushes
+
+struct GroupEntry {
+    int off, nk;
+    unsigned m0, m1;  // bodies (row 0 / row 1 of the tile) that opened the cell
+};
+
+// ------------------------------------------------------------ group build
+__global__ void nkids_kernel(const tt_oct_rec *rec, long long nn, int *nk) {
+    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < nn; v += (long long)gridDim.x * blockDim.x) {
+        int c = rec[v].first_child, k = 0;
+        const int end = rec[v].skip;
+        while (c >= 0 && c != end) {
+            ++k;
+            c = rec[c].skip;
+        }
+        nk[v] = k;
+    }
+}
+
+__global__ void groups_fill_kernel(const tt_oct_rec *rec, long long nn, const int *nk, const int *goff,
+                                   tt_oct_rec *grp) {
+    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < nn; v += (long long)gridDim.x * blockDim.x) {
+        if (v == 0) {  // the root's own entry
+            tt_oct_rec r = rec[0];
+            r.first_child = nk[0] > 0 ? 1 + goff[0] : -1;
+            r.skip = nk[0];
+            grp[0] = r;
+        }
+        int c = rec[v].first_child, k = 0;
+        const int end = rec[v].skip;
+        while (c >= 0 && c != end) {
+            tt_oct_rec r = rec[c];
+            r.first_child = nk[c] > 0 ? 1 + goff[c] : -1;
+            r.skip = nk[c];
+            grp[1 + goff[v] + k] = r;
+            ++k;
+            c = rec[c].skip;
+        }
+    }
+}
+
+__device__ __forceinline__ float dsq_at(int dsq_bits, int lvl) { return __int_as_float(dsq_bits - (lvl << 24)); }
+
+#ifndef TT_BHG_MINB
+#define TT_BHG_MINB 4
+#endif
+template <bool STATS, bool EXP_DSQ>
+__global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_bh_params P, const tt_oct_rec *grp) {
+    extern __shared__ __align__(128) unsigned char smem[];
+    float *s_dsq = reinterpret_cast<float *>(smem + 16);
+    GroupEntry *s_stack = reinterpret_cast<GroupEntry *>(smem + kSmemHdr);
+    if (threadIdx.x == 0) {
+        float d = P.dsq_root;
+        for (int l = 0; l < 64; ++l) {
+            s_dsq[l] = d;
+            d = __fmul_rn(d, 0.25f);
+        }
+    }
+    __syncthreads();
+
+    const int lane = threadIdx.x & 31;
+    const int warp = threadIdx.x >> 5;
+    GroupEntry *stk = s_stack + warp * kStackPerWarp;
+    // per-warp staging buffer of one child group (<= 8 records)
+    float4 *gbuf = reinterpret_cast<float4 *>(s_stack + (kBlock / 32) * kStackPerWarp) + warp * 16;
+    int4 *tbuf = reinterpret_cast<int4 *>(gbuf + 8);
+    const tt_oct_rec *g_rec = static_cast<const tt_oct_rec *>(P.c.tree.rec);
+    const long long n = P.c.n;
+    const int dsq_bits = __float_as_int(P.dsq_root);
+    const float nz = opaque_neg_zero(n);
+    const float2 e22 = make_float2(P.eps2, P.eps2);
+    const long long ntiles = (n + 32 * kBPL - 1) / (32 * kBPL);
+    for (;;) {
+        const long long tile = next_tile(P.c.counter);
+        if (tile >= ntiles) break;
+        long long pid[kBPL];
+        float4 b[kBPL];
+        int self[kBPL];
+        bool valid[kBPL];
+#pragma unroll
+        for (int j = 0; j < kBPL; ++j) {
+            const long long pos = tile * 32 * kBPL + 32 * j + lane;
+            valid[j] = pos < n;
+            pid[j] = valid[j] ? (P.c.order ? (long long)P.c.order[pos] : pos) : 0;
+            b[j] = valid[j] ? __ldg(P.bodies + pid[j]) : make_float4(0.f, 0.f, 0.f, 0.f);
+            self[j] = valid[j] ? (P.self_ids ? __ldg(P.self_ids + pid[j]) : (int)pid[j]) : -2;
+        }
+        bool lock = P.c.mode != TT_MODE_INDEPENDENT;
+        if (P.c.mode == TT_MODE_AUTO && P.c.auto_min_depth > 0) {
+            // the coherence test of kern_bh.cu (reading R19)
+            const int T = min(P.c.auto_min_depth, 10);
+            const float lo_x = (float)(P.c.root_center[0] - 0.5 * P.c.root_side);
+            const float lo_y = (float)(P.c.root_center[1] - 0.5 * P.c.root_side);
+            const float lo_z = (float)(P.c.root_center[2] - 0.5 * P.c.root_side);
+            const float sc = (float)((double)(1 << T) / P.c.root_side);
+            const int cmax = (1 << T) - 1;
+            unsigned cell[kBPL];
+#pragma unroll
+            for (int j = 0; j < kBPL; ++j) {
+                const unsigned cx = (unsigned)min(max(__float2int_rd((b[j].x - lo_x) * sc), 0), cmax);
+                const unsigned cy = (unsigned)min(max(__float2int_rd((b[j].y - lo_y) * sc), 0), cmax);
+                const unsigned cz = (unsigned)min(max(__float2int_rd((b[j].z - lo_z) * sc), 0), cmax);
+                cell[j] = (cx << (2 * T)) | (cy << T) | cz;
+            }
+            int changes = 0;
+#pragma unroll
+            for (int j = 0; j < kBPL; ++j) {
+                const unsigned up = __shfl_up_sync(TT_FULL, cell[j], 1);
+                const unsigned prev_row = j > 0 ? __shfl_sync(TT_FULL, cell[j > 0 ? j - 1 : 0], 31) : cell[j];
+                const unsigned prev = lane > 0 ? up : prev_row;
+                changes += __popc(__ballot_sync(TT_FULL, valid[j] && cell[j] != prev));
+            }
+            lock = P.c.auto_min_depth < 64 && changes < kAutoMaxChanges;
+        }
+
+        double X[kBPL], Y[kBPL], Z[kBPL];
+        unsigned visits[kBPL];
+#pragma unroll
+        for (int j = 0; j < kBPL; ++j) {
+            X[j] = Y[j] = Z[j] = 0.0;
+            visits[j] = 0;
+        }
+        unsigned fetches = 0, steps = 0;
+        if (lock) {
+            static_assert(kBPL == 2, "group walk is written for body pairs");
+            const float2 nbx = add2_rn(make_float2(nz, nz), make_float2(-b[0].x, -b[1].x));
+            const float2 nby = add2_rn(make_float2(nz, nz), make_float2(-b[0].y, -b[1].y));
+            const float2 nbz = add2_rn(make_float2(nz, nz), make_float2(-b[0].z, -b[1].z));
+            float2 ax = make_float2(0.f, 0.f), ay = ax, az = ax;
+            int since_flush = 0;
+            int sp = 0;
+            // the root group: entry 0 alone, tested by every valid body
+            int goff = 0, gnk = 1;
+            unsigned m0 = __ballot_sync(TT_FULL, valid[0]), m1 = __ballot_sync(TT_FULL, valid[1]);
+            for (;;) {
+                const bool in0 = (m0 >> lane) & 1u, in1 = (m1 >> lane) & 1u;
+                // stage the group: lane k loads child k (one request for the
+                // whole group, one round trip), the warp reads them back from
+                // shared memory with broadcast loads
+                if (lane < gnk) {
+                    float4 sg;
+                    int4 st4;
+                    ldg_rec256(grp + goff + lane, sg, st4);
+                    gbuf[lane] = sg;
+                    tbuf[lane] = st4;
+                }
+                __syncwarp();
+#pragma unroll 1
+                for (int k = 0; k < gnk; ++k) {
+                    const float4 g = gbuf[k];
+                    const int4 t = tbuf[k];
+                    if (STATS) {
+                        ++fetches;
+                        ++steps;
+                        visits[0] += in0;
+                        visits[1] += in1;
+                    }
+                    const float dl = EXP_DSQ ? dsq_at(dsq_bits, t.w) : s_dsq[t.w];
+                    const float2 dx = add2_rn(make_float2(g.x, g.x), nbx);
+                    const float2 dy = add2_rn(make_float2(g.y, g.y), nby);
+                    const float2 dz = add2_rn(make_float2(g.z, g.z), nbz);
+                    const float2 drsq = add2_rn(add2_rn(sqr2_rn(dx, nz), sqr2_rn(dy, nz)), sqr2_rn(dz, nz));
+                    const bool cell = t.x >= 0;
+                    const bool o0 = in0 && cell && drsq.x < dl;
+                    const bool o1 = in1 && cell && drsq.y < dl;
+                    const float2 mw = make_float2(in0 && !o0 && t.z != self[0] ? g.w : 0.f,
+                                                  in1 && !o1 && t.z != self[1] ? g.w : 0.f);
+                    const float2 r = add2_rn(drsq, e22);
+                    const float2 inv = make_float2(rsqrt_ftz(r.x), rsqrt_ftz(r.y));
+                    const float2 f = mul2_rn(mul2_rn(mw, mul2_rn(inv, inv)), inv);
+                    ax = fma2_rn(f, dx, ax);
+                    ay = fma2_rn(f, dy, ay);
+                    az = fma2_rn(f, dz, az);
+                    const unsigned om0 = __ballot_sync(TT_FULL, o0), om1 = __ballot_sync(TT_FULL, o1);
+                    if (om0 | om1) {
+                        if (lane == 0) stk[sp] = GroupEntry{t.x, t.y, om0, om1};
+                        ++sp;
+                    }
+                }
+                __syncwarp();  // the group buffer is reused by the next pop
+                since_flush += gnk;
+                if (since_flush >= kFlushEvery) {  // warp-uniform cadence
+                    X[0] += (double)ax.x;
+                    Y[0] += (double)ay.x;
+                    Z[0] += (double)az.x;
+                    X[1] += (double)ax.y;
+                    Y[1] += (double)ay.y;
+                    Z[1] += (double)az.y;
+                    ax = ay = az = make_float2(0.f, 0.f);
+                    since_flush = 0;
+                }
+                if (sp == 0) break;
+                --sp;
+                __syncwarp();
+                int4 e = make_int4(0, 0, 0, 0);
+                if (lane == 0) e = *reinterpret_cast<const int4 *>(stk + sp);
+                goff = __shfl_sync(TT_FULL, e.x, 0);
+                gnk = __shfl_sync(TT_FULL, e.y, 0);
+                m0 = (unsigned)__shfl_sync(TT_FULL, e.z, 0);
+                m1 = (unsigned)__shfl_sync(TT_FULL, e.w, 0);
+            }
+            X[0] += (double)ax.x;
+            Y[0] += (double)ay.x;
+            Z[0] += (double)az.x;
+            X[1] += (double)ax.y;
+            Y[1] += (double)ay.y;
+            Z[1] += (double)az.y;
+        } else {
+            // independent: the stackless rope walk of kern_bh.cu over the
+            // preorder records (through L1/L2)
+#pragma unroll
+            for (int j = 0; j < kBPL; ++j) {
+                int cur = valid[j] ? 0 : TT_END;
+                float sx = 0.f, sy = 0.f, sz = 0.f;
+                int cnt = 0;
+                while (cur != TT_END) {
+                    float4 g;
+                    int4 t;
+                    ldg_rec256(g_rec + cur, g, t);
+                    if (STATS) ++visits[j];
+                    const float dx = __fsub_rn(g.x, b[j].x), dy = __fsub_rn(g.y, b[j].y),
+                                dz = __fsub_rn(g.z, b[j].z);
+                    const float drsq = __fadd_rn(__fadd_rn(__fmul_rn(dx, dx), __fmul_rn(dy, dy)), __fmul_rn(dz, dz));
+                    const float dl = EXP_DSQ ? dsq_at(dsq_bits, t.w) : s_dsq[t.w];
+                    const bool open = t.x >= 0 && drsq < dl;
+                    const float inv = rsqrt_ftz(__fadd_rn(drsq, P.eps2));
+                    const float f = (!open && t.z != self[j]) ? g.w * (inv * inv) * inv : 0.0f;
+                    sx = fmaf(f, dx, sx);
+                    sy = fmaf(f, dy, sy);
+                    sz = fmaf(f, dz, sz);
+                    if (++cnt == kFlushEvery) {
+                        X[j] += (double)sx;
+                        Y[j] += (double)sy;
+                        Z[j] += (double)sz;
+                        sx = sy = sz = 0.f;
+                        cnt = 0;
+                    }
+                    cur = open ? t.x : t.y;
+                }
+                X[j] += (double)sx;
+                Y[j] += (double)sy;
+                Z[j] += (double)sz;
+            }
+            if (STATS) {
+                fetches = warp_sum(visits[0] + visits[1]);
+                steps = __reduce_max_sync(TT_FULL, max(visits[0], visits[1]));
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < kBPL; ++j) {
+            if (valid[j]) {
+                P.acc[pid[j]] = make_float4((float)X[j], (float)Y[j], (float)Z[j], 0.f);
+                if (STATS && P.c.st_visits) P.c.st_visits[pid[j]] = visits[j];
+            }
+        }
+        if (STATS) write_warp_stats(P.c, tile, fetches, steps, lock);
+        __syncwarp();
+    }
+    cta_finish(P.c.counter);
+}
+
+template <bool STATS, bool EXP_DSQ>
+int launch(const tt_bh_params &p, const tt_oct_rec *grp, const tt_launch_cfg &cfg) {
+    const size_t smem = kSmemHdr + (size_t)(kBlock / 32) * kStackPerWarp * sizeof(GroupEntry) + (kBlock / 32) * 16 * 16;
+    auto kern = bh_group_kernel<STATS, EXP_DSQ>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return (int)e;
+    int dev = 0, nsm = 0, occ = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kBlock, smem);
+    if (e != cudaSuccess) return (int)e;
+    if (cfg.ctas_per_sm > 0 && cfg.ctas_per_sm < occ) occ = cfg.ctas_per_sm;
+    if (occ < 1) occ = 1;
+    const long long ntiles = (p.c.n + 32 * kBPL - 1) / (32 * kBPL);
+    long long grid = (long long)nsm * occ;
+    const long long need = (ntiles + kBlock / 32 - 1) / (kBlock / 32);
+    if (grid > need) grid = need;
+    if (grid < 1) grid = 1;
+    kern<<<(unsigned)grid, kBlock, smem, (cudaStream_t)cfg.stream>>>(p, grp);
+    return (int)cudaGetLastError();
+}
+
+}  // namespace
+
+// Child-group array of an oct tree (built once per tree, kept with it).
+int tt_bh_groups_build(const void *rec, long long nn, void *stream, void **grp_out) {
+    cudaStream_t s = (cudaStream_t)stream;
+    const tt_oct_rec *r = static_cast<const tt_oct_rec *>(rec);
+    int *nk = nullptr, *goff = nullptr;
+    void *tmp = nullptr, *grp = nullptr;
+    size_t tb = 0;
+    cudaError_t e = cudaMallocAsync((void **)&nk, sizeof(int) * nn, s);
+    if (!e) e = cudaMallocAsync((void **)&goff, sizeof(int) * nn, s);
+    if (!e) e = cub::DeviceScan::ExclusiveSum(nullptr, tb, nk, goff, (int)nn, s);
+    if (!e) e = cudaMallocAsync(&tmp, tb, s);
+    if (!e) e = cudaMalloc(&grp, sizeof(tt_oct_rec) * (size_t)nn);
+    const unsigned G = (unsigned)std::min<long long>((nn + 255) / 256, 148 * 8);
+    if (!e) {
+        nkids_kernel<<<G, 256, 0, s>>>(r, nn, nk);
+        e = cub::DeviceScan::ExclusiveSum(tmp, tb, nk, goff, (int)nn, s);
+    }
+    if (!e) {
+        groups_fill_kernel<<<G, 256, 0, s>>>(r, nn, nk, goff, static_cast<tt_oct_rec *>(grp));
+        e = cudaGetLastError();
+    }
+    if (tmp) cudaFreeAsync(tmp, s);
+    if (goff) cudaFreeAsync(goff, s);
+    if (nk) cudaFreeAsync(nk, s);
+    if (!e) e = cudaStreamSynchronize(s);
+    if (e) {
+        if (grp) cudaFree(grp);
+        return (int)e;
+    }
+    *grp_out = grp;
+    return 0;
+}
+
+int tt_launch_bh_group(const tt_bh_params &p, const void *grp, const tt_launch_cfg &cfg) {
+    const bool stats = p.c.st_visits || p.c.st_warp_fetches || p.c.st_warp_steps || p.c.st_warp_mode;
+    const float r = p.dsq_root;
+    const bool exp_ok = r < INFINITY && r > 0.f && std::ldexp((double)r, -2 * p.c.height) >= (double)FLT_MIN;
+    const tt_oct_rec *g = static_cast<const tt_oct_rec *>(grp);
+    if (stats) return exp_ok ? launch<true, true>(p, g, cfg) : launch<true, false>(p, g, cfg);
+    return exp_ok ? launch<false, true>(p, g, cfg) : launch<false, false>(p, g, cfg);
+}

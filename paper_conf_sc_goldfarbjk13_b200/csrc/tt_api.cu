@@ -84,7 +84,8 @@ tt_status setup_common(const tt_tree *t, int kind, int64_t n, const tt_traverse_
         if (o->ctas_per_sm < 0) return TT_ERR_INVALID_ARG;
         if (o->ctas_per_sm > 0) cfg.ctas_per_sm = o->ctas_per_sm;
         if (o->variant != TT_VARIANT_AUTOROPES && o->variant != TT_VARIANT_RECURSIVE &&
-            o->variant != TT_VARIANT_STACK && o->variant != TT_VARIANT_SPLIT)
+            o->variant != TT_VARIANT_STACK && o->variant != TT_VARIANT_SPLIT && o->variant != TT_VARIANT_GROUPS &&
+            o->variant != TT_VARIANT_ROPES)
             return TT_ERR_INVALID_ARG;
         if (o->variant == TT_VARIANT_RECURSIVE && o->mode == TT_MODE_LOCKSTEP) return TT_ERR_UNSUPPORTED;
         cfg.variant = o->variant;
@@ -295,6 +296,7 @@ tt_status tt_tree_free(tt_tree *t) {
     if (!t) return TT_OK;
     cudaError_t e1 = cudaFree(t->d_blob);
     cudaError_t e2 = cudaFree(t->d_counters);
+    if (t->d_grp) cudaFree(t->d_grp);
     delete t;
     if (e1 != cudaSuccess) return cuda_fail(e1);
     if (e2 != cudaSuccess) return cuda_fail(e2);
@@ -355,6 +357,17 @@ tt_status tt_traverse_bh(const tt_tree *t, const float *bodies, const int32_t *s
     st = have_device();
     if (st != TT_OK) return st;
     if (cfg.variant == TT_VARIANT_SPLIT) return TT_ERR_UNSUPPORTED;  // PC only
+    // BH default: lockstep warps walk by child groups (kern_bh_group.cu);
+    // TT_VARIANT_ROPES keeps the per-node lockstep walk over ropes (kern_bh.cu)
+    if (cfg.variant == TT_VARIANT_AUTOROPES) cfg.variant = TT_VARIANT_GROUPS;
+    if (cfg.variant == TT_VARIANT_GROUPS) {
+        tt_tree *mt = const_cast<tt_tree *>(t);
+        std::lock_guard<std::mutex> lk(mt->grp_mu);
+        if (!mt->d_grp) {
+            const int e = tt_bh_groups_build(t->dev.rec, t->hdr.n_nodes, s, &mt->d_grp);
+            if (e) return cuda_fail((cudaError_t)e);
+        }
+    }
     p.bodies = reinterpret_cast<const float4 *>(bodies);
     p.self_ids = self_ids;
     // dsq_root = fl32(side^2 / theta^2) in fp64 (reading R8); theta = 0 -> +inf
@@ -368,7 +381,8 @@ tt_status tt_traverse_bh(const tt_tree *t, const float *bodies, const int32_t *s
     p.acc = reinterpret_cast<float4 *>(acc_out);
     return finish_launch(cfg.variant == TT_VARIANT_RECURSIVE ? tt_launch_bh_recursive(p, cfg)
                          : cfg.variant == TT_VARIANT_STACK   ? tt_launch_bh_stack(p, cfg)
-                                                             : tt_launch_bh(p, cfg));
+                         : cfg.variant == TT_VARIANT_GROUPS  ? tt_launch_bh_group(p, t->d_grp, cfg)
+                                                             : tt_launch_bh(p, cfg));  // ROPES
 }
 
 tt_status tt_traverse_pc(const tt_tree *t, const float *q, int64_t n, int32_t ld, float radius, uint32_t *count_out,
@@ -389,6 +403,7 @@ tt_status tt_traverse_pc(const tt_tree *t, const float *q, int64_t n, int32_t ld
     p.ld = ld;
     p.r2 = radius * radius;  // rn(r*r), reading R1
     p.count = count_out;
+    if (cfg.variant == TT_VARIANT_GROUPS || cfg.variant == TT_VARIANT_ROPES) return TT_ERR_UNSUPPORTED;  // BH only
     return finish_launch(cfg.variant == TT_VARIANT_RECURSIVE ? tt_launch_pc_recursive(p, t->hdr.dim, cfg)
                          : cfg.variant == TT_VARIANT_STACK   ? tt_launch_pc_stack(p, t->hdr.dim, cfg)
                          : cfg.variant == TT_VARIANT_SPLIT   ? tt_launch_pc_split(p, t->hdr.dim, cfg)
@@ -415,8 +430,9 @@ tt_status tt_traverse_knn(const tt_tree *t, const float *q, int64_t n, int32_t l
     p.k = k;
     p.idx = idx_out;
     p.d2 = d2_out;
-    if (cfg.variant == TT_VARIANT_STACK || cfg.variant == TT_VARIANT_SPLIT)
-        return TT_ERR_UNSUPPORTED;  // guided kernels already keep rope stacks; SPLIT is PC only
+    if (cfg.variant == TT_VARIANT_STACK || cfg.variant == TT_VARIANT_SPLIT || cfg.variant == TT_VARIANT_GROUPS ||
+        cfg.variant == TT_VARIANT_ROPES)
+        return TT_ERR_UNSUPPORTED;  // guided kernels already keep rope stacks; SPLIT is PC, GROUPS / ROPES BH only
     return finish_launch(cfg.variant == TT_VARIANT_RECURSIVE ? tt_launch_knn_recursive(p, t->hdr.dim, cfg)
                                                             : tt_launch_knn(p, t->hdr.dim, cfg));
 }
@@ -438,8 +454,9 @@ tt_status tt_traverse_vp(const tt_tree *t, const float *q, int64_t n, int32_t ld
     p.ld = ld;
     p.idx = idx_out;
     p.d2 = d2_out;
-    if (cfg.variant == TT_VARIANT_STACK || cfg.variant == TT_VARIANT_SPLIT)
-        return TT_ERR_UNSUPPORTED;  // guided kernels already keep rope stacks; SPLIT is PC only
+    if (cfg.variant == TT_VARIANT_STACK || cfg.variant == TT_VARIANT_SPLIT || cfg.variant == TT_VARIANT_GROUPS ||
+        cfg.variant == TT_VARIANT_ROPES)
+        return TT_ERR_UNSUPPORTED;  // guided kernels already keep rope stacks; SPLIT is PC, GROUPS / ROPES BH only
     return finish_launch(cfg.variant == TT_VARIANT_RECURSIVE ? tt_launch_vp_recursive(p, t->hdr.dim, cfg)
                                                             : tt_launch_vp(p, t->hdr.dim, cfg));
 }

@@ -5,6 +5,7 @@
 
 #include <cstddef>
 #include <cstdint>
+#include <mutex>
 
 #include <vector_types.h>
 
@@ -143,6 +144,8 @@ struct tt_tree {
     tt_dev_tree dev;
     uint32_t *d_counters;  // [TT_COUNTER_SLOTS][2]
     unsigned slot_next;
+    void *d_grp = nullptr;  // OCT: child-group records (kern_bh_group.cu), built on first use
+    std::mutex grp_mu;
 };
 
 // Launchers (kernels/*.cu).  Return a cudaError_t as int.
@@ -164,6 +167,9 @@ int tt_launch_knn_recursive(const tt_knn_params &p, int dim, const tt_launch_cfg
 int tt_launch_vp_recursive(const tt_vp_params &p, int dim, const tt_launch_cfg &cfg);
 // explicit rope-stack variant, unguided kernels (kern_stack.cu)
 int tt_launch_bh_stack(const tt_bh_params &p, const tt_launch_cfg &cfg);
+// lockstep walk by child groups (kern_bh_group.cu)
+int tt_bh_groups_build(const void *rec, long long nn, void *stream, void **grp_out);
+int tt_launch_bh_group(const tt_bh_params &p, const void *grp, const tt_launch_cfg &cfg);
 int tt_launch_pc_stack(const tt_pc_params &p, int dim, const tt_launch_cfg &cfg);
 // one point's traversal split over a 16-lane group (kern_pc_split.cu)
 int tt_launch_pc_split(const tt_pc_params &p, int dim, const tt_launch_cfg &cfg);

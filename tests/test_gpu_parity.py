@@ -749,3 +749,43 @@ def test_pc_split_small_trees_and_buckets():
     b = ttgen.plummer(100, seed=7)
     with pytest.raises(P.TTError):
         P.tt_traverse_bh(P.tt_tree_upload(P.build_oct(b)), dev(b), 0.5, 0.05, variant="split")
+
+
+# ------------------------------------------- BH lockstep walk by child groups
+@pytest.mark.parametrize("mode", MODES)
+@pytest.mark.parametrize("sorted_", [False, True])
+def test_bh_groups_variant(bh_small, mode, sorted_):
+    """TT_VARIANT_GROUPS: a lockstep warp expands whole cells; every body tests
+    exactly its recursive walk's nodes (visit counts equal the oracle's), the
+    warp fetches equal the Fig.8 union, accelerations within 1e-4."""
+    b, ot, ref, tree = bh_small
+    bd = dev(b)
+    order = P.tt_sort_points(tree, bd) if sorted_ else None
+    st = P.Stats.alloc(len(b), "cuda")
+    acc = P.tt_traverse_bh(tree, bd, 0.5, 0.05, order=order, mode=mode, stats=st, variant="groups").cpu().numpy()
+    err = rel_err(acc, ref.out[0])
+    assert err.max() <= BH_TOL, err.max()
+    assert np.array_equal(st.visits.cpu().numpy(), ref.visits)
+    if mode == "lockstep":
+        o = order.cpu().numpy() if sorted_ else np.arange(len(b))
+        union = oracle.unguided_warp_union(ot, b[o], 0.5, W=32 * P._lib.BH_POINTS_PER_LANE)
+        assert np.array_equal(st.warp_fetches.cpu().numpy()[:len(union)], union)
+
+
+def test_bh_groups_theta0_buckets_and_1m():
+    from tests import brute
+    b = ttgen.plummer(3001, seed=204)
+    b[100, :3] = b[101, :3] = b[102, :3]  # a depth-32 bucket
+    tree = P.tt_tree_upload(P.build_oct(b))
+    acc = P.tt_traverse_bh(tree, dev(b), 0.0, 0.05, mode="lockstep", variant="groups").cpu().numpy()
+    assert rel_err(acc, brute.direct_sum(b, 0.05)).max() <= BH_TOL
+    c = ttgen.CONFIGS["bh_1m_plummer"]
+    b = ttgen.plummer(c["n"], c["seed"])
+    tree = P.tt_build_oct_device(dev(b))
+    bd = dev(b)
+    perm = P.tt_sort_points(tree, bd)
+    acc = P.tt_traverse_bh(tree, bd, c["theta"], c["eps"], order=perm, variant="groups").cpu().numpy()
+    sample = np.concatenate([np.random.default_rng(5).choice(len(b), 3000, replace=False),
+                             np.argsort(np.linalg.norm(b[:, :3], axis=1))[:500]])
+    ref = oracle.bh(oracle.build_oct(b), b[sample], c["theta"], c["eps"], self_ids=sample)
+    assert rel_err(acc[sample], ref.out[0]).max() <= BH_TOL
