@@ -325,6 +325,7 @@ int launch(const tt_bh_params &p, const tt_oct_rec *grp, const tt_launch_cfg &cf
 // Child-group array of an oct tree (built once per tree, kept with it).
 int tt_bh_groups_build(const void *rec, long long nn, void *stream, void **grp_out) {
     cudaStream_t s = (cudaStream_t)stream;
+    tt_keep_pool_memory();
     const tt_oct_rec *r = static_cast<const tt_oct_rec *>(rec);
     int *nk = nullptr, *goff = nullptr;
     void *tmp = nullptr, *grp = nullptr;
@@ -333,7 +334,8 @@ int tt_bh_groups_build(const void *rec, long long nn, void *stream, void **grp_o
     if (!e) e = cudaMallocAsync((void **)&goff, sizeof(int) * nn, s);
     if (!e) e = cub::DeviceScan::ExclusiveSum(nullptr, tb, nk, goff, (int)nn, s);
     if (!e) e = cudaMallocAsync(&tmp, tb, s);
-    if (!e) e = cudaMalloc(&grp, sizeof(tt_oct_rec) * (size_t)nn);
+    // stream-ordered from the kept pool: time stepping builds one per step
+    if (!e) e = cudaMallocAsync(&grp, sizeof(tt_oct_rec) * (size_t)nn, s);
     const unsigned G = (unsigned)std::min<long long>((nn + 255) / 256, 148 * 8);
     if (!e) {
         nkids_kernel<<<G, 256, 0, s>>>(r, nn, nk);
@@ -346,9 +348,8 @@ int tt_bh_groups_build(const void *rec, long long nn, void *stream, void **grp_o
     if (tmp) cudaFreeAsync(tmp, s);
     if (goff) cudaFreeAsync(goff, s);
     if (nk) cudaFreeAsync(nk, s);
-    if (!e) e = cudaStreamSynchronize(s);
     if (e) {
-        if (grp) cudaFree(grp);
+        if (grp) cudaFreeAsync(grp, s);
         return (int)e;
     }
     *grp_out = grp;

@@ -296,7 +296,7 @@ tt_status tt_tree_free(tt_tree *t) {
     if (!t) return TT_OK;
     cudaError_t e1 = cudaFree(t->d_blob);
     cudaError_t e2 = cudaFree(t->d_counters);
-    if (t->d_grp) cudaFree(t->d_grp);
+    if (t->d_grp) cudaFreeAsync(t->d_grp, 0);  // stream-ordered pool memory (kern_bh_group.cu)
     delete t;
     if (e1 != cudaSuccess) return cuda_fail(e1);
     if (e2 != cudaSuccess) return cuda_fail(e2);
