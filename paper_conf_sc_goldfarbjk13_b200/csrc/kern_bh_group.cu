@@ -24,6 +24,10 @@
 
 #include <cub/device/device_scan.cuh>
 
+#include <mutex>
+#include <unordered_map>
+#include <vector>
+
 #include "kern_common.cuh"
 
 namespace {
@@ -320,12 +324,50 @@ int launch(const tt_bh_params &p, const tt_oct_rec *grp, const tt_launch_cfg &cf
     return (int)cudaGetLastError();
 }
 
+// Group arrays are recycled between trees: BH time stepping builds a tree,
+// and so a group array, every step, and a fresh cudaMalloc per step costs
+// milliseconds (pool allocations were fragmented by the sort's scratch).
+// tt_tree_free returns the array here after its cudaFree of the blob has
+// synchronised the device, so a recycled array is never still in use.
+std::mutex g_grp_mu;
+std::unordered_map<void *, size_t> g_grp_size;  // every group array ever allocated
+std::vector<void *> g_grp_free;
+
+void *grp_take(size_t bytes) {
+    {
+        std::lock_guard<std::mutex> lk(g_grp_mu);
+        for (size_t i = 0; i < g_grp_free.size(); ++i) {
+            void *p = g_grp_free[i];
+            const size_t sz = g_grp_size[p];
+            if (sz >= bytes && sz <= 2 * bytes) {
+                g_grp_free.erase(g_grp_free.begin() + (long)i);
+                return p;
+            }
+        }
+    }
+    void *p = nullptr;
+    if (cudaMalloc(&p, bytes) != cudaSuccess) return nullptr;
+    std::lock_guard<std::mutex> lk(g_grp_mu);
+    g_grp_size[p] = bytes;
+    return p;
+}
+
 }  // namespace
+
+void tt_bh_groups_release(void *grp) {
+    if (!grp) return;
+    std::lock_guard<std::mutex> lk(g_grp_mu);
+    if (g_grp_free.size() >= 4) {  // keep a few
+        cudaFree(grp);
+        g_grp_size.erase(grp);
+        return;
+    }
+    g_grp_free.push_back(grp);
+}
 
 // Child-group array of an oct tree (built once per tree, kept with it).
 int tt_bh_groups_build(const void *rec, long long nn, void *stream, void **grp_out) {
     cudaStream_t s = (cudaStream_t)stream;
-    tt_keep_pool_memory();
     const tt_oct_rec *r = static_cast<const tt_oct_rec *>(rec);
     int *nk = nullptr, *goff = nullptr;
     void *tmp = nullptr, *grp = nullptr;
@@ -334,8 +376,10 @@ int tt_bh_groups_build(const void *rec, long long nn, void *stream, void **grp_o
     if (!e) e = cudaMallocAsync((void **)&goff, sizeof(int) * nn, s);
     if (!e) e = cub::DeviceScan::ExclusiveSum(nullptr, tb, nk, goff, (int)nn, s);
     if (!e) e = cudaMallocAsync(&tmp, tb, s);
-    // stream-ordered from the kept pool: time stepping builds one per step
-    if (!e) e = cudaMallocAsync(&grp, sizeof(tt_oct_rec) * (size_t)nn, s);
+    if (!e) {
+        grp = grp_take(sizeof(tt_oct_rec) * (size_t)nn);
+        if (!grp) e = cudaErrorMemoryAllocation;
+    }
     const unsigned G = (unsigned)std::min<long long>((nn + 255) / 256, 148 * 8);
     if (!e) {
         nkids_kernel<<<G, 256, 0, s>>>(r, nn, nk);
@@ -349,7 +393,7 @@ int tt_bh_groups_build(const void *rec, long long nn, void *stream, void **grp_o
     if (goff) cudaFreeAsync(goff, s);
     if (nk) cudaFreeAsync(nk, s);
     if (e) {
-        if (grp) cudaFreeAsync(grp, s);
+        if (grp) tt_bh_groups_release(grp);
         return (int)e;
     }
     *grp_out = grp;

@@ -12,6 +12,9 @@
 
 #include "tt_internal.h"
 
+// kern_bh_group.cu: return a tree's child-group array for reuse
+void tt_bh_groups_release(void *grp);
+
 // build_nn_gpu.cu (declared here rather than in tt_internal.h)
 int tt_build_nn_gpu_impl(const float *pts, long long n, int dim, int ld, void *stream, tt_blob_header *hdr,
                          void **blob);
@@ -296,7 +299,7 @@ tt_status tt_tree_free(tt_tree *t) {
     if (!t) return TT_OK;
     cudaError_t e1 = cudaFree(t->d_blob);
     cudaError_t e2 = cudaFree(t->d_counters);
-    if (t->d_grp) cudaFreeAsync(t->d_grp, 0);  // stream-ordered pool memory (kern_bh_group.cu)
+    tt_bh_groups_release(t->d_grp);  // recycled (kern_bh_group.cu); cudaFree above synchronised
     delete t;
     if (e1 != cudaSuccess) return cuda_fail(e1);
     if (e2 != cudaSuccess) return cuda_fail(e2);
