@@ -789,3 +789,19 @@ def test_bh_groups_theta0_buckets_and_1m():
                              np.argsort(np.linalg.norm(b[:, :3], axis=1))[:500]])
     ref = oracle.bh(oracle.build_oct(b), b[sample], c["theta"], c["eps"], self_ids=sample)
     assert rel_err(acc[sample], ref.out[0]).max() <= BH_TOL
+
+
+def test_bh_group_arrays_recycled_across_trees():
+    """Child-group arrays are returned to a small cache when a tree is freed
+    and reused by later trees (time stepping builds one per step): trees of
+    changing sizes, each checked against the oracle."""
+    import gc
+    for n, seed in ((20011, 1), (3, 2), (20011, 3), (50000, 4), (777, 5), (20011, 6)):
+        b = ttgen.plummer(n, seed=300 + seed)
+        tree = P.tt_build_oct_device(dev(b))
+        acc = P.tt_traverse_bh(tree, dev(b), 0.5, 0.05, mode="lockstep").cpu().numpy()
+        ref = oracle.bh(oracle.build_oct(b), b, 0.5, 0.05, self_ids=np.arange(n))
+        assert rel_err(acc, ref.out[0]).max() <= BH_TOL, n
+        tree.free()
+        del tree
+        gc.collect()
