@@ -17,7 +17,7 @@
 //
 // Group record (32 B, like tt_oct_rec): {com.xyz, mass} +
 // {group offset of the node's children | -1, number of children, body | -1,
-// level}; entry 0 is the root, the children of a cell are contiguous.
+// level << 24}; entry 0 is the root, the children of a cell are contiguous.
 #include <climits>
 #include <cfloat>
 #include <cmath>
@@ -29,6 +29,7 @@
 #include <vector>
 
 #include "kern_common.cuh"
+
 
 namespace {
 
@@ -65,6 +66,7 @@ __global__ void groups_fill_kernel(const tt_oct_rec *rec, long long nn, const in
             tt_oct_rec r = rec[0];
             r.first_child = nk[0] > 0 ? 1 + goff[0] : -1;
             r.skip = nk[0];
+            r.level <<= 24;
             grp[0] = r;
         }
         int c = rec[v].first_child, k = 0;
@@ -73,6 +75,7 @@ __global__ void groups_fill_kernel(const tt_oct_rec *rec, long long nn, const in
             tt_oct_rec r = rec[c];
             r.first_child = nk[c] > 0 ? 1 + goff[c] : -1;
             r.skip = nk[c];
+            r.level <<= 24;  // the exponent step of dsq_L (level * 2^24): one IADD per child
             grp[1 + goff[v] + k] = r;
             ++k;
             c = rec[c].skip;
@@ -196,7 +199,7 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                         visits[0] += in0;
                         visits[1] += in1;
                     }
-                    const float dl = EXP_DSQ ? dsq_at(dsq_bits, t.w) : s_dsq[t.w];
+                    const float dl = EXP_DSQ ? __int_as_float(dsq_bits - t.w) : s_dsq[t.w >> 24];
                     const float2 dx = add2_rn(make_float2(g.x, g.x), nbx);
                     const float2 dy = add2_rn(make_float2(g.y, g.y), nby);
                     const float2 dz = add2_rn(make_float2(g.z, g.z), nbz);
