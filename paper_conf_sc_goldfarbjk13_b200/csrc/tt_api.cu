@@ -362,7 +362,11 @@ tt_status tt_traverse_bh(const tt_tree *t, const float *bodies, const int32_t *s
     if (cfg.variant == TT_VARIANT_SPLIT) return TT_ERR_UNSUPPORTED;  // PC only
     // BH default: lockstep warps walk by child groups (kern_bh_group.cu);
     // TT_VARIANT_ROPES keeps the per-node lockstep walk over ropes (kern_bh.cu)
-    if (cfg.variant == TT_VARIANT_AUTOROPES) cfg.variant = TT_VARIANT_GROUPS;
+    // (the child-group stack holds 8 entries per level: deeper custom trees
+    // take the stackless per-node walk, or fail if groups were requested)
+    const bool groups_fit = 8 * (t->hdr.height + 2) <= 320;  // kStackPerWarp of kern_bh_group.cu
+    if (cfg.variant == TT_VARIANT_AUTOROPES) cfg.variant = groups_fit ? TT_VARIANT_GROUPS : TT_VARIANT_ROPES;
+    if (cfg.variant == TT_VARIANT_GROUPS && !groups_fit) return TT_ERR_TREE_TOO_DEEP;
     if (cfg.variant == TT_VARIANT_GROUPS) {
         tt_tree *mt = const_cast<tt_tree *>(t);
         std::lock_guard<std::mutex> lk(mt->grp_mu);
