@@ -805,3 +805,22 @@ def test_bh_group_arrays_recycled_across_trees():
         tree.free()
         del tree
         gc.collect()
+
+
+def test_bh_default_falls_back_for_trees_deeper_than_group_stack(bh_small):
+    """A custom tree whose declared height exceeds the child-group stack
+    (8 entries per level) but not TT_MAX_HEIGHT: the default BH path takes the
+    per-node rope walk (same visits, within 1e-4); an explicit request for
+    the child-group walk fails with TT_ERR_TREE_TOO_DEEP."""
+    b, ot, ref, _ = bh_small
+    h = P.build_oct(b)
+    h.desc.height = P._lib.MAX_HEIGHT  # legal for the pack, too deep for the group stack
+    tree = P.tt_tree_upload(h)
+    bd = dev(b)
+    st = P.Stats.alloc(len(b), "cuda")
+    acc = P.tt_traverse_bh(tree, bd, 0.5, 0.05, mode="lockstep", stats=st).cpu().numpy()
+    assert rel_err(acc, ref.out[0]).max() <= BH_TOL
+    assert np.array_equal(st.visits.cpu().numpy(), ref.visits)
+    with pytest.raises(P.TTError) as e:
+        P.tt_traverse_bh(tree, bd, 0.5, 0.05, variant="groups")
+    assert e.value.status == -4
