@@ -110,11 +110,13 @@ inline void header_base(tt_blob_header &h, int kind, int dim, int leaf, long lon
 
 // cudaMalloc the blob, zero it, write the header
 inline cudaError_t alloc_blob(const tt_blob_header &h, cudaStream_t s, void **blob) {
-    cudaError_t e = cudaMalloc(blob, h.total);
+    // recycled from freed device-built trees when one fits (tt_api.cu):
+    // time stepping builds a tree every step
+    cudaError_t e = (cudaError_t)tt_blob_take((size_t)h.total, blob);
     if (e) return e;
     if ((e = cudaMemsetAsync(*blob, 0, h.total, s)) ||
         (e = cudaMemcpyAsync(*blob, &h, sizeof(h), cudaMemcpyHostToDevice, s))) {
-        cudaFree(*blob);
+        tt_blob_release(*blob);
         *blob = nullptr;
     }
     return e;

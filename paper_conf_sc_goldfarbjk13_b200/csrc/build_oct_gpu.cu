@@ -319,7 +319,7 @@ int tt_build_oct_gpu_impl(const float *bodies_f, long long n, void *stream, tt_b
     records_kernel<<<GN, 256, 0, s>>>(n_nodes, A, newidx, rec);
     leaf_fix_kernel<<<GN, 256, 0, s>>>(bodies, n_nodes, A, newidx, rec);
     if ((e = cudaGetLastError()) || (e = cudaStreamSynchronize(s))) {
-        cudaFree(blob);
+        tt_blob_release(blob);
         return e;
     }
     *hdr_out = h;

@@ -25,6 +25,7 @@
 #include <cub/device/device_scan.cuh>
 
 #include <mutex>
+#include <type_traits>
 #include <unordered_map>
 #include <vector>
 
@@ -60,7 +61,7 @@ __global__ void nkids_kernel(const tt_oct_rec *rec, long long nn, int *nk) {
 }
 
 __global__ void groups_fill_kernel(const tt_oct_rec *rec, long long nn, const int *nk, const int *goff,
-                                   tt_oct_rec *grp) {
+                                   tt_oct_rec *grp, int *leaf_of, long long np) {
     for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < nn; v += (long long)gridDim.x * blockDim.x) {
         if (v == 0) {  // the root's own entry
             tt_oct_rec r = rec[0];
@@ -68,6 +69,7 @@ __global__ void groups_fill_kernel(const tt_oct_rec *rec, long long nn, const in
             r.skip = nk[0];
             r.level <<= 24;
             grp[0] = r;
+            if (r.first_child < 0 && r.body >= 0 && r.body < np) leaf_of[r.body] = 0;
         }
         int c = rec[v].first_child, k = 0;
         const int end = rec[v].skip;
@@ -77,6 +79,7 @@ __global__ void groups_fill_kernel(const tt_oct_rec *rec, long long nn, const in
             r.skip = nk[c];
             r.level <<= 24;  // the exponent step of dsq_L (level * 2^24): one IADD per child
             grp[1 + goff[v] + k] = r;
+            if (r.first_child < 0 && r.body >= 0 && r.body < np) leaf_of[r.body] = 1 + goff[v] + k;
             ++k;
             c = rec[c].skip;
         }
@@ -89,7 +92,8 @@ __device__ __forceinline__ float dsq_at(int dsq_bits, int lvl) { return __int_as
 #define TT_BHG_MINB 4
 #endif
 template <bool STATS, bool EXP_DSQ>
-__global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_bh_params P, const tt_oct_rec *grp) {
+__global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_bh_params P, const tt_oct_rec *grp,
+                                                                                 const int *leaf_of, long long np) {
     extern __shared__ __align__(128) unsigned char smem[];
     float *s_dsq = reinterpret_cast<float *>(smem + 16);
     GroupEntry *s_stack = reinterpret_cast<GroupEntry *>(smem + kSmemHdr);
@@ -165,6 +169,29 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
             visits[j] = 0;
         }
         unsigned fetches = 0, steps = 0;
+        // The self test (skip the leaf holding the body itself) only
+        // matters where that leaf's term is not exactly zero: a leaf at
+        // the body's own position contributes f * 0 = 0 whenever f is
+        // finite (eps > 0).  A warp whose bodies all sit exactly on their
+        // own leaves (the normal case: the tree was built from them)
+        // walks without the per-child test; others keep it.
+        bool ok[kBPL];
+#pragma unroll
+        for (int j = 0; j < kBPL; ++j) {
+            ok[j] = !valid[j] || self[j] < 0 || (long long)self[j] >= np;
+            if (!ok[j]) {
+                const int lf = __ldg(leaf_of + self[j]);
+                if (lf < 0) {
+                    ok[j] = true;  // no leaf is tested against this id
+                } else {
+                    const float4 c = __ldg(reinterpret_cast<const float4 *>(grp + lf));
+                    const float inv = rsqrt_ftz(__fadd_rn(0.f, P.eps2));
+                    const float f = __fmul_rn(__fmul_rn(c.w, __fmul_rn(inv, inv)), inv);
+                    ok[j] = c.x == b[j].x && c.y == b[j].y && c.z == b[j].z && isfinite(f);
+                }
+            }
+        }
+        const bool need_self = __any_sync(TT_FULL, !(ok[0] && ok[1]));
         if (lock) {
             static_assert(kBPL == 2, "group walk is written for body pairs");
             const float2 nbx = add2_rn(make_float2(nz, nz), make_float2(-b[0].x, -b[1].x));
@@ -176,75 +203,84 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
             // the root group: entry 0 alone, tested by every valid body
             int goff = 0, gnk = 1;
             unsigned m0 = __ballot_sync(TT_FULL, valid[0]), m1 = __ballot_sync(TT_FULL, valid[1]);
-            for (;;) {
-                const bool in0 = (m0 >> lane) & 1u, in1 = (m1 >> lane) & 1u;
-                // stage the group: lane k loads child k (one request for the
-                // whole group, one round trip), the warp reads them back from
-                // shared memory with broadcast loads
-                if (lane < gnk) {
-                    float4 sg;
-                    int4 st4;
-                    ldg_rec256(grp + goff + lane, sg, st4);
-                    gbuf[lane] = sg;
-                    tbuf[lane] = st4;
-                }
-                __syncwarp();
+            auto walk = [&](auto self_chk) {
+                constexpr bool SELF = decltype(self_chk)::value;
+                for (;;) {
+                    const bool in0 = (m0 >> lane) & 1u, in1 = (m1 >> lane) & 1u;
+                    // stage the group: lane k loads child k (one request for the
+                    // whole group, one round trip), the warp reads them back from
+                    // shared memory with broadcast loads
+                    if (lane < gnk) {
+                        float4 sg;
+                        int4 st4;
+                        ldg_rec256(grp + goff + lane, sg, st4);
+                        gbuf[lane] = sg;
+                        tbuf[lane] = st4;
+                    }
+                    __syncwarp();
 #pragma unroll 1
-                for (int k = 0; k < gnk; ++k) {
-                    const float4 g = gbuf[k];
-                    const int4 t = tbuf[k];
-                    if (STATS) {
-                        ++fetches;
-                        ++steps;
-                        visits[0] += in0;
-                        visits[1] += in1;
+                    for (int k = 0; k < gnk; ++k) {
+                        const float4 g = gbuf[k];
+                        const int4 t = tbuf[k];
+                        if (STATS) {
+                            ++fetches;
+                            ++steps;
+                            visits[0] += in0;
+                            visits[1] += in1;
+                        }
+                        const float dl = EXP_DSQ ? __int_as_float(dsq_bits - t.w) : s_dsq[t.w >> 24];
+                        const float2 dx = add2_rn(make_float2(g.x, g.x), nbx);
+                        const float2 dy = add2_rn(make_float2(g.y, g.y), nby);
+                        const float2 dz = add2_rn(make_float2(g.z, g.z), nbz);
+                        const float2 drsq = add2_rn(add2_rn(sqr2_rn(dx, nz), sqr2_rn(dy, nz)), sqr2_rn(dz, nz));
+                        const bool cell = t.x >= 0;
+                        const bool o0 = in0 && cell && drsq.x < dl;
+                        const bool o1 = in1 && cell && drsq.y < dl;
+                        const bool k0 = in0 && !o0 && (!SELF || t.z != self[0]);
+                        const bool k1 = in1 && !o1 && (!SELF || t.z != self[1]);
+                        const float2 mw = make_float2(k0 ? g.w : 0.f, k1 ? g.w : 0.f);
+                        const float2 r = add2_rn(drsq, e22);
+                        const float2 inv = make_float2(rsqrt_ftz(r.x), rsqrt_ftz(r.y));
+                        float2 f = mul2_rn(mul2_rn(mw, mul2_rn(inv, inv)), inv);
+                        // the checked walk also serves eps = 0, where a skipped
+                        // leaf at distance 0 has inv = inf (0 * inf): select
+                        if (SELF) f = make_float2(k0 ? f.x : 0.f, k1 ? f.y : 0.f);
+                        ax = fma2_rn(f, dx, ax);
+                        ay = fma2_rn(f, dy, ay);
+                        az = fma2_rn(f, dz, az);
+                        // one vote per child; the two ballots only when some body
+                        // opens it (one vote: -1.5% vs two ballots per child)
+                        if (__any_sync(TT_FULL, o0 || o1)) {
+                            const unsigned om0 = __ballot_sync(TT_FULL, o0), om1 = __ballot_sync(TT_FULL, o1);
+                            if (lane == 0) stk[sp] = GroupEntry{t.x, t.y, om0, om1};
+                            ++sp;
+                        }
                     }
-                    const float dl = EXP_DSQ ? __int_as_float(dsq_bits - t.w) : s_dsq[t.w >> 24];
-                    const float2 dx = add2_rn(make_float2(g.x, g.x), nbx);
-                    const float2 dy = add2_rn(make_float2(g.y, g.y), nby);
-                    const float2 dz = add2_rn(make_float2(g.z, g.z), nbz);
-                    const float2 drsq = add2_rn(add2_rn(sqr2_rn(dx, nz), sqr2_rn(dy, nz)), sqr2_rn(dz, nz));
-                    const bool cell = t.x >= 0;
-                    const bool o0 = in0 && cell && drsq.x < dl;
-                    const bool o1 = in1 && cell && drsq.y < dl;
-                    const float2 mw = make_float2(in0 && !o0 && t.z != self[0] ? g.w : 0.f,
-                                                  in1 && !o1 && t.z != self[1] ? g.w : 0.f);
-                    const float2 r = add2_rn(drsq, e22);
-                    const float2 inv = make_float2(rsqrt_ftz(r.x), rsqrt_ftz(r.y));
-                    const float2 f = mul2_rn(mul2_rn(mw, mul2_rn(inv, inv)), inv);
-                    ax = fma2_rn(f, dx, ax);
-                    ay = fma2_rn(f, dy, ay);
-                    az = fma2_rn(f, dz, az);
-                    // one vote per child; the two ballots only when some body
-                    // opens it (one vote: -1.5% vs two ballots per child)
-                    if (__any_sync(TT_FULL, o0 || o1)) {
-                        const unsigned om0 = __ballot_sync(TT_FULL, o0), om1 = __ballot_sync(TT_FULL, o1);
-                        if (lane == 0) stk[sp] = GroupEntry{t.x, t.y, om0, om1};
-                        ++sp;
+                    __syncwarp();  // the group buffer is reused by the next pop
+                    since_flush += gnk;
+                    if (since_flush >= kFlushEvery) {  // warp-uniform cadence
+                        X[0] += (double)ax.x;
+                        Y[0] += (double)ay.x;
+                        Z[0] += (double)az.x;
+                        X[1] += (double)ax.y;
+                        Y[1] += (double)ay.y;
+                        Z[1] += (double)az.y;
+                        ax = ay = az = make_float2(0.f, 0.f);
+                        since_flush = 0;
                     }
+                    if (sp == 0) break;
+                    --sp;
+                    __syncwarp();
+                    int4 e = make_int4(0, 0, 0, 0);
+                    if (lane == 0) e = *reinterpret_cast<const int4 *>(stk + sp);
+                    goff = __shfl_sync(TT_FULL, e.x, 0);
+                    gnk = __shfl_sync(TT_FULL, e.y, 0);
+                    m0 = (unsigned)__shfl_sync(TT_FULL, e.z, 0);
+                    m1 = (unsigned)__shfl_sync(TT_FULL, e.w, 0);
                 }
-                __syncwarp();  // the group buffer is reused by the next pop
-                since_flush += gnk;
-                if (since_flush >= kFlushEvery) {  // warp-uniform cadence
-                    X[0] += (double)ax.x;
-                    Y[0] += (double)ay.x;
-                    Z[0] += (double)az.x;
-                    X[1] += (double)ax.y;
-                    Y[1] += (double)ay.y;
-                    Z[1] += (double)az.y;
-                    ax = ay = az = make_float2(0.f, 0.f);
-                    since_flush = 0;
-                }
-                if (sp == 0) break;
-                --sp;
-                __syncwarp();
-                int4 e = make_int4(0, 0, 0, 0);
-                if (lane == 0) e = *reinterpret_cast<const int4 *>(stk + sp);
-                goff = __shfl_sync(TT_FULL, e.x, 0);
-                gnk = __shfl_sync(TT_FULL, e.y, 0);
-                m0 = (unsigned)__shfl_sync(TT_FULL, e.z, 0);
-                m1 = (unsigned)__shfl_sync(TT_FULL, e.w, 0);
-            }
+            };
+            if (need_self) walk(std::true_type{});
+            else walk(std::false_type{});
             X[0] += (double)ax.x;
             Y[0] += (double)ay.x;
             Z[0] += (double)az.x;
@@ -306,7 +342,7 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
 }
 
 template <bool STATS, bool EXP_DSQ>
-int launch(const tt_bh_params &p, const tt_oct_rec *grp, const tt_launch_cfg &cfg) {
+int launch(const tt_bh_params &p, const tt_oct_rec *grp, const int *leaf_of, long long np, const tt_launch_cfg &cfg) {
     const size_t smem = kSmemHdr + (size_t)(kBlock / 32) * kStackPerWarp * sizeof(GroupEntry) + (kBlock / 32) * 16 * 16;
     auto kern = bh_group_kernel<STATS, EXP_DSQ>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -323,7 +359,7 @@ int launch(const tt_bh_params &p, const tt_oct_rec *grp, const tt_launch_cfg &cf
     const long long need = (ntiles + kBlock / 32 - 1) / (kBlock / 32);
     if (grid > need) grid = need;
     if (grid < 1) grid = 1;
-    kern<<<(unsigned)grid, kBlock, smem, (cudaStream_t)cfg.stream>>>(p, grp);
+    kern<<<(unsigned)grid, kBlock, smem, (cudaStream_t)cfg.stream>>>(p, grp, leaf_of, np);
     return (int)cudaGetLastError();
 }
 
@@ -369,7 +405,7 @@ void tt_bh_groups_release(void *grp) {
 }
 
 // Child-group array of an oct tree (built once per tree, kept with it).
-int tt_bh_groups_build(const void *rec, long long nn, void *stream, void **grp_out) {
+int tt_bh_groups_build(const void *rec, long long nn, long long np, void *stream, void **grp_out) {
     cudaStream_t s = (cudaStream_t)stream;
     const tt_oct_rec *r = static_cast<const tt_oct_rec *>(rec);
     int *nk = nullptr, *goff = nullptr;
@@ -380,16 +416,20 @@ int tt_bh_groups_build(const void *rec, long long nn, void *stream, void **grp_o
     if (!e) e = cub::DeviceScan::ExclusiveSum(nullptr, tb, nk, goff, (int)nn, s);
     if (!e) e = cudaMallocAsync(&tmp, tb, s);
     if (!e) {
-        grp = grp_take(sizeof(tt_oct_rec) * (size_t)nn);
+        // records, then leaf_of[np]: the group index of the leaf whose body
+        // is each id (-1 for ids no leaf names first)
+        grp = grp_take(sizeof(tt_oct_rec) * (size_t)nn + sizeof(int) * (size_t)np);
         if (!grp) e = cudaErrorMemoryAllocation;
     }
+    int *leaf_of = grp ? reinterpret_cast<int *>(static_cast<tt_oct_rec *>(grp) + nn) : nullptr;
+    if (!e && np > 0) e = cudaMemsetAsync(leaf_of, 0xff, sizeof(int) * (size_t)np, s);
     const unsigned G = (unsigned)std::min<long long>((nn + 255) / 256, 148 * 8);
     if (!e) {
         nkids_kernel<<<G, 256, 0, s>>>(r, nn, nk);
         e = cub::DeviceScan::ExclusiveSum(tmp, tb, nk, goff, (int)nn, s);
     }
     if (!e) {
-        groups_fill_kernel<<<G, 256, 0, s>>>(r, nn, nk, goff, static_cast<tt_oct_rec *>(grp));
+        groups_fill_kernel<<<G, 256, 0, s>>>(r, nn, nk, goff, static_cast<tt_oct_rec *>(grp), leaf_of, np);
         e = cudaGetLastError();
     }
     if (tmp) cudaFreeAsync(tmp, s);
@@ -403,11 +443,12 @@ int tt_bh_groups_build(const void *rec, long long nn, void *stream, void **grp_o
     return 0;
 }
 
-int tt_launch_bh_group(const tt_bh_params &p, const void *grp, const tt_launch_cfg &cfg) {
+int tt_launch_bh_group(const tt_bh_params &p, const void *grp, long long nn, long long np, const tt_launch_cfg &cfg) {
     const bool stats = p.c.st_visits || p.c.st_warp_fetches || p.c.st_warp_steps || p.c.st_warp_mode;
     const float r = p.dsq_root;
     const bool exp_ok = r < INFINITY && r > 0.f && std::ldexp((double)r, -2 * p.c.height) >= (double)FLT_MIN;
     const tt_oct_rec *g = static_cast<const tt_oct_rec *>(grp);
-    if (stats) return exp_ok ? launch<true, true>(p, g, cfg) : launch<true, false>(p, g, cfg);
-    return exp_ok ? launch<false, true>(p, g, cfg) : launch<false, false>(p, g, cfg);
+    const int *lf = reinterpret_cast<const int *>(g + nn);
+    if (stats) return exp_ok ? launch<true, true>(p, g, lf, np, cfg) : launch<true, false>(p, g, lf, np, cfg);
+    return exp_ok ? launch<false, true>(p, g, lf, np, cfg) : launch<false, false>(p, g, lf, np, cfg);
 }

@@ -8,7 +8,10 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include <new>
+#include <unordered_map>
+#include <vector>
 
 #include "tt_internal.h"
 
@@ -137,6 +140,57 @@ tt_status finish_launch(int err) {
 }
 
 }  // namespace
+
+// Blob cache of the GPU builders.  A fresh cudaMalloc / cudaFree of a
+// tens-of-MB blob per time step cost 1-10 ms each (and varied run to run);
+// freed blobs are kept (at most kBlobCacheKeep) and reused by a later build
+// whose blob fits in [bytes, 2 * bytes].
+namespace {
+std::mutex g_blob_mu;
+std::unordered_map<void *, size_t> g_blob_size;  // every cached-kind blob alive or free
+std::vector<void *> g_blob_free;
+constexpr size_t kBlobCacheKeep = 2;
+}  // namespace
+
+int tt_blob_take(size_t bytes, void **out) {
+    {
+        std::lock_guard<std::mutex> lk(g_blob_mu);
+        for (size_t i = 0; i < g_blob_free.size(); ++i) {
+            void *p = g_blob_free[i];
+            const size_t sz = g_blob_size[p];
+            if (sz >= bytes && sz <= 2 * bytes) {
+                g_blob_free.erase(g_blob_free.begin() + (long)i);
+                *out = p;
+                return cudaSuccess;
+            }
+        }
+    }
+    void *p = nullptr;
+    cudaError_t e = cudaMalloc(&p, bytes);
+    if (e) return e;
+    std::lock_guard<std::mutex> lk(g_blob_mu);
+    g_blob_size[p] = bytes;
+    *out = p;
+    return cudaSuccess;
+}
+
+bool tt_blob_is_cached_kind(void *blob) {
+    std::lock_guard<std::mutex> lk(g_blob_mu);
+    return g_blob_size.count(blob) != 0;
+}
+
+void tt_blob_release(void *blob) {
+    if (!blob) return;
+    std::lock_guard<std::mutex> lk(g_blob_mu);
+    if (g_blob_free.size() >= kBlobCacheKeep) {
+        // evict the oldest free blob, keep the newest
+        void *old = g_blob_free.front();
+        g_blob_free.erase(g_blob_free.begin());
+        g_blob_size.erase(old);
+        cudaFree(old);
+    }
+    g_blob_free.push_back(blob);
+}
 
 extern "C" {
 
@@ -297,9 +351,15 @@ tt_status tt_tree_upload(const tt_tree_desc *d, tt_stream s, tt_tree **out) {
 
 tt_status tt_tree_free(tt_tree *t) {
     if (!t) return TT_OK;
-    cudaError_t e1 = cudaFree(t->d_blob);
+    cudaError_t e1;
+    if (tt_blob_is_cached_kind(t->d_blob)) {  // GPU-built: recycled once the device is idle
+        e1 = cudaDeviceSynchronize();
+        if (e1 == cudaSuccess) tt_blob_release(t->d_blob);
+    } else {
+        e1 = cudaFree(t->d_blob);
+    }
     cudaError_t e2 = cudaFree(t->d_counters);
-    tt_bh_groups_release(t->d_grp);  // recycled (kern_bh_group.cu); cudaFree above synchronised
+    tt_bh_groups_release(t->d_grp);  // recycled (kern_bh_group.cu); the device was synchronised above
     delete t;
     if (e1 != cudaSuccess) return cuda_fail(e1);
     if (e2 != cudaSuccess) return cuda_fail(e2);
@@ -371,7 +431,7 @@ tt_status tt_traverse_bh(const tt_tree *t, const float *bodies, const int32_t *s
         tt_tree *mt = const_cast<tt_tree *>(t);
         std::lock_guard<std::mutex> lk(mt->grp_mu);
         if (!mt->d_grp) {
-            const int e = tt_bh_groups_build(t->dev.rec, t->hdr.n_nodes, s, &mt->d_grp);
+            const int e = tt_bh_groups_build(t->dev.rec, t->hdr.n_nodes, t->hdr.n_points, s, &mt->d_grp);
             if (e) return cuda_fail((cudaError_t)e);
         }
     }
@@ -388,7 +448,7 @@ tt_status tt_traverse_bh(const tt_tree *t, const float *bodies, const int32_t *s
     p.acc = reinterpret_cast<float4 *>(acc_out);
     return finish_launch(cfg.variant == TT_VARIANT_RECURSIVE ? tt_launch_bh_recursive(p, cfg)
                          : cfg.variant == TT_VARIANT_STACK   ? tt_launch_bh_stack(p, cfg)
-                         : cfg.variant == TT_VARIANT_GROUPS  ? tt_launch_bh_group(p, t->d_grp, cfg)
+                         : cfg.variant == TT_VARIANT_GROUPS  ? tt_launch_bh_group(p, t->d_grp, t->hdr.n_nodes, t->hdr.n_points, cfg)
                                                              : tt_launch_bh(p, cfg));  // ROPES
 }
 

@@ -824,3 +824,29 @@ def test_bh_default_falls_back_for_trees_deeper_than_group_stack(bh_small):
     with pytest.raises(P.TTError) as e:
         P.tt_traverse_bh(tree, bd, 0.5, 0.05, variant="groups")
     assert e.value.status == -4
+
+
+@pytest.mark.parametrize("case", ["shifted", "eps0", "foreign_ids"])
+def test_bh_groups_self_test_only_where_it_matters(case):
+    """The child-group walk drops its per-child self test in warps whose bodies
+    all sit exactly on their own leaves with eps > 0 (that leaf's term is then
+    f * 0 = 0).  Warps where that does not hold keep the test: queries moved
+    off their leaves (every other warp tile), eps = 0 (the term would be
+    inf * 0), and self ids naming other bodies' leaves."""
+    b = ttgen.plummer(20011, seed=311)
+    ot = oracle.build_oct(b)
+    tree = P.tt_tree_upload(P.build_oct(b))
+    q = b.copy()
+    ids = np.arange(len(b))
+    eps = 0.05
+    if case == "shifted":
+        moved = (np.arange(len(b)) // 64) % 2 == 1
+        q[moved, :3] += np.float32(1e-3)
+    elif case == "eps0":
+        eps = 0.0
+    else:
+        ids = np.roll(ids, 1)
+    acc = P.tt_traverse_bh(tree, dev(q), 0.5, eps, self_ids=perm_i32(ids), mode="lockstep").cpu().numpy()
+    ref = oracle.bh(ot, q, 0.5, eps, self_ids=ids)
+    assert np.isfinite(acc).all() and np.isfinite(ref.out[0]).all()
+    assert rel_err(acc, ref.out[0]).max() <= BH_TOL
