@@ -105,6 +105,33 @@ tt_status setup_common(const tt_tree *t, int kind, int64_t n, const tt_traverse_
     return TT_OK;
 }
 
+// Tile-counter arrays of tree handles, recycled: a tree per time step would
+// otherwise cudaMalloc / cudaFree 256 B per step (each cudaFree synchronises).
+std::mutex g_ctr_mu;
+std::vector<uint32_t *> g_ctr_free;
+
+cudaError_t counters_take(uint32_t **out) {
+    {
+        std::lock_guard<std::mutex> lk(g_ctr_mu);
+        if (!g_ctr_free.empty()) {
+            *out = g_ctr_free.back();
+            g_ctr_free.pop_back();
+            return cudaSuccess;
+        }
+    }
+    return cudaMalloc((void **)out, sizeof(uint32_t) * 2 * TT_COUNTER_SLOTS);
+}
+
+void counters_release(uint32_t *c) {
+    if (!c) return;
+    std::lock_guard<std::mutex> lk(g_ctr_mu);
+    if (g_ctr_free.size() >= 8) {
+        cudaFree(c);
+        return;
+    }
+    g_ctr_free.push_back(c);
+}
+
 // Wrap a device blob (already in device memory, owned) into a tree handle.
 tt_status adopt_blob(const tt_blob_header &h, void *d_blob, cudaStream_t cs, tt_tree **out) {
     tt_tree *t = new (std::nothrow) tt_tree();
@@ -112,11 +139,11 @@ tt_status adopt_blob(const tt_blob_header &h, void *d_blob, cudaStream_t cs, tt_
     t->hdr = h;
     t->bytes = (size_t)h.total;
     t->d_blob = d_blob;
-    cudaError_t e = cudaMalloc((void **)&t->d_counters, sizeof(uint32_t) * 2 * TT_COUNTER_SLOTS);
+    cudaError_t e = counters_take(&t->d_counters);
     if (e == cudaSuccess) e = cudaMemsetAsync(t->d_counters, 0, sizeof(uint32_t) * 2 * TT_COUNTER_SLOTS, cs);
     if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
     if (e != cudaSuccess) {
-        if (t->d_counters) cudaFree(t->d_counters);
+        if (t->d_counters) counters_release(t->d_counters);
         delete t;
         return cuda_fail(e);
     }
@@ -358,7 +385,8 @@ tt_status tt_tree_free(tt_tree *t) {
     } else {
         e1 = cudaFree(t->d_blob);
     }
-    cudaError_t e2 = cudaFree(t->d_counters);
+    counters_release(t->d_counters);  // the device is idle (synchronised above)
+    const cudaError_t e2 = cudaSuccess;
     tt_bh_groups_release(t->d_grp);  // recycled (kern_bh_group.cu); the device was synchronised above
     delete t;
     if (e1 != cudaSuccess) return cuda_fail(e1);
