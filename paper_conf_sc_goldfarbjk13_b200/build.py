@@ -18,7 +18,7 @@ CU = ["tt_api.cu", "kern_bh.cu", "kern_bh_group.cu", "kern_pc.cu", "kern_pc_spli
       "build_oct_gpu.cu", "build_kd_gpu.cu", "build_vp_gpu.cu", "build_nn_gpu.cu",
       "kern_integrate.cu", "kern_diag.cu"]
 CPP = ["host_build.cpp", "pack.cpp"]
-HDRS = ["tt_internal.h", "kern_common.cuh"]
+HDRS = ["tt_internal.h", "kern_common.cuh", "blob_cache.h", "build_common.cuh"]
 
 
 def _newer(src_list, out):

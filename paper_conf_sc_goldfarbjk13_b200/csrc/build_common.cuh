@@ -10,6 +10,7 @@
 #include <vector>
 
 #include "kern_common.cuh"
+#include "blob_cache.h"
 
 namespace {
 

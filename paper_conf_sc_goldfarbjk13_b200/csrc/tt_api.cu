@@ -14,6 +14,7 @@
 #include <vector>
 
 #include "tt_internal.h"
+#include "blob_cache.h"
 
 // kern_bh_group.cu: return a tree's child-group array for reuse
 void tt_bh_groups_release(void *grp);

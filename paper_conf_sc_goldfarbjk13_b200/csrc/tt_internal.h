@@ -168,11 +168,6 @@ int tt_launch_vp_recursive(const tt_vp_params &p, int dim, const tt_launch_cfg &
 // explicit rope-stack variant, unguided kernels (kern_stack.cu)
 int tt_launch_bh_stack(const tt_bh_params &p, const tt_launch_cfg &cfg);
 // lockstep walk by child groups (kern_bh_group.cu)
-// Device blobs of GPU-built trees: cudaMalloc'd, recycled on tt_tree_free
-// (after a device synchronisation) into a small cache (tt_api.cu).
-int tt_blob_take(size_t bytes, void **out);  // a cudaError_t
-void tt_blob_release(void *blob);  // caller guarantees the blob is idle
-bool tt_blob_is_cached_kind(void *blob);
 int tt_bh_groups_build(const void *rec, long long nn, long long np, void *stream, void **grp_out);
 int tt_launch_bh_group(const tt_bh_params &p, const void *grp, long long nn, long long np, const tt_launch_cfg &cfg);
 int tt_launch_pc_stack(const tt_pc_params &p, int dim, const tt_launch_cfg &cfg);
