@@ -244,11 +244,14 @@ __global__ void __launch_bounds__(kBlock, 4) bh_kernel(const tt_bh_params P) {
                         w[2 * p] = o0 ? INT_MAX : min(w[2 * p], lvl);
                         w[2 * p + 1] = o1 ? INT_MAX : min(w[2 * p + 1], lvl);
                         // branch-free update (some lane almost always interacts)
-                        const float2 mw = make_float2(a0 && !o0 && t.z != self[2 * p] ? g.w : 0.f,
-                                                      a1 && !o1 && t.z != self[2 * p + 1] ? g.w : 0.f);
+                        const bool k0 = a0 && !o0 && t.z != self[2 * p];
+                        const bool k1 = a1 && !o1 && t.z != self[2 * p + 1];
+                        const float2 mw = make_float2(k0 ? g.w : 0.f, k1 ? g.w : 0.f);
                         const float2 r = add2_rn(drsq, e22);
                         const float2 inv = make_float2(rsqrt_ftz(r.x), rsqrt_ftz(r.y));
-                        const float2 f = mul2_rn(mul2_rn(mw, mul2_rn(inv, inv)), inv);
+                        float2 f = mul2_rn(mul2_rn(mw, mul2_rn(inv, inv)), inv);
+                        // eps = 0: a skipped term at distance 0 has inv = inf (0 * inf)
+                        f = make_float2(k0 ? f.x : 0.f, k1 ? f.y : 0.f);
                         ax[p] = fma2_rn(f, dx, ax[p]);
                         ay[p] = fma2_rn(f, dy, ay[p]);
                         az[p] = fma2_rn(f, dz, az[p]);

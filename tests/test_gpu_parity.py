@@ -826,8 +826,9 @@ def test_bh_default_falls_back_for_trees_deeper_than_group_stack(bh_small):
     assert e.value.status == -4
 
 
-@pytest.mark.parametrize("case", ["shifted", "eps0", "foreign_ids"])
-def test_bh_groups_self_test_only_where_it_matters(case):
+@pytest.mark.parametrize("case,variant", [("shifted", "autoropes"), ("eps0", "autoropes"), ("foreign_ids", "autoropes"),
+                                          ("eps0", "ropes")])
+def test_bh_groups_self_test_only_where_it_matters(case, variant):
     """The child-group walk drops its per-child self test in warps whose bodies
     all sit exactly on their own leaves with eps > 0 (that leaf's term is then
     f * 0 = 0).  Warps where that does not hold keep the test: queries moved
@@ -846,7 +847,8 @@ def test_bh_groups_self_test_only_where_it_matters(case):
         eps = 0.0
     else:
         ids = np.roll(ids, 1)
-    acc = P.tt_traverse_bh(tree, dev(q), 0.5, eps, self_ids=perm_i32(ids), mode="lockstep").cpu().numpy()
+    acc = P.tt_traverse_bh(tree, dev(q), 0.5, eps, self_ids=perm_i32(ids), mode="lockstep",
+                           variant=variant).cpu().numpy()
     ref = oracle.bh(ot, q, 0.5, eps, self_ids=ids)
     assert np.isfinite(acc).all() and np.isfinite(ref.out[0]).all()
     assert rel_err(acc, ref.out[0]).max() <= BH_TOL
