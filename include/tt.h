@@ -301,7 +301,7 @@ typedef enum tt_variant {
 
 /* Barnes-Hut force pass (Fig.9): bodies float4 (x,y,z,m) rows;
  * self_ids[i] (nullable; default i) is the leaf body id whose interaction
- * point i skips (R9).  A cell is opened iff it is a cell and
+ * point i skips (R9); a negative id skips nothing.  A cell is opened iff it is a cell and
  * |com - x|^2 < dsq_L, dsq_L = dsq_root * 0.25^L, dsq_root = (side/theta)^2
  * (theta == 0 -> +inf: every cell opened).  acc_out: float4 (ax,ay,az,0),
  * G = 1, softening eps.  Opening decisions use the pinned fp32 sequence R0. */

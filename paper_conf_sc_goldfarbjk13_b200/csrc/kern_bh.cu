@@ -22,6 +22,10 @@
 
 #include "kern_common.cuh"
 
+// a negative self id means "no self leaf": -2 matches no record's body field
+// (cells carry -1 there)
+static __device__ __forceinline__ int tt_self_id(int s) { return s < 0 ? -2 : s; }
+
 namespace {
 
 using namespace tt;
@@ -127,7 +131,7 @@ __global__ void __launch_bounds__(kBlock, 4) bh_kernel(const tt_bh_params P) {
             bd[j].valid = pos < n;
             bd[j].pid = bd[j].valid ? (P.c.order ? (long long)P.c.order[pos] : pos) : 0;
             bd[j].b = bd[j].valid ? __ldg(P.bodies + bd[j].pid) : make_float4(0.f, 0.f, 0.f, 0.f);
-            bd[j].self = bd[j].valid ? (P.self_ids ? __ldg(P.self_ids + bd[j].pid) : (int)bd[j].pid) : -2;
+            bd[j].self = bd[j].valid ? (P.self_ids ? tt_self_id(__ldg(P.self_ids + bd[j].pid)) : (int)bd[j].pid) : -2;
             bd[j].wait = bd[j].valid ? INT_MAX : -1;
             bd[j].visits = 0;
         }

@@ -31,6 +31,10 @@
 
 #include "kern_common.cuh"
 
+// a negative self id means "no self leaf": -2 matches no record's body field
+// (cells carry -1 there)
+static __device__ __forceinline__ int tt_self_id(int s) { return s < 0 ? -2 : s; }
+
 
 namespace {
 
@@ -131,7 +135,7 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
             valid[j] = pos < n;
             pid[j] = valid[j] ? (P.c.order ? (long long)P.c.order[pos] : pos) : 0;
             b[j] = valid[j] ? __ldg(P.bodies + pid[j]) : make_float4(0.f, 0.f, 0.f, 0.f);
-            self[j] = valid[j] ? (P.self_ids ? __ldg(P.self_ids + pid[j]) : (int)pid[j]) : -2;
+            self[j] = valid[j] ? (P.self_ids ? tt_self_id(__ldg(P.self_ids + pid[j])) : (int)pid[j]) : -2;
         }
         bool lock = P.c.mode != TT_MODE_INDEPENDENT;
         if (P.c.mode == TT_MODE_AUTO && P.c.auto_min_depth > 0) {
@@ -175,6 +179,9 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
         // finite (eps > 0).  A warp whose bodies all sit exactly on their
         // own leaves (the normal case: the tree was built from them)
         // walks without the per-child test; others keep it.
+        // (eps = 0: every warp keeps the checked walk, whose select also
+        // zeroes opened cells at distance 0 -- 0 * inf otherwise)
+        const bool eps_ok = isfinite(rsqrt_ftz(__fadd_rn(0.f, P.eps2)));
         bool ok[kBPL];
 #pragma unroll
         for (int j = 0; j < kBPL; ++j) {
@@ -190,6 +197,7 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                     ok[j] = c.x == b[j].x && c.y == b[j].y && c.z == b[j].z && isfinite(f);
                 }
             }
+            ok[j] = ok[j] && eps_ok;
         }
         const bool need_self = __any_sync(TT_FULL, !(ok[0] && ok[1]));
         if (lock) {

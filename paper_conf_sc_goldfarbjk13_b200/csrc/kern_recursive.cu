@@ -13,6 +13,10 @@
 // Selected with tt_traverse_opts.variant = TT_VARIANT_RECURSIVE.
 #include "kern_common.cuh"
 
+// a negative self id means "no self leaf": -2 matches no record's body field
+// (cells carry -1 there)
+static __device__ __forceinline__ int tt_self_id(int s) { return s < 0 ? -2 : s; }
+
 namespace {
 
 using namespace tt;
@@ -55,7 +59,7 @@ __global__ void __launch_bounds__(kBlock) bh_rec_kernel(const tt_bh_params P) {
     for (long long pos = blockIdx.x * (long long)blockDim.x + threadIdx.x; pos < P.c.n;
          pos += (long long)gridDim.x * blockDim.x) {
         const long long pid = P.c.order ? (long long)P.c.order[pos] : pos;
-        BhCtx c{rec, __ldg(P.bodies + pid), P.self_ids ? __ldg(P.self_ids + pid) : (int)pid, P.eps2, 0, 0, 0, 0};
+        BhCtx c{rec, __ldg(P.bodies + pid), P.self_ids ? tt_self_id(__ldg(P.self_ids + pid)) : (int)pid, P.eps2, 0, 0, 0, 0};
         bh_rec(c, 0, P.dsq_root);
         P.acc[pid] = make_float4((float)c.ax, (float)c.ay, (float)c.az, 0.f);
         if (P.c.st_visits) P.c.st_visits[pid] = c.visits;

@@ -27,6 +27,10 @@
 
 #include "kern_common.cuh"
 
+// a negative self id means "no self leaf": -2 matches no record's body field
+// (cells carry -1 there)
+static __device__ __forceinline__ int tt_self_id(int s) { return s < 0 ? -2 : s; }
+
 namespace {
 
 using namespace tt;
@@ -104,7 +108,7 @@ __global__ void __launch_bounds__(kBlock) bh_stack_kernel(const tt_bh_params P, 
         const long long pid = valid ? (P.c.order ? (long long)P.c.order[pos] : pos) : 0;
         BhLane L;
         L.b = valid ? __ldg(P.bodies + pid) : make_float4(0.f, 0.f, 0.f, 0.f);
-        L.self = valid ? (P.self_ids ? __ldg(P.self_ids + pid) : (int)pid) : -2;
+        L.self = valid ? (P.self_ids ? tt_self_id(__ldg(P.self_ids + pid)) : (int)pid) : -2;
         L.ax = L.ay = L.az = 0.f;
         L.AX = L.AY = L.AZ = 0.0;
         unsigned visits = 0, fetches = 0, steps = 0;

@@ -827,7 +827,7 @@ def test_bh_default_falls_back_for_trees_deeper_than_group_stack(bh_small):
 
 
 @pytest.mark.parametrize("case,variant", [("shifted", "autoropes"), ("eps0", "autoropes"), ("foreign_ids", "autoropes"),
-                                          ("eps0", "ropes")])
+                                          ("eps0", "ropes"), ("eps0_no_self", "autoropes")])
 def test_bh_groups_self_test_only_where_it_matters(case, variant):
     """The child-group walk drops its per-child self test in warps whose bodies
     all sit exactly on their own leaves with eps > 0 (that leaf's term is then
@@ -845,6 +845,14 @@ def test_bh_groups_self_test_only_where_it_matters(case, variant):
         q[moved, :3] += np.float32(1e-3)
     elif case == "eps0":
         eps = 0.0
+    elif case == "eps0_no_self":
+        # self ids naming no leaf and eps = 0: queries strictly inside the
+        # cloud, off every body (a body's own leaf would be a 1/0 term)
+        eps = 0.0
+        ids = np.full(len(b), -1)
+        q = q[:4096].copy()
+        q[:, :3] = (q[:, :3] * np.float32(0.5) + np.float32(1e-4)).astype(np.float32)
+        ids = ids[:4096]
     else:
         ids = np.roll(ids, 1)
     acc = P.tt_traverse_bh(tree, dev(q), 0.5, eps, self_ids=perm_i32(ids), mode="lockstep",
