@@ -117,7 +117,7 @@ inline cudaError_t alloc_blob(const tt_blob_header &h, cudaStream_t s, void **bl
     if (e) return e;
     if ((e = cudaMemsetAsync(*blob, 0, h.total, s)) ||
         (e = cudaMemcpyAsync(*blob, &h, sizeof(h), cudaMemcpyHostToDevice, s))) {
-        tt_blob_release(*blob);
+        tt_blob_discard(*blob);
         *blob = nullptr;
     }
     return e;

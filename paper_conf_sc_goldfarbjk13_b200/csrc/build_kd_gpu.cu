@@ -358,7 +358,7 @@ int tt_build_kd_gpu_impl(const float *pts, long long n, int D, int ld, int L, vo
     kd_points_kernel<<<G, 256, 0, s>>>(n, D, dp, pts, ld, ids, reinterpret_cast<float *>(base + h.off_pts),
                                       reinterpret_cast<int *>(base + h.off_pid));
     if ((e = cudaGetLastError()) || (e = cudaStreamSynchronize(s))) {
-        tt_blob_release(blob);
+        tt_blob_discard(blob);
         return e;
     }
     *hdr_out = h;

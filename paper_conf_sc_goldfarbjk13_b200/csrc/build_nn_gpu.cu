@@ -294,7 +294,7 @@ int tt_build_nn_gpu_impl(const float *pts, long long n, int D, int ld, void *str
                                                      reinterpret_cast<float *>(base + h.off_vpt),
                                                      reinterpret_cast<int *>(base + h.off_pid));
     if ((e = cudaGetLastError()) || (e = cudaStreamSynchronize(s))) {
-        tt_blob_release(blob);
+        tt_blob_discard(blob);
         return e;
     }
     *hdr_out = h;

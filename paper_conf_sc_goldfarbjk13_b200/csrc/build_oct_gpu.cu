@@ -307,6 +307,9 @@ int tt_build_oct_gpu_impl(const float *bodies_f, long long n, void *stream, tt_b
     for (int d = 0; d < 3; ++d) h.root_center[d] = cube.c[d];
     h.root_side = cube.side;
     h.rec_bytes = 32;
+    // R9 trees: more than 8 children only in depth-32 buckets (height 33),
+    // whose children are leaves (same bits as pack.cpp computes)
+    h.oct_flags = (height <= 32 ? TT_OCT_NARROW : 0) | TT_OCT_FEW_CELL_KIDS;
     int *newidx = W.get<int>(n_nodes);
     if (W.e) return W.e;
     if ((e = renumber_top_first(A.level, n_nodes, 32, h, newidx, W))) return e;
@@ -319,7 +322,7 @@ int tt_build_oct_gpu_impl(const float *bodies_f, long long n, void *stream, tt_b
     records_kernel<<<GN, 256, 0, s>>>(n_nodes, A, newidx, rec);
     leaf_fix_kernel<<<GN, 256, 0, s>>>(bodies, n_nodes, A, newidx, rec);
     if ((e = cudaGetLastError()) || (e = cudaStreamSynchronize(s))) {
-        tt_blob_release(blob);
+        tt_blob_discard(blob);
         return e;
     }
     *hdr_out = h;

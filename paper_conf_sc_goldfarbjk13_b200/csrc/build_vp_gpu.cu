@@ -205,7 +205,7 @@ int build_vp(const float *pts, long long n, int ld, cudaStream_t s, tt_blob_head
                                         reinterpret_cast<float *>(base + h.off_vpt),
                                         reinterpret_cast<int *>(base + h.off_pid));
     if ((e = cudaGetLastError()) || (e = cudaStreamSynchronize(s))) {
-        tt_blob_release(blob);
+        tt_blob_discard(blob);
         return e;
     }
     *hdr_out = h;

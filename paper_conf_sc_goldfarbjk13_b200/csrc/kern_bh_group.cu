@@ -95,7 +95,9 @@ __device__ __forceinline__ float dsq_at(int dsq_bits, int lvl) { return __int_as
 #ifndef TT_BHG_MINB
 #define TT_BHG_MINB 4
 #endif
-template <bool STATS, bool EXP_DSQ>
+// WIDE: some node has more than 8 children (a depth-32 bucket of more than 8
+// coincident bodies, R9, or a custom tree): groups are staged 8 at a time.
+template <bool STATS, bool EXP_DSQ, bool WIDE>
 __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_bh_params P, const tt_oct_rec *grp,
                                                                                  const int *leaf_of, long long np) {
     extern __shared__ __align__(128) unsigned char smem[];
@@ -217,17 +219,21 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                     const bool in0 = (m0 >> lane) & 1u, in1 = (m1 >> lane) & 1u;
                     // stage the group: lane k loads child k (one request for the
                     // whole group, one round trip), the warp reads them back from
-                    // shared memory with broadcast loads
-                    if (lane < gnk) {
+                    // shared memory with broadcast loads; the buffer holds 8
+                    // records, so a WIDE tree stages larger groups 8 at a time
+                    const int gall = gnk;
+                    for (int c0 = 0;; c0 += 8) {
+                    const int cn = WIDE ? min(gall - c0, 8) : gall;
+                    if (lane < cn) {
                         float4 sg;
                         int4 st4;
-                        ldg_rec256(grp + goff + lane, sg, st4);
+                        ldg_rec256(grp + goff + c0 + lane, sg, st4);
                         gbuf[lane] = sg;
                         tbuf[lane] = st4;
                     }
                     __syncwarp();
 #pragma unroll 1
-                    for (int k = 0; k < gnk; ++k) {
+                    for (int k = 0; k < cn; ++k) {
                         const float4 g = gbuf[k];
                         const int4 t = tbuf[k];
                         if (STATS) {
@@ -264,8 +270,10 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                             ++sp;
                         }
                     }
-                    __syncwarp();  // the group buffer is reused by the next pop
-                    since_flush += gnk;
+                    __syncwarp();  // the group buffer is reused by the next chunk / pop
+                    if (!WIDE || c0 + 8 >= gall) break;
+                    }
+                    since_flush += gall;
                     if (since_flush >= kFlushEvery) {  // warp-uniform cadence
                         X[0] += (double)ax.x;
                         Y[0] += (double)ay.x;
@@ -349,10 +357,10 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
     cta_finish(P.c.counter);
 }
 
-template <bool STATS, bool EXP_DSQ>
+template <bool STATS, bool EXP_DSQ, bool WIDE>
 int launch(const tt_bh_params &p, const tt_oct_rec *grp, const int *leaf_of, long long np, const tt_launch_cfg &cfg) {
     const size_t smem = kSmemHdr + (size_t)(kBlock / 32) * kStackPerWarp * sizeof(GroupEntry) + (kBlock / 32) * 16 * 16;
-    auto kern = bh_group_kernel<STATS, EXP_DSQ>;
+    auto kern = bh_group_kernel<STATS, EXP_DSQ, WIDE>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return (int)e;
     int dev = 0, nsm = 0, occ = 0;
@@ -374,19 +382,26 @@ int launch(const tt_bh_params &p, const tt_oct_rec *grp, const int *leaf_of, lon
 // Group arrays are recycled between trees: BH time stepping builds a tree,
 // and so a group array, every step, and a fresh cudaMalloc per step costs
 // milliseconds (pool allocations were fragmented by the sort's scratch).
-// tt_tree_free returns the array here after its cudaFree of the blob has
-// synchronised the device, so a recycled array is never still in use.
+// tt_tree_free returns the array here only after a successful device
+// synchronisation, so a recycled array is never still in use; arrays are
+// handed out again only on the device they were allocated on.
+struct GrpInfo {
+    size_t bytes;
+    int device;
+};
 std::mutex g_grp_mu;
-std::unordered_map<void *, size_t> g_grp_size;  // every group array ever allocated
+std::unordered_map<void *, GrpInfo> g_grp_info;  // every group array alive or free
 std::vector<void *> g_grp_free;
 
 void *grp_take(size_t bytes) {
+    int dev = -1;
+    cudaGetDevice(&dev);
     {
         std::lock_guard<std::mutex> lk(g_grp_mu);
         for (size_t i = 0; i < g_grp_free.size(); ++i) {
             void *p = g_grp_free[i];
-            const size_t sz = g_grp_size[p];
-            if (sz >= bytes && sz <= 2 * bytes) {
+            const GrpInfo &gi = g_grp_info[p];
+            if (gi.device == dev && gi.bytes >= bytes && gi.bytes <= 2 * bytes) {
                 g_grp_free.erase(g_grp_free.begin() + (long)i);
                 return p;
             }
@@ -395,18 +410,27 @@ void *grp_take(size_t bytes) {
     void *p = nullptr;
     if (cudaMalloc(&p, bytes) != cudaSuccess) return nullptr;
     std::lock_guard<std::mutex> lk(g_grp_mu);
-    g_grp_size[p] = bytes;
+    g_grp_info[p] = GrpInfo{bytes, dev};
     return p;
 }
 
 }  // namespace
 
+void tt_bh_groups_discard(void *grp) {
+    if (!grp) return;
+    {
+        std::lock_guard<std::mutex> lk(g_grp_mu);
+        g_grp_info.erase(grp);
+    }
+    cudaFree(grp);
+}
+
 void tt_bh_groups_release(void *grp) {
     if (!grp) return;
     std::lock_guard<std::mutex> lk(g_grp_mu);
     if (g_grp_free.size() >= 4) {  // keep a few
+        g_grp_info.erase(grp);
         cudaFree(grp);
-        g_grp_size.erase(grp);
         return;
     }
     g_grp_free.push_back(grp);
@@ -444,19 +468,27 @@ int tt_bh_groups_build(const void *rec, long long nn, long long np, void *stream
     if (goff) cudaFreeAsync(goff, s);
     if (nk) cudaFreeAsync(nk, s);
     if (e) {
-        if (grp) tt_bh_groups_release(grp);
+        if (grp) {
+            cudaStreamSynchronize(s);
+            tt_bh_groups_discard(grp);
+        }
         return (int)e;
     }
     *grp_out = grp;
     return 0;
 }
 
-int tt_launch_bh_group(const tt_bh_params &p, const void *grp, long long nn, long long np, const tt_launch_cfg &cfg) {
+int tt_launch_bh_group(const tt_bh_params &p, const void *grp, long long nn, long long np, bool wide,
+                       const tt_launch_cfg &cfg) {
     const bool stats = p.c.st_visits || p.c.st_warp_fetches || p.c.st_warp_steps || p.c.st_warp_mode;
     const float r = p.dsq_root;
     const bool exp_ok = r < INFINITY && r > 0.f && std::ldexp((double)r, -2 * p.c.height) >= (double)FLT_MIN;
     const tt_oct_rec *g = static_cast<const tt_oct_rec *>(grp);
     const int *lf = reinterpret_cast<const int *>(g + nn);
-    if (stats) return exp_ok ? launch<true, true>(p, g, lf, np, cfg) : launch<true, false>(p, g, lf, np, cfg);
-    return exp_ok ? launch<false, true>(p, g, lf, np, cfg) : launch<false, false>(p, g, lf, np, cfg);
+    if (wide) {  // rare (buckets of > 8 coincident bodies): no specialisations beyond stats
+        if (stats) return launch<true, false, true>(p, g, lf, np, cfg);
+        return launch<false, false, true>(p, g, lf, np, cfg);
+    }
+    if (stats) return exp_ok ? launch<true, true, false>(p, g, lf, np, cfg) : launch<true, false, false>(p, g, lf, np, cfg);
+    return exp_ok ? launch<false, true, false>(p, g, lf, np, cfg) : launch<false, false, false>(p, g, lf, np, cfg);
 }

@@ -110,6 +110,24 @@ void plan(const tt_tree_desc *d, tt_blob_header &h, std::vector<int32_t> *newidx
     }
     h.top_levels = L;
     h.top_count = (int32_t)acc;
+    if (d->kind == TT_KIND_OCT) {
+        // what the child-group BH walk may assume (kern_bh_group.cu): at most 8
+        // children staged per group and at most 8 cell children pushed per level.
+        // R9 trees: only depth-32 buckets exceed 8 children, and those are
+        // leaves -- the GPU builder writes the same bits from the height alone.
+        int64_t max_kids = 0, max_cell_kids = 0;
+        for (int64_t v = 0; v < d->n_nodes; ++v) {
+            int64_t k = 0, kc = 0;
+            for (int32_t c = d->first_child[v]; c >= 0 && c < d->skip[v]; c = d->skip[c]) {
+                ++k;
+                kc += d->first_child[c] >= 0;
+            }
+            if (k > max_kids) max_kids = k;
+            if (kc > max_cell_kids) max_cell_kids = kc;
+        }
+        h.oct_flags = ((d->height <= 32 && max_kids <= 8) ? TT_OCT_NARROW : 0) |
+                      (max_cell_kids <= 8 ? TT_OCT_FEW_CELL_KIDS : 0);
+    }
     h.rec_bytes = (d->kind == TT_KIND_VP || d->kind == TT_KIND_NN) ? 16 : 32;
     uint64_t off = align256(sizeof(tt_blob_header));
     h.off_rec = off;

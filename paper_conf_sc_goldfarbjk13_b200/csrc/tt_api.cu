@@ -16,8 +16,10 @@
 #include "tt_internal.h"
 #include "blob_cache.h"
 
-// kern_bh_group.cu: return a tree's child-group array for reuse
+// kern_bh_group.cu: return a tree's child-group array for reuse (device
+// idle), or free it for good
 void tt_bh_groups_release(void *grp);
+void tt_bh_groups_discard(void *grp);
 
 // build_nn_gpu.cu (declared here rather than in tt_internal.h)
 int tt_build_nn_gpu_impl(const float *pts, long long n, int dim, int ld, void *stream, tt_blob_header *hdr,
@@ -108,29 +110,36 @@ tt_status setup_common(const tt_tree *t, int kind, int64_t n, const tt_traverse_
 
 // Tile-counter arrays of tree handles, recycled: a tree per time step would
 // otherwise cudaMalloc / cudaFree 256 B per step (each cudaFree synchronises).
+// (kept per device: a process that switches devices never gets another GPU's)
 std::mutex g_ctr_mu;
-std::vector<uint32_t *> g_ctr_free;
+std::vector<std::pair<uint32_t *, int>> g_ctr_free;
 
 cudaError_t counters_take(uint32_t **out) {
+    int dev = -1;
+    cudaGetDevice(&dev);
     {
         std::lock_guard<std::mutex> lk(g_ctr_mu);
-        if (!g_ctr_free.empty()) {
-            *out = g_ctr_free.back();
-            g_ctr_free.pop_back();
+        for (size_t i = g_ctr_free.size(); i-- > 0;) {
+            if (g_ctr_free[i].second != dev) continue;
+            *out = g_ctr_free[i].first;
+            g_ctr_free.erase(g_ctr_free.begin() + (long)i);
             return cudaSuccess;
         }
     }
     return cudaMalloc((void **)out, sizeof(uint32_t) * 2 * TT_COUNTER_SLOTS);
 }
 
+// caller guarantees the device is idle and current
 void counters_release(uint32_t *c) {
     if (!c) return;
+    int dev = -1;
+    cudaGetDevice(&dev);
     std::lock_guard<std::mutex> lk(g_ctr_mu);
     if (g_ctr_free.size() >= 8) {
         cudaFree(c);
         return;
     }
-    g_ctr_free.push_back(c);
+    g_ctr_free.emplace_back(c, dev);
 }
 
 // Wrap a device blob (already in device memory, owned) into a tree handle.
@@ -174,19 +183,29 @@ tt_status finish_launch(int err) {
 // freed blobs are kept (at most kBlobCacheKeep) and reused by a later build
 // whose blob fits in [bytes, 2 * bytes].
 namespace {
+struct BlobInfo {
+    size_t bytes;
+    int device;
+};
 std::mutex g_blob_mu;
-std::unordered_map<void *, size_t> g_blob_size;  // every cached-kind blob alive or free
+std::unordered_map<void *, BlobInfo> g_blob_info;  // every cached-kind blob alive or free
 std::vector<void *> g_blob_free;
 constexpr size_t kBlobCacheKeep = 2;
+int current_device() {
+    int d = -1;
+    cudaGetDevice(&d);
+    return d;
+}
 }  // namespace
 
 int tt_blob_take(size_t bytes, void **out) {
+    const int dev = current_device();
     {
         std::lock_guard<std::mutex> lk(g_blob_mu);
         for (size_t i = 0; i < g_blob_free.size(); ++i) {
             void *p = g_blob_free[i];
-            const size_t sz = g_blob_size[p];
-            if (sz >= bytes && sz <= 2 * bytes) {
+            const BlobInfo &bi = g_blob_info[p];
+            if (bi.device == dev && bi.bytes >= bytes && bi.bytes <= 2 * bytes) {
                 g_blob_free.erase(g_blob_free.begin() + (long)i);
                 *out = p;
                 return cudaSuccess;
@@ -197,14 +216,14 @@ int tt_blob_take(size_t bytes, void **out) {
     cudaError_t e = cudaMalloc(&p, bytes);
     if (e) return e;
     std::lock_guard<std::mutex> lk(g_blob_mu);
-    g_blob_size[p] = bytes;
+    g_blob_info[p] = BlobInfo{bytes, dev};
     *out = p;
     return cudaSuccess;
 }
 
 bool tt_blob_is_cached_kind(void *blob) {
     std::lock_guard<std::mutex> lk(g_blob_mu);
-    return g_blob_size.count(blob) != 0;
+    return g_blob_info.count(blob) != 0;
 }
 
 void tt_blob_release(void *blob) {
@@ -214,10 +233,19 @@ void tt_blob_release(void *blob) {
         // evict the oldest free blob, keep the newest
         void *old = g_blob_free.front();
         g_blob_free.erase(g_blob_free.begin());
-        g_blob_size.erase(old);
+        g_blob_info.erase(old);
         cudaFree(old);
     }
     g_blob_free.push_back(blob);
+}
+
+void tt_blob_discard(void *blob) {
+    if (!blob) return;
+    {
+        std::lock_guard<std::mutex> lk(g_blob_mu);
+        g_blob_info.erase(blob);  // a later cudaMalloc may return this address
+    }
+    cudaFree(blob);
 }
 
 extern "C" {
@@ -295,11 +323,11 @@ tt_status tt_build_oct_device(const float *bodies, int64_t n, tt_stream s, tt_tr
     const int e = tt_build_oct_gpu_impl(bodies, n, s, &h, &d_blob);
     if (e) return cuda_fail((cudaError_t)e);
     if (h.height > TT_MAX_HEIGHT) {
-        cudaFree(d_blob);
+        tt_blob_discard(d_blob);
         return TT_ERR_TREE_TOO_DEEP;
     }
     st = adopt_blob(h, d_blob, (cudaStream_t)s, out);
-    if (st != TT_OK) cudaFree(d_blob);
+    if (st != TT_OK) tt_blob_discard(d_blob);
     return st;
 }
 
@@ -314,7 +342,7 @@ tt_status tt_build_kd_device(const float *pts, int64_t n, int32_t dim, int32_t l
     const int e = tt_build_kd_gpu_impl(pts, n, dim, ld, leaf_size, s, &h, &d_blob);
     if (e) return cuda_fail((cudaError_t)e);
     st = adopt_blob(h, d_blob, (cudaStream_t)s, out);
-    if (st != TT_OK) cudaFree(d_blob);
+    if (st != TT_OK) tt_blob_discard(d_blob);
     return st;
 }
 
@@ -329,11 +357,11 @@ tt_status tt_build_vp_device(const float *pts, int64_t n, int32_t dim, int32_t l
     const int e = tt_build_vp_gpu_impl(pts, n, dim, ld, s, &h, &d_blob);
     if (e) return cuda_fail((cudaError_t)e);
     if (h.height > TT_MAX_HEIGHT) {
-        cudaFree(d_blob);
+        tt_blob_discard(d_blob);
         return TT_ERR_TREE_TOO_DEEP;
     }
     st = adopt_blob(h, d_blob, (cudaStream_t)s, out);
-    if (st != TT_OK) cudaFree(d_blob);
+    if (st != TT_OK) tt_blob_discard(d_blob);
     return st;
 }
 
@@ -347,11 +375,11 @@ tt_status tt_build_nn_device(const float *pts, int64_t n, int32_t dim, int32_t l
     const int e = tt_build_nn_gpu_impl(pts, n, dim, ld, s, &h, &d_blob);
     if (e) return cuda_fail((cudaError_t)e);
     if (h.height > TT_MAX_HEIGHT) {
-        cudaFree(d_blob);
+        tt_blob_discard(d_blob);
         return TT_ERR_TREE_TOO_DEEP;
     }
     st = adopt_blob(h, d_blob, (cudaStream_t)s, out);
-    if (st != TT_OK) cudaFree(d_blob);
+    if (st != TT_OK) tt_blob_discard(d_blob);
     return st;
 }
 
@@ -379,20 +407,24 @@ tt_status tt_tree_upload(const tt_tree_desc *d, tt_stream s, tt_tree **out) {
 
 tt_status tt_tree_free(tt_tree *t) {
     if (!t) return TT_OK;
-    cudaError_t e1;
-    if (tt_blob_is_cached_kind(t->d_blob)) {  // GPU-built: recycled once the device is idle
-        e1 = cudaDeviceSynchronize();
-        if (e1 == cudaSuccess) tt_blob_release(t->d_blob);
+    // Buffers are recycled (blob of a GPU-built tree, tile counters, child
+    // groups) only once the device is known idle; if the synchronisation
+    // fails they are freed instead, never handed to a later tree.
+    const cudaError_t e1 = cudaDeviceSynchronize();
+    const bool idle = e1 == cudaSuccess;
+    if (tt_blob_is_cached_kind(t->d_blob)) {
+        if (idle) tt_blob_release(t->d_blob);
+        else tt_blob_discard(t->d_blob);
     } else {
-        e1 = cudaFree(t->d_blob);
+        cudaFree(t->d_blob);
     }
-    counters_release(t->d_counters);  // the device is idle (synchronised above)
-    const cudaError_t e2 = cudaSuccess;
-    tt_bh_groups_release(t->d_grp);  // recycled (kern_bh_group.cu); the device was synchronised above
+    if (idle) counters_release(t->d_counters);
+    else cudaFree(t->d_counters);
+    if (idle) tt_bh_groups_release(t->d_grp);
+    else tt_bh_groups_discard(t->d_grp);
+    if (t->grp_ready) cudaEventDestroy(t->grp_ready);
     delete t;
-    if (e1 != cudaSuccess) return cuda_fail(e1);
-    if (e2 != cudaSuccess) return cuda_fail(e2);
-    return TT_OK;
+    return idle ? TT_OK : cuda_fail(e1);
 }
 
 tt_status tt_tree_get_info(const tt_tree *t, tt_tree_info *o) {
@@ -451,18 +483,35 @@ tt_status tt_traverse_bh(const tt_tree *t, const float *bodies, const int32_t *s
     if (cfg.variant == TT_VARIANT_SPLIT) return TT_ERR_UNSUPPORTED;  // PC only
     // BH default: lockstep warps walk by child groups (kern_bh_group.cu);
     // TT_VARIANT_ROPES keeps the per-node lockstep walk over ropes (kern_bh.cu)
-    // (the child-group stack holds 8 entries per level: deeper custom trees
-    // take the stackless per-node walk, or fail if groups were requested)
-    const bool groups_fit = 8 * (t->hdr.height + 2) <= 320;  // kStackPerWarp of kern_bh_group.cu
+    // (the child-group stack holds 8 entries per level: deeper custom trees,
+    // or trees with more than 8 cell children per node -- tt_blob_header
+    // oct_flags -- take the stackless per-node walk, or fail if groups were
+    // requested; more than 8 children in all (depth-32 buckets) are staged 8
+    // at a time by the WIDE kernel)
+    const bool groups_fit = 8 * (t->hdr.height + 2) <= 320 &&  // kStackPerWarp of kern_bh_group.cu
+                            (t->hdr.oct_flags & TT_OCT_FEW_CELL_KIDS);
+    const bool wide = !(t->hdr.oct_flags & TT_OCT_NARROW);
     if (cfg.variant == TT_VARIANT_AUTOROPES) cfg.variant = groups_fit ? TT_VARIANT_GROUPS : TT_VARIANT_ROPES;
     if (cfg.variant == TT_VARIANT_GROUPS && !groups_fit) return TT_ERR_TREE_TOO_DEEP;
     if (cfg.variant == TT_VARIANT_GROUPS) {
         tt_tree *mt = const_cast<tt_tree *>(t);
         std::lock_guard<std::mutex> lk(mt->grp_mu);
         if (!mt->d_grp) {
-            const int e = tt_bh_groups_build(t->dev.rec, t->hdr.n_nodes, t->hdr.n_points, s, &mt->d_grp);
+            void *g = nullptr;
+            int e = tt_bh_groups_build(t->dev.rec, t->hdr.n_nodes, t->hdr.n_points, s, &g);
             if (e) return cuda_fail((cudaError_t)e);
+            // launches on other streams wait for the build (queued on s)
+            if (!mt->grp_ready) e = cudaEventCreateWithFlags(&mt->grp_ready, cudaEventDisableTiming);
+            if (!e) e = cudaEventRecord(mt->grp_ready, (cudaStream_t)s);
+            if (e) {
+                cudaStreamSynchronize((cudaStream_t)s);
+                tt_bh_groups_release(g);
+                return cuda_fail((cudaError_t)e);
+            }
+            mt->d_grp = g;
         }
+        const cudaError_t e = cudaStreamWaitEvent((cudaStream_t)s, mt->grp_ready, 0);
+        if (e) return cuda_fail(e);
     }
     p.bodies = reinterpret_cast<const float4 *>(bodies);
     p.self_ids = self_ids;
@@ -477,7 +526,7 @@ tt_status tt_traverse_bh(const tt_tree *t, const float *bodies, const int32_t *s
     p.acc = reinterpret_cast<float4 *>(acc_out);
     return finish_launch(cfg.variant == TT_VARIANT_RECURSIVE ? tt_launch_bh_recursive(p, cfg)
                          : cfg.variant == TT_VARIANT_STACK   ? tt_launch_bh_stack(p, cfg)
-                         : cfg.variant == TT_VARIANT_GROUPS  ? tt_launch_bh_group(p, t->d_grp, t->hdr.n_nodes, t->hdr.n_points, cfg)
+                         : cfg.variant == TT_VARIANT_GROUPS  ? tt_launch_bh_group(p, t->d_grp, t->hdr.n_nodes, t->hdr.n_points, wide, cfg)
                                                              : tt_launch_bh(p, cfg));  // ROPES
 }
 

@@ -7,6 +7,7 @@
 #include <cstdint>
 #include <mutex>
 
+#include <cuda_runtime_api.h>
 #include <vector_types.h>
 
 #include "../../include/tt.h"
@@ -17,6 +18,9 @@
 #define TT_TOP_BYTES (32 * 1024)  /* shared-memory budget for the staged top levels */
 #define TT_COUNTER_SLOTS 256      /* tile-scheduler counter slots per tree */
 #define TT_TOP_LEVELS_MAX 32      /* levels tracked in the header's level_prefix */
+// tt_blob_header.oct_flags (what the child-group BH walk may assume):
+#define TT_OCT_NARROW 1           /* height <= 32 and every node has <= 8 children */
+#define TT_OCT_FEW_CELL_KIDS 2    /* every node has <= 8 children that are cells    */
 
 // ---------------------------------------------------------------------------
 // Packed node records: one 32-byte sector per node, two 128-bit field groups
@@ -59,7 +63,8 @@ static_assert(sizeof(tt_nn_rec) == 16, "nn header = one 128-bit group");
 // the blob start (position independent: the blob can be broadcast as bytes).
 struct tt_blob_header {
     uint32_t magic, version;
-    int32_t kind, dim, dp, height, leaf_size, top_levels, top_count, pad0;
+    int32_t kind, dim, dp, height, leaf_size, top_levels, top_count;
+    int32_t oct_flags;  // OCT: TT_OCT_* bits below (0 for other kinds / unknown)
     // level_prefix[L] = number of nodes with level < L, for L <= top_levels; the
     // top region is numbered level by level, so its first level_prefix[L]
     // records are exactly the top L levels (each kernel stages what fits).
@@ -145,6 +150,7 @@ struct tt_tree {
     uint32_t *d_counters;  // [TT_COUNTER_SLOTS][2]
     unsigned slot_next;
     void *d_grp = nullptr;  // OCT: child-group records (kern_bh_group.cu), built on first use
+    cudaEvent_t grp_ready = nullptr;  // recorded on the stream of that build
     std::mutex grp_mu;
 };
 
@@ -169,7 +175,8 @@ int tt_launch_vp_recursive(const tt_vp_params &p, int dim, const tt_launch_cfg &
 int tt_launch_bh_stack(const tt_bh_params &p, const tt_launch_cfg &cfg);
 // lockstep walk by child groups (kern_bh_group.cu)
 int tt_bh_groups_build(const void *rec, long long nn, long long np, void *stream, void **grp_out);
-int tt_launch_bh_group(const tt_bh_params &p, const void *grp, long long nn, long long np, const tt_launch_cfg &cfg);
+int tt_launch_bh_group(const tt_bh_params &p, const void *grp, long long nn, long long np, bool wide,
+                       const tt_launch_cfg &cfg);
 int tt_launch_pc_stack(const tt_pc_params &p, int dim, const tt_launch_cfg &cfg);
 // one point's traversal split over a 16-lane group (kern_pc_split.cu)
 int tt_launch_pc_split(const tt_pc_params &p, int dim, const tt_launch_cfg &cfg);

@@ -860,3 +860,32 @@ def test_bh_groups_self_test_only_where_it_matters(case, variant):
     ref = oracle.bh(ot, q, 0.5, eps, self_ids=ids)
     assert np.isfinite(acc).all() and np.isfinite(ref.out[0]).all()
     assert rel_err(acc, ref.out[0]).max() <= BH_TOL
+
+
+@pytest.mark.parametrize("dup", [9, 40])
+@pytest.mark.parametrize("builder", ["host", "device"])
+def test_bh_groups_wide_buckets(dup, builder):
+    """A depth-32 bucket (R9) of more than 8 coincident bodies: its cell has
+    `dup` leaf children, more than the 8-record staging buffer of the
+    child-group walk, which then stages groups 8 at a time (header
+    oct_flags without TT_OCT_NARROW).  Every mode against the oracle: visits
+    exact, accelerations within 1e-4 (theta = 0.5 and theta = 0)."""
+    b = ttgen.plummer(5003, seed=320 + dup)
+    b[200:200 + dup, :3] = b[7, :3]
+    b[3000:3000 + dup, :3] = b[4000, :3]  # and a second one in another warp tile
+    ot = oracle.build_oct(b)
+    assert ot.height == 33
+    tree = P.tt_tree_upload(P.build_oct(b)) if builder == "host" else P.tt_build_oct_device(dev(b))
+    bd = dev(b)
+    for theta in (0.5, 0.0):
+        ref = oracle.bh(ot, b, theta, 0.05, self_ids=np.arange(len(b)), stats=True)
+        for mode in MODES:
+            st = P.Stats.alloc(len(b), "cuda")
+            acc = P.tt_traverse_bh(tree, bd, theta, 0.05, mode=mode, stats=st).cpu().numpy()
+            assert rel_err(acc, ref.out[0]).max() <= BH_TOL, (theta, mode)
+            assert np.array_equal(st.visits.cpu().numpy(), ref.visits), (theta, mode)
+        if theta == 0.5:
+            st = P.Stats.alloc(len(b), "cuda")
+            P.tt_traverse_bh(tree, bd, theta, 0.05, mode="lockstep", stats=st)
+            union = oracle.unguided_warp_union(ot, b, 0.5, W=32 * P._lib.BH_POINTS_PER_LANE)
+            assert np.array_equal(st.warp_fetches.cpu().numpy()[:len(union)], union)

@@ -146,7 +146,7 @@ def test_nn_blob_records_and_points():
 # ------------------------------------------------------------- blob layout
 HDR = np.dtype([("magic", "<u4"), ("version", "<u4"), ("kind", "<i4"), ("dim", "<i4"), ("dp", "<i4"),
                 ("height", "<i4"), ("leaf_size", "<i4"), ("top_levels", "<i4"), ("top_count", "<i4"),
-                ("pad0", "<i4"), ("level_prefix", "<i4", 33), ("pad1", "<i4"), ("n_nodes", "<i8"), ("n_points", "<i8"), ("root_center", "<f8", 3),
+                ("oct_flags", "<i4"), ("level_prefix", "<i4", 33), ("pad1", "<i4"), ("n_nodes", "<i8"), ("n_points", "<i8"), ("root_center", "<f8", 3),
                 ("root_side", "<f8"), ("off_rec", "<u8"), ("off_box", "<u8"), ("off_pts", "<u8"),
                 ("off_pid", "<u8"), ("off_vpt", "<u8"), ("total", "<u8"), ("rec_bytes", "<u8"), ("off_cbox", "<u8")])
 
@@ -167,6 +167,7 @@ def test_oct_blob_top_first_layout_preserves_preorder():
     hd = {k: (int(v) if np.ndim(v) == 0 else v) for k, v in
           zip(HDR.names, np.frombuffer(blob[:HDR.itemsize].tobytes(), HDR)[0])}
     assert hd["magic"] == 0x31425454 and hd["kind"] == 1 and hd["n_nodes"] == h.n_nodes
+    assert hd["oct_flags"] == 3  # NARROW | FEW_CELL_KIDS: no depth-32 bucket
     rec = np.frombuffer(blob[hd["off_rec"]:hd["off_rec"] + 32 * h.n_nodes].tobytes(),
                         dtype=[("g", "<f4", 4), ("fc", "<i4"), ("skip", "<i4"), ("body", "<i4"), ("lvl", "<i4")])
     top = hd["top_count"]
@@ -183,6 +184,20 @@ def test_oct_blob_top_first_layout_preserves_preorder():
     assert np.array_equal(rec["lvl"][seq], h.array("level"))
     assert np.array_equal(rec["body"][seq], h.array("body"))
     assert np.array_equal(rec["g"][seq], h.array("com"))
+
+
+@pytest.mark.parametrize("dup", [2, 8, 9, 40])
+def test_oct_blob_flags_for_buckets(dup):
+    """A depth-32 bucket (R9) of `dup` coincident bodies: height 33, so the
+    header says "not narrow" (the child-group walk stages its groups 8 at a
+    time); its children are leaves, so at most 8 cell children per node."""
+    b = ttgen.plummer(500, seed=106)
+    b[10:10 + dup, :3] = b[3, :3]
+    h = P.build_oct(b)
+    blob = h.pack()
+    hd = {k: (int(v) if np.ndim(v) == 0 else v) for k, v in
+          zip(HDR.names, np.frombuffer(blob[:HDR.itemsize].tobytes(), HDR)[0])}
+    assert hd["height"] == 33 and hd["oct_flags"] == 2
 
 
 def test_kd_blob_children_and_points():
