@@ -78,18 +78,18 @@ def lib():
         L.or_export_i64.argtypes = [P, I, P]
         L.or_export_f32.argtypes = [P, I, P]
         L.or_tree_order.argtypes = [P, P]
-        L.or_pc.argtypes = [P, P, I64, I, F, P, P, P, I]
+        L.or_pc.argtypes = [P, P, I64, I, F, P, P, P, P, I]
         L.or_bh_dsq_root.restype = F
         L.or_bh_dsq_root.argtypes = [P, F]
-        L.or_bh.argtypes = [P, P, P, I64, F, F, P, P, P, I]
-        L.or_knn.argtypes = [P, P, I64, I, I, P, P, P, P, I]
-        L.or_vp.argtypes = [P, P, I64, I, P, P, P, P, I]
+        L.or_bh.argtypes = [P, P, P, I64, F, F, P, P, P, P, I]
+        L.or_knn.argtypes = [P, P, I64, I, I, P, P, P, P, P, I]
+        L.or_vp.argtypes = [P, P, I64, I, P, P, P, P, P, I]
         L.or_sort_keys.argtypes = [P, P, I64, I, P, I]
         L.or_unguided_warp_union.argtypes = [P, P, I64, I, I, F, P, I]
-        L.or_knn_lockstep.argtypes = [P, P, I64, I, I, P, P, P, P, I]
-        L.or_vp_lockstep.argtypes = [P, P, I64, I, P, P, P, P, I]
-        L.or_nn.argtypes = [P, P, I64, I, P, P, P, P, I]
-        L.or_nn_lockstep.argtypes = [P, P, I64, I, P, P, P, P, I]
+        L.or_knn_lockstep.argtypes = [P, P, I64, I, I, P, P, P, P, P, P, I]
+        L.or_vp_lockstep.argtypes = [P, P, I64, I, P, P, P, P, P, P, I]
+        L.or_nn.argtypes = [P, P, I64, I, P, P, P, P, P, I]
+        L.or_nn_lockstep.argtypes = [P, P, I64, I, P, P, P, P, P, P, I]
         L.or_max_threads.restype = I
         _lib = L
     return _lib
@@ -194,7 +194,8 @@ def _threads(t):
 class Result:
     out: tuple
     visits: np.ndarray | None = None
-    hash: np.ndarray | None = None
+    hash: np.ndarray | None = None       # order-sensitive: h = h*31 + pre + 1
+    set_hash: np.ndarray | None = None   # order-insensitive: sum of mix64(pre + 1)
 
 
 def pc(tree: Tree, q: np.ndarray, radius: float, threads=None, stats=False) -> Result:
@@ -203,9 +204,10 @@ def pc(tree: Tree, q: np.ndarray, radius: float, threads=None, stats=False) -> R
     cnt = np.empty(m, np.uint32)
     v = np.empty(m, np.int64) if stats else None
     h = np.empty(m, np.uint64) if stats else None
-    rc = lib().or_pc(tree._h, _p(q), m, q.shape[1], float(radius), _p(cnt), _p(v), _p(h), _threads(threads))
+    sh = np.empty(m, np.uint64) if stats else None
+    rc = lib().or_pc(tree._h, _p(q), m, q.shape[1], float(radius), _p(cnt), _p(v), _p(h), _p(sh), _threads(threads))
     assert rc == 0
-    return Result((cnt,), v, h)
+    return Result((cnt,), v, h, sh)
 
 
 def bh_dsq_root(tree: Tree, theta: float) -> float:
@@ -220,10 +222,11 @@ def bh(tree: Tree, bodies: np.ndarray, theta: float, eps: float, self_ids=None,
     sid = None if self_ids is None else np.ascontiguousarray(self_ids, dtype=np.int64)
     v = np.empty(m, np.int64) if stats else None
     h = np.empty(m, np.uint64) if stats else None
-    rc = lib().or_bh(tree._h, _p(b), _p(sid), m, float(theta), float(eps), _p(acc), _p(v), _p(h),
+    sh = np.empty(m, np.uint64) if stats else None
+    rc = lib().or_bh(tree._h, _p(b), _p(sid), m, float(theta), float(eps), _p(acc), _p(v), _p(h), _p(sh),
                      _threads(threads))
     assert rc == 0
-    return Result((acc,), v, h)
+    return Result((acc,), v, h, sh)
 
 
 def knn(tree: Tree, q: np.ndarray, k: int, threads=None, stats=False) -> Result:
@@ -233,9 +236,10 @@ def knn(tree: Tree, q: np.ndarray, k: int, threads=None, stats=False) -> Result:
     d2 = np.empty((m, k), np.float32)
     v = np.empty(m, np.int64) if stats else None
     h = np.empty(m, np.uint64) if stats else None
-    rc = lib().or_knn(tree._h, _p(q), m, q.shape[1], k, _p(idx), _p(d2), _p(v), _p(h), _threads(threads))
+    sh = np.empty(m, np.uint64) if stats else None
+    rc = lib().or_knn(tree._h, _p(q), m, q.shape[1], k, _p(idx), _p(d2), _p(v), _p(h), _p(sh), _threads(threads))
     assert rc == 0
-    return Result((idx, d2), v, h)
+    return Result((idx, d2), v, h, sh)
 
 
 def vp(tree: Tree, q: np.ndarray, threads=None, stats=False) -> Result:
@@ -245,9 +249,10 @@ def vp(tree: Tree, q: np.ndarray, threads=None, stats=False) -> Result:
     d2 = np.empty(m, np.float32)
     v = np.empty(m, np.int64) if stats else None
     h = np.empty(m, np.uint64) if stats else None
-    rc = lib().or_vp(tree._h, _p(q), m, q.shape[1], _p(idx), _p(d2), _p(v), _p(h), _threads(threads))
+    sh = np.empty(m, np.uint64) if stats else None
+    rc = lib().or_vp(tree._h, _p(q), m, q.shape[1], _p(idx), _p(d2), _p(v), _p(h), _p(sh), _threads(threads))
     assert rc == 0
-    return Result((idx, d2), v, h)
+    return Result((idx, d2), v, h, sh)
 
 
 def nn(tree: Tree, q: np.ndarray, threads=None, stats=False) -> Result:
@@ -258,9 +263,10 @@ def nn(tree: Tree, q: np.ndarray, threads=None, stats=False) -> Result:
     d2 = np.empty(m, np.float32)
     v = np.empty(m, np.int64) if stats else None
     h = np.empty(m, np.uint64) if stats else None
-    rc = lib().or_nn(tree._h, _p(q), m, q.shape[1], _p(idx), _p(d2), _p(v), _p(h), _threads(threads))
+    sh = np.empty(m, np.uint64) if stats else None
+    rc = lib().or_nn(tree._h, _p(q), m, q.shape[1], _p(idx), _p(d2), _p(v), _p(h), _p(sh), _threads(threads))
     assert rc == 0
-    return Result((idx, d2), v, h)
+    return Result((idx, d2), v, h, sh)
 
 
 def sort_keys(tree: Tree, q: np.ndarray, threads=None) -> np.ndarray:
@@ -288,40 +294,62 @@ def unguided_warp_union(tree: Tree, pts_in_warp_order: np.ndarray, param: float,
     return out
 
 
-def knn_lockstep(tree: Tree, q: np.ndarray, k: int, threads=None):
+@dataclass
+class LockstepResult:
+    """Guided lockstep simulation (Fig.8 + the §4.3 majority vote).
+
+    out: per-lane results; lane_visits / lane_hash: nodes each lane tested
+    and their order hash; warp_tests: nodes each warp tested (pops, Table 2's
+    numerator); warp_fetches: pops with an active lane (nodes
+    expanded; reading R22)."""
+    out: tuple
+    lane_visits: np.ndarray
+    lane_hash: np.ndarray
+    warp_tests: np.ndarray
+    warp_fetches: np.ndarray
+
+    def __iter__(self):  # (idx, d2, lane_visits, warp_fetches), the round-1 tuple
+        return iter((*self.out, self.lane_visits, self.warp_fetches))
+
+    def __getitem__(self, i):
+        return tuple(self)[i]
+
+
+def _lockstep(fn, tree, q, k=None, threads=None):
     q = _f32(q)
     m = len(q)
-    idx = np.empty((m, k), np.int64)
-    d2 = np.empty((m, k), np.float32)
+    shape = (m, k) if k is not None else (m,)
+    idx = np.empty(shape, np.int64)
+    d2 = np.empty(shape, np.float32)
     lv = np.empty(m, np.int64)
-    wf = np.empty((m + 31) // 32, np.int64)
-    rc = lib().or_knn_lockstep(tree._h, _p(q), m, q.shape[1], k, _p(idx), _p(d2), _p(lv), _p(wf),
-                               _threads(threads))
+    lh = np.empty(m, np.uint64)
+    nw = (m + 31) // 32
+    wf = np.empty(nw, np.int64)
+    wt = np.empty(nw, np.int64)
+    args = [tree._h, _p(q), m, q.shape[1]] + ([k] if k is not None else [])
+    rc = fn(*args, _p(idx), _p(d2), _p(lv), _p(wf), _p(wt), _p(lh), _threads(threads))
     assert rc == 0
-    return idx, d2, lv, wf
+    return LockstepResult((idx, d2), lv, lh, wt, wf)
 
 
-def vp_lockstep(tree: Tree, q: np.ndarray, threads=None):
-    q = _f32(q)
-    m = len(q)
-    idx = np.empty(m, np.int64)
-    d2 = np.empty(m, np.float32)
-    lv = np.empty(m, np.int64)
-    wf = np.empty((m + 31) // 32, np.int64)
-    rc = lib().or_vp_lockstep(tree._h, _p(q), m, q.shape[1], _p(idx), _p(d2), _p(lv), _p(wf),
-                              _threads(threads))
-    assert rc == 0
-    return idx, d2, lv, wf
+def knn_lockstep(tree: Tree, q: np.ndarray, k: int, threads=None) -> LockstepResult:
+    return _lockstep(lib().or_knn_lockstep, tree, q, k, threads)
 
 
-def nn_lockstep(tree: Tree, q: np.ndarray, threads=None):
-    q = _f32(q)
-    m = len(q)
-    idx = np.empty(m, np.int64)
-    d2 = np.empty(m, np.float32)
-    lv = np.empty(m, np.int64)
-    wf = np.empty((m + 31) // 32, np.int64)
-    rc = lib().or_nn_lockstep(tree._h, _p(q), m, q.shape[1], _p(idx), _p(d2), _p(lv), _p(wf),
-                              _threads(threads))
-    assert rc == 0
-    return idx, d2, lv, wf
+def vp_lockstep(tree: Tree, q: np.ndarray, threads=None) -> LockstepResult:
+    return _lockstep(lib().or_vp_lockstep, tree, q, None, threads)
+
+
+def nn_lockstep(tree: Tree, q: np.ndarray, threads=None) -> LockstepResult:
+    return _lockstep(lib().or_nn_lockstep, tree, q, None, threads)
+
+
+def work_expansion(warp_nodes: np.ndarray, independent_visits: np.ndarray, W: int = 32) -> np.ndarray:
+    """Table 2's metric per warp: nodes the warp accesses in
+    the lockstep traversal / nodes of its longest non-lockstep traversal.
+    independent_visits: per-point N-mode visit counts in warp order."""
+    v = np.asarray(independent_visits, np.float64)
+    nw = len(warp_nodes)
+    pad = nw * W - len(v)
+    longest = np.concatenate([v, np.zeros(pad)]).reshape(nw, W).max(1)
+    return np.asarray(warp_nodes, np.float64) / longest
