@@ -234,6 +234,24 @@ typedef struct tt_stats {
     uint32_t *warp_steps;    /* [ceil(n/T)] loop iterations of the warp          */
     uint8_t *warp_mode;      /* [ceil(n/T)] 1 = lockstep, 2 = independent,
                                 3 = lockstep switched to independent          */
+    /* Per-point hashes of the nodes the point tested (nullable; requesting
+     * either builds, once per tree, a map from device node to canonical
+     * preorder id pre -- the numbering of tt_tree_desc):
+     *   visit_hash: h = h*31 + pre + 1 over the tested nodes in the order the
+     *     point tested them (the recursive order, §3.3, is kept by
+     *     every independent walk, the per-node lockstep BH / PC walks and the
+     *     explicit-stack variants; kNN / VP / NN lockstep lanes follow the
+     *     warp's majority-vote order, §4.3).  Written 0 for points of walks
+     *     that do not keep a per-point order: BH child-group lockstep tiles
+     *     and TT_VARIANT_SPLIT (reading R23);
+     *   visit_set: sum over the tested nodes of mix64(pre + 1) mod 2^64
+     *     (mix64 = the splitmix64 finaliser): order-insensitive, written by
+     *     every walk.                                                        */
+    uint64_t *visit_hash;    /* [n]                                              */
+    uint64_t *visit_set;     /* [n]                                              */
+    uint32_t *point_tests;   /* [n] kNN / PC: bucket points whose distance the
+                                point computed (SURVEY §8(d) kNN bytes: 16 B per
+                                inner node + 32 B per leaf point); nullable     */
 } tt_stats;
 
 typedef struct tt_traverse_opts {

@@ -59,7 +59,8 @@ class tt_tree_info(C.Structure):
 
 class tt_stats(C.Structure):
     _fields_ = [("visits", C.c_void_p), ("warp_fetches", C.c_void_p), ("warp_steps", C.c_void_p),
-                ("warp_mode", C.c_void_p)]
+                ("warp_mode", C.c_void_p), ("visit_hash", C.c_void_p), ("visit_set", C.c_void_p),
+                ("point_tests", C.c_void_p)]
 
 
 class tt_traverse_opts(C.Structure):

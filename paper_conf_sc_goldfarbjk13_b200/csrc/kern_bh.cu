@@ -15,8 +15,10 @@
 // its own traversal visits next.  The warp descends iff any
 // active lane opens the cell (__any_sync = Fig.8's warp_and of masks).
 // Each lane therefore tests exactly its own recursive visit sequence: opening
-// decisions and per-point visit counts are identical to the independent walk
-// (results differ only by the fp32->fp64 flush cadence of the accumulator).
+// decisions, per-point visit counts and visit order are identical to the
+// independent walk, and so are the results (the fp32 partials are flushed
+// into fp64 per body after every kFlush of its own visits, as the
+// independent walk does; an inactive step adds an exact +0).
 #include <cfloat>
 #include <cmath>
 
@@ -215,67 +217,96 @@ __global__ void __launch_bounds__(kBlock, 4) bh_kernel(const tt_bh_params P) {
             const float e2 = __shfl_sync(TT_FULL, eps2, 0);
             const float2 e22 = make_float2(e2, e2);
 
-            for (;;) {
-#pragma unroll 1
-                for (int k = 0; k < kFlush; ++k) {
-                    // lockstep: one warp-uniform address, served by L1 (top levels
-                    // included -- they are also at [0, top) of the global array);
-                    // measured 2.7% faster than the smem/global select here
-                    float4 g;
-                    int4 t;
-                    ldg_rec256(grec + cur, g, t);
-                    if (STATS) ++steps;
-                    const int lvl = t.w;
-                    const float dl = EXP_DSQ ? dsq_at(dbits, lvl) : s_dsq[lvl];
-                    const bool cell = t.x >= 0;
-                    bool any_open = false;
+            // fp32 partials are flushed into fp64 per BODY after every kFlush
+            // of its own visits -- the cadence of the independent walk, whose
+            // terms are the same ops in the same order (an inactive step adds
+            // an exact +0), so L and N results are bit-identical
+            unsigned fc[kBPL];
 #pragma unroll
-                    for (int p = 0; p < NP; ++p) {
-                        const float2 dx = add2_rn(make_float2(g.x, g.x), nbx[p]);
-                        const float2 dy = add2_rn(make_float2(g.y, g.y), nby[p]);
-                        const float2 dz = add2_rn(make_float2(g.z, g.z), nbz[p]);
-                        // rn(rn(rn(dx^2) + rn(dy^2)) + rn(dz^2)): the pinned order (R0)
-                        const float2 drsq = add2_rn(add2_rn(sqr2_rn(dx, nz), sqr2_rn(dy, nz)), sqr2_rn(dz, nz));
-                        const bool a0 = lvl <= w[2 * p], a1 = lvl <= w[2 * p + 1];
-                        const bool o0 = a0 && cell && drsq.x < dl;
-                        const bool o1 = a1 && cell && drsq.y < dl;
-                        if (STATS) {
-                            bd[2 * p].visits += a0;
-                            bd[2 * p + 1].visits += a1;
-                        }
-                        // active ? (open ? follow : wait at lvl) : keep -- as a min
-                        // (an inactive lane has lvl > wait)
-                        w[2 * p] = o0 ? INT_MAX : min(w[2 * p], lvl);
-                        w[2 * p + 1] = o1 ? INT_MAX : min(w[2 * p + 1], lvl);
-                        // branch-free update (some lane almost always interacts)
-                        const bool k0 = a0 && !o0 && t.z != self[2 * p];
-                        const bool k1 = a1 && !o1 && t.z != self[2 * p + 1];
-                        const float2 mw = make_float2(k0 ? g.w : 0.f, k1 ? g.w : 0.f);
-                        const float2 r = add2_rn(drsq, e22);
-                        const float2 inv = make_float2(rsqrt_ftz(r.x), rsqrt_ftz(r.y));
-                        float2 f = mul2_rn(mul2_rn(mw, mul2_rn(inv, inv)), inv);
-                        // eps = 0: a skipped term at distance 0 has inv = inf (0 * inf)
-                        f = make_float2(k0 ? f.x : 0.f, k1 ? f.y : 0.f);
-                        ax[p] = fma2_rn(f, dx, ax[p]);
-                        ay[p] = fma2_rn(f, dy, ay[p]);
-                        az[p] = fma2_rn(f, dz, az[p]);
-                        any_open = any_open || o0 || o1;
-                    }
-                    cur = __any_sync(TT_FULL, any_open) ? t.x : t.y;
-                    if (cur == TT_END) break;
-                }
-                // fp32 partials -> fp64 (warp-uniform cadence)
+            for (int j = 0; j < kBPL; ++j) fc[j] = 0;
+            VHash vh[kBPL];
+            const bool hashing = STATS && P.c.pre;
+#pragma unroll 1
+            for (;;) {
+                // lockstep: one warp-uniform address, served by L1 (top levels
+                // included -- they are also at [0, top) of the global array);
+                // measured 2.7% faster than the smem/global select here
+                float4 g;
+                int4 t;
+                ldg_rec256(grec + cur, g, t);
+                if (STATS) ++steps;
+                const int lvl = t.w;
+                const float dl = EXP_DSQ ? dsq_at(dbits, lvl) : s_dsq[lvl];
+                const bool cell = t.x >= 0;
+                bool any_open = false;
 #pragma unroll
                 for (int p = 0; p < NP; ++p) {
-                    bd[2 * p].acc.X += (double)ax[p].x;
-                    bd[2 * p].acc.Y += (double)ay[p].x;
-                    bd[2 * p].acc.Z += (double)az[p].x;
-                    bd[2 * p + 1].acc.X += (double)ax[p].y;
-                    bd[2 * p + 1].acc.Y += (double)ay[p].y;
-                    bd[2 * p + 1].acc.Z += (double)az[p].y;
-                    ax[p] = ay[p] = az[p] = make_float2(0.f, 0.f);
+                    const float2 dx = add2_rn(make_float2(g.x, g.x), nbx[p]);
+                    const float2 dy = add2_rn(make_float2(g.y, g.y), nby[p]);
+                    const float2 dz = add2_rn(make_float2(g.z, g.z), nbz[p]);
+                    // rn(rn(rn(dx^2) + rn(dy^2)) + rn(dz^2)): the pinned order (R0)
+                    const float2 drsq = add2_rn(add2_rn(sqr2_rn(dx, nz), sqr2_rn(dy, nz)), sqr2_rn(dz, nz));
+                    const bool a0 = lvl <= w[2 * p], a1 = lvl <= w[2 * p + 1];
+                    const bool o0 = a0 && cell && drsq.x < dl;
+                    const bool o1 = a1 && cell && drsq.y < dl;
+                    if (STATS) {
+                        bd[2 * p].visits += a0;
+                        bd[2 * p + 1].visits += a1;
+                        if (hashing) {
+                            vh[2 * p].add_if(a0, P.c.pre, cur);
+                            vh[2 * p + 1].add_if(a1, P.c.pre, cur);
+                        }
+                    }
+                    // active ? (open ? follow : wait at lvl) : keep -- as a min
+                    // (an inactive lane has lvl > wait)
+                    w[2 * p] = o0 ? INT_MAX : min(w[2 * p], lvl);
+                    w[2 * p + 1] = o1 ? INT_MAX : min(w[2 * p + 1], lvl);
+                    // branch-free update (some lane almost always interacts)
+                    const bool k0 = a0 && !o0 && t.z != self[2 * p];
+                    const bool k1 = a1 && !o1 && t.z != self[2 * p + 1];
+                    const float2 mw = make_float2(k0 ? g.w : 0.f, k1 ? g.w : 0.f);
+                    const float2 r = add2_rn(drsq, e22);
+                    const float2 inv = make_float2(rsqrt_ftz(r.x), rsqrt_ftz(r.y));
+                    float2 f = mul2_rn(mul2_rn(mw, mul2_rn(inv, inv)), inv);
+                    // eps = 0: a skipped term at distance 0 has inv = inf (0 * inf)
+                    f = make_float2(k0 ? f.x : 0.f, k1 ? f.y : 0.f);
+                    ax[p] = fma2_rn(f, dx, ax[p]);
+                    ay[p] = fma2_rn(f, dy, ay[p]);
+                    az[p] = fma2_rn(f, dz, az[p]);
+                    any_open = any_open || o0 || o1;
+                    fc[2 * p] += a0;
+                    fc[2 * p + 1] += a1;
+                    if (fc[2 * p] == kFlush) {
+                        bd[2 * p].acc.X += (double)ax[p].x;
+                        bd[2 * p].acc.Y += (double)ay[p].x;
+                        bd[2 * p].acc.Z += (double)az[p].x;
+                        ax[p].x = ay[p].x = az[p].x = 0.f;
+                        fc[2 * p] = 0;
+                    }
+                    if (fc[2 * p + 1] == kFlush) {
+                        bd[2 * p + 1].acc.X += (double)ax[p].y;
+                        bd[2 * p + 1].acc.Y += (double)ay[p].y;
+                        bd[2 * p + 1].acc.Z += (double)az[p].y;
+                        ax[p].y = ay[p].y = az[p].y = 0.f;
+                        fc[2 * p + 1] = 0;
+                    }
                 }
+                cur = __any_sync(TT_FULL, any_open) ? t.x : t.y;
                 if (cur == TT_END) break;
+            }
+#pragma unroll
+            for (int p = 0; p < NP; ++p) {
+                bd[2 * p].acc.X += (double)ax[p].x;
+                bd[2 * p].acc.Y += (double)ay[p].x;
+                bd[2 * p].acc.Z += (double)az[p].x;
+                bd[2 * p + 1].acc.X += (double)ax[p].y;
+                bd[2 * p + 1].acc.Y += (double)ay[p].y;
+                bd[2 * p + 1].acc.Z += (double)az[p].y;
+            }
+            if (hashing) {
+#pragma unroll
+                for (int j = 0; j < kBPL; ++j)
+                    if (bd[j].valid) vh[j].store(P.c, bd[j].pid);
             }
 
             fetches = steps;
@@ -283,13 +314,17 @@ __global__ void __launch_bounds__(kBlock, 4) bh_kernel(const tt_bh_params P) {
 #pragma unroll
             for (int j = 0; j < kBPL; ++j) {
                 int cur = bd[j].valid ? 0 : TT_END;
+                VHash vh;
                 while (cur != TT_END) {
 #pragma unroll 1
                     for (int k = 0; k < kFlush; ++k) {
                         float4 g;
                         int4 t;
                         ld_rec(s_base, g_base, top, cur, g, t);
-                        if (STATS) ++bd[j].visits;
+                        if (STATS) {
+                            ++bd[j].visits;
+                            if (P.c.pre) vh.add(P.c.pre, cur);
+                        }
                         float dx, dy, sx, sy;
                         sub2_rn(g.x, g.y, bd[j].b.x, bd[j].b.y, dx, dy);
                         sqr2_rn(dx, dy, sx, sy);
@@ -306,6 +341,7 @@ __global__ void __launch_bounds__(kBlock, 4) bh_kernel(const tt_bh_params P) {
                     }
                     bd[j].acc.flush();
                 }
+                if (STATS && P.c.pre && bd[j].valid) vh.store(P.c, bd[j].pid);
             }
             if (STATS) {
                 unsigned v = 0, mx = 0;
@@ -358,7 +394,7 @@ int launch(const tt_bh_params &p, const tt_launch_cfg &cfg) {
 }  // namespace
 
 int tt_launch_bh(const tt_bh_params &p, const tt_launch_cfg &cfg) {
-    const bool stats = p.c.st_visits || p.c.st_warp_fetches || p.c.st_warp_steps || p.c.st_warp_mode;
+    const bool stats = stats_on(p.c);
     // exponent-arithmetic dsq is exact iff dsq_root * 0.25^height is a normal float
     // (or dsq_root = +inf, theta = 0); otherwise use the shared-memory table
     const float r = p.dsq_root;

@@ -65,7 +65,7 @@ __global__ void nkids_kernel(const tt_oct_rec *rec, long long nn, int *nk) {
 }
 
 __global__ void groups_fill_kernel(const tt_oct_rec *rec, long long nn, const int *nk, const int *goff,
-                                   tt_oct_rec *grp, int *leaf_of, long long np) {
+                                   tt_oct_rec *grp, int *leaf_of, long long np, int *gsrc) {
     for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < nn; v += (long long)gridDim.x * blockDim.x) {
         if (v == 0) {  // the root's own entry
             tt_oct_rec r = rec[0];
@@ -73,6 +73,7 @@ __global__ void groups_fill_kernel(const tt_oct_rec *rec, long long nn, const in
             r.skip = nk[0];
             r.level <<= 24;
             grp[0] = r;
+            gsrc[0] = 0;
             if (r.first_child < 0 && r.body >= 0 && r.body < np) leaf_of[r.body] = 0;
         }
         int c = rec[v].first_child, k = 0;
@@ -83,6 +84,7 @@ __global__ void groups_fill_kernel(const tt_oct_rec *rec, long long nn, const in
             r.skip = nk[c];
             r.level <<= 24;  // the exponent step of dsq_L (level * 2^24): one IADD per child
             grp[1 + goff[v] + k] = r;
+            gsrc[1 + goff[v] + k] = c;  // the device node (stats hashes map it to its preorder id)
             if (r.first_child < 0 && r.body >= 0 && r.body < np) leaf_of[r.body] = 1 + goff[v] + k;
             ++k;
             c = rec[c].skip;
@@ -99,7 +101,8 @@ __device__ __forceinline__ float dsq_at(int dsq_bits, int lvl) { return __int_as
 // coincident bodies, R9, or a custom tree): groups are staged 8 at a time.
 template <bool STATS, bool EXP_DSQ, bool WIDE>
 __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_bh_params P, const tt_oct_rec *grp,
-                                                                                 const int *leaf_of, long long np) {
+                                                                                 const int *leaf_of, long long np,
+                                                                                 const int *gsrc) {
     extern __shared__ __align__(128) unsigned char smem[];
     float *s_dsq = reinterpret_cast<float *>(smem + 16);
     GroupEntry *s_stack = reinterpret_cast<GroupEntry *>(smem + kSmemHdr);
@@ -175,6 +178,8 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
             visits[j] = 0;
         }
         unsigned fetches = 0, steps = 0;
+        VHash vh[kBPL];
+        const bool hashing = STATS && P.c.pre;
         // The self test (skip the leaf holding the body itself) only
         // matters where that leaf's term is not exactly zero: a leaf at
         // the body's own position contributes f * 0 = 0 whenever f is
@@ -241,6 +246,14 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                             ++steps;
                             visits[0] += in0;
                             visits[1] += in1;
+                            if (hashing && (in0 || in1)) {
+                                // the visited SET only: a body's tests are in DFS-over-
+                                // groups order, not the recursive order (reading R23)
+                                const unsigned long long m = vh_mix64(
+                                    (unsigned long long)(unsigned)__ldg(P.c.pre + __ldg(gsrc + goff + c0 + k)) + 1ull);
+                                if (in0) vh[0].s += m;
+                                if (in1) vh[1].s += m;
+                            }
                         }
                         const float dl = EXP_DSQ ? __int_as_float(dsq_bits - t.w) : s_dsq[t.w >> 24];
                         const float2 dx = add2_rn(make_float2(g.x, g.x), nbx);
@@ -315,7 +328,10 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                     float4 g;
                     int4 t;
                     ldg_rec256(g_rec + cur, g, t);
-                    if (STATS) ++visits[j];
+                    if (STATS) {
+                        ++visits[j];
+                        if (hashing) vh[j].add(P.c.pre, cur);
+                    }
                     const float dx = __fsub_rn(g.x, b[j].x), dy = __fsub_rn(g.y, b[j].y),
                                 dz = __fsub_rn(g.z, b[j].z);
                     const float drsq = __fadd_rn(__fadd_rn(__fmul_rn(dx, dx), __fmul_rn(dy, dy)), __fmul_rn(dz, dz));
@@ -349,6 +365,7 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
             if (valid[j]) {
                 P.acc[pid[j]] = make_float4((float)X[j], (float)Y[j], (float)Z[j], 0.f);
                 if (STATS && P.c.st_visits) P.c.st_visits[pid[j]] = visits[j];
+                if (hashing) vh[j].store(P.c, pid[j], !lock);  // lockstep: set only
             }
         }
         if (STATS) write_warp_stats(P.c, tile, fetches, steps, lock);
@@ -358,7 +375,8 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
 }
 
 template <bool STATS, bool EXP_DSQ, bool WIDE>
-int launch(const tt_bh_params &p, const tt_oct_rec *grp, const int *leaf_of, long long np, const tt_launch_cfg &cfg) {
+int launch(const tt_bh_params &p, const tt_oct_rec *grp, const int *leaf_of, long long np, const int *gsrc,
+           const tt_launch_cfg &cfg) {
     const size_t smem = kSmemHdr + (size_t)(kBlock / 32) * kStackPerWarp * sizeof(GroupEntry) + (kBlock / 32) * 16 * 16;
     auto kern = bh_group_kernel<STATS, EXP_DSQ, WIDE>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -375,7 +393,7 @@ int launch(const tt_bh_params &p, const tt_oct_rec *grp, const int *leaf_of, lon
     const long long need = (ntiles + kBlock / 32 - 1) / (kBlock / 32);
     if (grid > need) grid = need;
     if (grid < 1) grid = 1;
-    kern<<<(unsigned)grid, kBlock, smem, (cudaStream_t)cfg.stream>>>(p, grp, leaf_of, np);
+    kern<<<(unsigned)grid, kBlock, smem, (cudaStream_t)cfg.stream>>>(p, grp, leaf_of, np, gsrc);
     return (int)cudaGetLastError();
 }
 
@@ -449,8 +467,9 @@ int tt_bh_groups_build(const void *rec, long long nn, long long np, void *stream
     if (!e) e = cudaMallocAsync(&tmp, tb, s);
     if (!e) {
         // records, then leaf_of[np]: the group index of the leaf whose body
-        // is each id (-1 for ids no leaf names first)
-        grp = grp_take(sizeof(tt_oct_rec) * (size_t)nn + sizeof(int) * (size_t)np);
+        // is each id (-1 for ids no leaf names first), then gsrc[nn]: the
+        // device node of each group entry
+        grp = grp_take(sizeof(tt_oct_rec) * (size_t)nn + sizeof(int) * (size_t)np + sizeof(int) * (size_t)nn);
         if (!grp) e = cudaErrorMemoryAllocation;
     }
     int *leaf_of = grp ? reinterpret_cast<int *>(static_cast<tt_oct_rec *>(grp) + nn) : nullptr;
@@ -461,7 +480,8 @@ int tt_bh_groups_build(const void *rec, long long nn, long long np, void *stream
         e = cub::DeviceScan::ExclusiveSum(tmp, tb, nk, goff, (int)nn, s);
     }
     if (!e) {
-        groups_fill_kernel<<<G, 256, 0, s>>>(r, nn, nk, goff, static_cast<tt_oct_rec *>(grp), leaf_of, np);
+        groups_fill_kernel<<<G, 256, 0, s>>>(r, nn, nk, goff, static_cast<tt_oct_rec *>(grp), leaf_of, np,
+                                             leaf_of + np);
         e = cudaGetLastError();
     }
     if (tmp) cudaFreeAsync(tmp, s);
@@ -480,15 +500,16 @@ int tt_bh_groups_build(const void *rec, long long nn, long long np, void *stream
 
 int tt_launch_bh_group(const tt_bh_params &p, const void *grp, long long nn, long long np, bool wide,
                        const tt_launch_cfg &cfg) {
-    const bool stats = p.c.st_visits || p.c.st_warp_fetches || p.c.st_warp_steps || p.c.st_warp_mode;
+    const bool stats = stats_on(p.c);
     const float r = p.dsq_root;
     const bool exp_ok = r < INFINITY && r > 0.f && std::ldexp((double)r, -2 * p.c.height) >= (double)FLT_MIN;
     const tt_oct_rec *g = static_cast<const tt_oct_rec *>(grp);
     const int *lf = reinterpret_cast<const int *>(g + nn);
+    const int *gs = lf + np;
     if (wide) {  // rare (buckets of > 8 coincident bodies): no specialisations beyond stats
-        if (stats) return launch<true, false, true>(p, g, lf, np, cfg);
-        return launch<false, false, true>(p, g, lf, np, cfg);
+        if (stats) return launch<true, false, true>(p, g, lf, np, gs, cfg);
+        return launch<false, false, true>(p, g, lf, np, gs, cfg);
     }
-    if (stats) return exp_ok ? launch<true, true, false>(p, g, lf, np, cfg) : launch<true, false, false>(p, g, lf, np, cfg);
-    return exp_ok ? launch<false, true, false>(p, g, lf, np, cfg) : launch<false, false, false>(p, g, lf, np, cfg);
+    if (stats) return exp_ok ? launch<true, true, false>(p, g, lf, np, gs, cfg) : launch<true, false, false>(p, g, lf, np, gs, cfg);
+    return exp_ok ? launch<false, true, false>(p, g, lf, np, gs, cfg) : launch<false, false, false>(p, g, lf, np, gs, cfg);
 }

@@ -316,6 +316,44 @@ __device__ __forceinline__ int warp_key_changes(unsigned long long key, bool val
 
 __device__ __forceinline__ unsigned warp_sum(unsigned v) { return __reduce_add_sync(TT_FULL, v); }
 
+// any stats array requested -> the STATS instantiation
+inline bool stats_on(const tt_common_params &c) {
+    return c.st_visits || c.st_warp_fetches || c.st_warp_steps || c.st_warp_mode || c.st_hash || c.st_set ||
+           c.st_point_tests;
+}
+
+// Per-point visit hashes (tt_stats.visit_hash / visit_set): the order hash
+// h = h*31 + pre + 1 over the nodes the point tests, in the order it tests
+// them (autoropes keep the recursive order, §3.3), and the set
+// hash s = sum of mix64(pre + 1) (mix64 = the splitmix64 finaliser), where
+// pre is the node's canonical preorder id.  Only the STATS instantiations
+// compute them, and only when the caller asked (c.pre != nullptr).
+__device__ __forceinline__ unsigned long long vh_mix64(unsigned long long z) {
+    z ^= z >> 30;
+    z *= 0xbf58476d1ce4e5b9ull;
+    z ^= z >> 27;
+    z *= 0x94d049bb133111ebull;
+    z ^= z >> 31;
+    return z;
+}
+struct VHash {
+    unsigned long long h = 0, s = 0;
+    __device__ __forceinline__ void add(const int32_t *pre, int node) {
+        const unsigned long long v = (unsigned long long)(unsigned)__ldg(pre + node) + 1ull;
+        h = h * 31ull + v;
+        s += vh_mix64(v);
+    }
+    __device__ __forceinline__ void add_if(bool on, const int32_t *pre, int node) {
+        if (on) add(pre, node);
+    }
+    // order = false: the walk keeps the visited set but not the order (the
+    // order slot is written 0)
+    __device__ __forceinline__ void store(const tt_common_params &c, long long pid, bool order = true) const {
+        if (c.st_hash) c.st_hash[pid] = order ? h : 0ull;
+        if (c.st_set) c.st_set[pid] = s;
+    }
+};
+
 // Stats writer for the warp tile (lane 0).
 __device__ __forceinline__ void write_warp_stats(const tt_common_params &c, long long tile, unsigned fetches,
                                                  unsigned steps, bool lock, bool switched = false) {

@@ -196,7 +196,9 @@ __global__ void __launch_bounds__(kBlock, TT_KNN_MINB) knn_kernel(const tt_knn_p
 
         KBest<KT> kb;
         kb.init(k);
-        unsigned visits = 0, fetches = 0, steps = 0;
+        unsigned visits = 0, fetches = 0, steps = 0, ptests = 0;
+        VHash vh;
+        const bool hashing = STATS && P.c.pre;
         // independent-walk state: the whole tile (N mode), or the rest of it
         // after a dynamic L->N switch
         int n_sp = 0;
@@ -215,6 +217,7 @@ __global__ void __launch_bounds__(kBlock, TT_KNN_MINB) knn_kernel(const tt_knn_p
                 if (STATS) {
                     ++steps;
                     visits += in;
+                    if (hashing) vh.add_if(in, P.c.pre, cur);
                 }
                 const bool active = in && !(kb.worst() < INF && lb > kb.worst());
                 const unsigned act = __ballot_sync(TT_FULL, active);
@@ -256,7 +259,14 @@ __global__ void __launch_bounds__(kBlock, TT_KNN_MINB) knn_kernel(const tt_knn_p
                     if (in) {
                         n_cur = cur;
                         n_lb = lb;
-                        if (STATS) --visits;
+                        if (STATS) {
+                            --visits;
+                            if (hashing) {  // the N loop re-takes this test: undo its hash step
+                                const unsigned long long v = (unsigned long long)(unsigned)__ldg(P.c.pre + cur) + 1ull;
+                                vh.h = (vh.h - v) * 0xef7bdef7bdef7bdfull;  // * 31^-1 mod 2^64
+                                vh.s -= vh_mix64(v);
+                            }
+                        }
                     } else if (n_sp > 0) {
                         --n_sp;
                         n_cur = n_node[n_sp * 32 + lane];
@@ -273,7 +283,10 @@ __global__ void __launch_bounds__(kBlock, TT_KNN_MINB) knn_kernel(const tt_knn_p
                     int4 t, u;
                     ld_rec(s_rec, g_rec, top, cur, t, u);
                     if (t.x < 0) {
-                        if (active) leaf_update<DIM, KT>(P, u.z, u.w, DP, q, kb);
+                        if (active) {
+                            leaf_update<DIM, KT>(P, u.z, u.w, DP, q, kb);
+                            if (STATS) ptests += (unsigned)u.w;
+                        }
                     } else {
                         float lbl, lbr;
                         child_lbs<DIM>(s_cbox, g_cbox, DP, top, cur, q, lbl, lbr);
@@ -314,12 +327,16 @@ __global__ void __launch_bounds__(kBlock, TT_KNN_MINB) knn_kernel(const tt_knn_p
             int cur = n_cur;
             float lb = n_lb;
             while (cur != TT_END) {
-                if (STATS) ++visits;
+                if (STATS) {
+                    ++visits;
+                    if (hashing) vh.add(P.c.pre, cur);
+                }
                 if (!(kb.worst() < INF && lb > kb.worst())) {  // can_correlate
                     int4 t, u;
                     ld_rec(s_rec, g_rec, top, cur, t, u);
                     if (t.x < 0) {
                         leaf_update<DIM, KT>(P, u.z, u.w, DP, q, kb);
+                        if (STATS) ptests += (unsigned)u.w;
                     } else {
                         float lbl, lbr;
                         child_lbs<DIM>(s_cbox, g_cbox, DP, top, cur, q, lbl, lbr);
@@ -358,6 +375,8 @@ __global__ void __launch_bounds__(kBlock, TT_KNN_MINB) knn_kernel(const tt_knn_p
                 }
             }
             if (STATS && P.c.st_visits) P.c.st_visits[pid] = visits;
+            if (STATS && P.c.st_point_tests) P.c.st_point_tests[pid] = ptests;
+            if (hashing) vh.store(P.c, pid);
         }
         if (STATS) write_warp_stats(P.c, tile, fetches, steps, lock, lock && run_n);
         __syncwarp();
@@ -401,7 +420,7 @@ int launch(const tt_knn_params &p, const tt_launch_cfg &cfg) {
 
 template <int DIM, int KT>
 int launch_k(const tt_knn_params &p, const tt_launch_cfg &cfg) {
-    const bool stats = p.c.st_visits || p.c.st_warp_fetches || p.c.st_warp_steps || p.c.st_warp_mode;
+    const bool stats = stats_on(p.c);
     return stats ? launch<DIM, KT, true>(p, cfg) : launch<DIM, KT, false>(p, cfg);
 }
 

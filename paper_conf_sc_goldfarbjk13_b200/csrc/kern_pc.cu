@@ -101,7 +101,9 @@ __global__ void __launch_bounds__(kBlock) pc_kernel(const tt_pc_params P) {
             lock = P.c.auto_min_depth < 64 && warp_key_changes(code << (maxl - lv), valid) < kAutoMaxChanges;
         }
 
-        unsigned count = 0, visits = 0, fetches = 0, steps = 0;
+        unsigned count = 0, visits = 0, fetches = 0, steps = 0, ptests = 0;
+        VHash vh;
+        const bool hashing = STATS && P.c.pre;
         if (lock) {
             int wait = valid ? INT_MAX : -1;
             int cur = 0;
@@ -112,11 +114,15 @@ __global__ void __launch_bounds__(kBlock) pc_kernel(const tt_pc_params P) {
                 const bool active = nd.t.w <= wait;
                 bool descend = false;
                 if (active) {
-                    if (STATS) ++visits;
+                    if (STATS) {
+                        ++visits;
+                        if (hashing) vh.add(P.c.pre, cur);
+                    }
                     if (pinned_boxd2<DIM>(q, nd.lo, nd.hi) > P.r2) {
                         wait = nd.t.w;                       // !can_correlate: truncate
                     } else if (nd.t.x < 0) {
                         count += leaf_count<DIM>(P, g_rec, cur, q, DP);  // update_correlation
+                        if (STATS) ptests += (unsigned)__ldg(&g_rec[cur].pcount);
                         wait = nd.t.w;
                     } else {
                         descend = true;
@@ -131,11 +137,18 @@ __global__ void __launch_bounds__(kBlock) pc_kernel(const tt_pc_params P) {
             while (cur != TT_END) {
                 PcNode<DIM> nd;
                 ld_node<DIM>(s_rec, s_box, g_rec, g_box, DP, top, cur, nd);
-                if (STATS) ++visits;
+                if (STATS) {
+                    ++visits;
+                    if (hashing) vh.add(P.c.pre, cur);
+                }
                 bool descend = false;
                 if (pinned_boxd2<DIM>(q, nd.lo, nd.hi) <= P.r2) {
-                    if (nd.t.x < 0) count += leaf_count<DIM>(P, g_rec, cur, q, DP);
-                    else descend = true;
+                    if (nd.t.x < 0) {
+                        count += leaf_count<DIM>(P, g_rec, cur, q, DP);
+                        if (STATS) ptests += (unsigned)__ldg(&g_rec[cur].pcount);
+                    } else {
+                        descend = true;
+                    }
                 }
                 cur = descend ? nd.t.x : nd.t.z;
             }
@@ -147,6 +160,8 @@ __global__ void __launch_bounds__(kBlock) pc_kernel(const tt_pc_params P) {
         if (valid) {
             P.count[pid] = count;
             if (STATS && P.c.st_visits) P.c.st_visits[pid] = visits;
+            if (STATS && P.c.st_point_tests) P.c.st_point_tests[pid] = ptests;
+            if (hashing) vh.store(P.c, pid);
         }
         if (STATS) write_warp_stats(P.c, tile, fetches, steps, lock);
     }
@@ -178,7 +193,7 @@ int launch(const tt_pc_params &p, const tt_launch_cfg &cfg) {
 
 template <int DIM>
 int launch_dim(const tt_pc_params &p, const tt_launch_cfg &cfg) {
-    const bool stats = p.c.st_visits || p.c.st_warp_fetches || p.c.st_warp_steps || p.c.st_warp_mode;
+    const bool stats = stats_on(p.c);
     return stats ? launch<DIM, true>(p, cfg) : launch<DIM, false>(p, cfg);
 }
 

@@ -88,7 +88,9 @@ __global__ void __launch_bounds__(kBlock) pc_split_kernel(const tt_pc_params P) 
 #pragma unroll
             for (int d = 0; d < DIM; ++d) q[d] = 0.f;
 
-        unsigned count = 0, visits = 0;
+        unsigned count = 0, visits = 0, ptests = 0;
+        unsigned long long vset = 0;  // set hash only: the lanes split the walk (reading R23)
+        const bool hashing = STATS && P.c.pre;
         int cur = valid ? 0 : TT_END;
         // the top kSplitLevels levels along the bits of `sub`
 #pragma unroll
@@ -98,11 +100,17 @@ __global__ void __launch_bounds__(kBlock) pc_split_kernel(const tt_pc_params P) 
             int4 t;
             float lo[DIM], hi[DIM];
             ld_node<DIM>(s_rec, s_box, g_rec, g_box, DP, top, cur, t, lo, hi);
-            if (STATS && rep) ++visits;
+            if (STATS && rep) {
+                ++visits;
+                if (hashing) vset += vh_mix64((unsigned long long)(unsigned)__ldg(P.c.pre + cur) + 1ull);
+            }
             if (pinned_boxd2<DIM>(q, lo, hi) > P.r2) {
                 cur = TT_END;                                    // !can_correlate
             } else if (t.x < 0) {
-                if (rep) count += leaf_count<DIM>(P, g_rec, cur, q, DP);
+                if (rep) {
+                    count += leaf_count<DIM>(P, g_rec, cur, q, DP);
+                    if (STATS) ptests += (unsigned)__ldg(&g_rec[cur].pcount);
+                }
                 cur = TT_END;
             } else {
                 cur = ((sub >> (kSplitLevels - 1 - l)) & 1) ? t.y : t.x;
@@ -115,11 +123,18 @@ __global__ void __launch_bounds__(kBlock) pc_split_kernel(const tt_pc_params P) 
                 int4 t;
                 float lo[DIM], hi[DIM];
                 ld_node<DIM>(s_rec, s_box, g_rec, g_box, DP, top, cur, t, lo, hi);
-                if (STATS) ++visits;
+                if (STATS) {
+                    ++visits;
+                    if (hashing) vset += vh_mix64((unsigned long long)(unsigned)__ldg(P.c.pre + cur) + 1ull);
+                }
                 bool descend = false;
                 if (pinned_boxd2<DIM>(q, lo, hi) <= P.r2) {
-                    if (t.x < 0) count += leaf_count<DIM>(P, g_rec, cur, q, DP);
-                    else descend = true;
+                    if (t.x < 0) {
+                        count += leaf_count<DIM>(P, g_rec, cur, q, DP);
+                        if (STATS) ptests += (unsigned)__ldg(&g_rec[cur].pcount);
+                    } else {
+                        descend = true;
+                    }
                 }
                 cur = descend ? t.x : t.z;
             }
@@ -128,11 +143,20 @@ __global__ void __launch_bounds__(kBlock) pc_split_kernel(const tt_pc_params P) 
 #pragma unroll
         for (int o = kGroup / 2; o > 0; o >>= 1) {
             count += __shfl_xor_sync(TT_FULL, count, o);
-            if (STATS) visits += __shfl_xor_sync(TT_FULL, visits, o);
+            if (STATS) {
+                visits += __shfl_xor_sync(TT_FULL, visits, o);
+                ptests += __shfl_xor_sync(TT_FULL, ptests, o);
+                vset += __shfl_xor_sync(TT_FULL, vset, o);
+            }
         }
         if (valid && sub == 0) {
             P.count[pid] = count;
             if (STATS && P.c.st_visits) P.c.st_visits[pid] = visits;
+            if (STATS && P.c.st_point_tests) P.c.st_point_tests[pid] = ptests;
+            if (hashing) {
+                if (P.c.st_hash) P.c.st_hash[pid] = 0ull;  // no per-point order
+                if (P.c.st_set) P.c.st_set[pid] = vset;
+            }
         }
     }
     cta_finish(P.c.counter);
@@ -163,7 +187,7 @@ int launch(const tt_pc_params &p, const tt_launch_cfg &cfg) {
 
 template <int DIM>
 int launch_dim(const tt_pc_params &p, const tt_launch_cfg &cfg) {
-    return p.c.st_visits ? launch<DIM, true>(p, cfg) : launch<DIM, false>(p, cfg);
+    return stats_on(p.c) ? launch<DIM, true>(p, cfg) : launch<DIM, false>(p, cfg);
 }
 
 }  // namespace

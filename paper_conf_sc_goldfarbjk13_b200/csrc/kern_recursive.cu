@@ -32,10 +32,13 @@ struct BhCtx {
     float eps2;
     double ax, ay, az;
     unsigned visits;
+    const int32_t *pre;  // stats hashes (nullable)
+    VHash vh;
 };
 
 __device__ void bh_rec(BhCtx &c, int node, float dsq) {
     ++c.visits;
+    if (c.pre) c.vh.add(c.pre, node);
     const float4 g = __ldg(reinterpret_cast<const float4 *>(&c.rec[node].gx));
     const int4 t = __ldg(reinterpret_cast<const int4 *>(&c.rec[node].first_child));
     const float dx = __fsub_rn(g.x, c.b.x), dy = __fsub_rn(g.y, c.b.y), dz = __fsub_rn(g.z, c.b.z);
@@ -59,10 +62,12 @@ __global__ void __launch_bounds__(kBlock) bh_rec_kernel(const tt_bh_params P) {
     for (long long pos = blockIdx.x * (long long)blockDim.x + threadIdx.x; pos < P.c.n;
          pos += (long long)gridDim.x * blockDim.x) {
         const long long pid = P.c.order ? (long long)P.c.order[pos] : pos;
-        BhCtx c{rec, __ldg(P.bodies + pid), P.self_ids ? tt_self_id(__ldg(P.self_ids + pid)) : (int)pid, P.eps2, 0, 0, 0, 0};
+        BhCtx c{rec, __ldg(P.bodies + pid), P.self_ids ? tt_self_id(__ldg(P.self_ids + pid)) : (int)pid, P.eps2, 0, 0, 0, 0,
+                P.c.pre, VHash{}};
         bh_rec(c, 0, P.dsq_root);
         P.acc[pid] = make_float4((float)c.ax, (float)c.ay, (float)c.az, 0.f);
         if (P.c.st_visits) P.c.st_visits[pid] = c.visits;
+        if (c.pre) c.vh.store(P.c, pid);
     }
 }
 
@@ -74,12 +79,15 @@ struct PcCtx {
     int dp;
     float q[DIM];
     float r2;
-    unsigned count, visits;
+    unsigned count, visits, ptests;
+    const int32_t *pre;
+    VHash vh;
 };
 
 template <int DIM>
 __device__ void pc_rec(PcCtx<DIM> &c, int node) {
     ++c.visits;
+    if (c.pre) c.vh.add(c.pre, node);
     float lo[DIM], hi[DIM];
     load_row_nc<DIM>(lo, c.box + (size_t)node * 2 * c.dp);
     load_row_nc<DIM>(hi, c.box + (size_t)node * 2 * c.dp + c.dp);
@@ -87,6 +95,7 @@ __device__ void pc_rec(PcCtx<DIM> &c, int node) {
     const int4 t = __ldg(reinterpret_cast<const int4 *>(c.rec + node));
     if (t.x < 0) {  // update_correlation
         const int4 u = __ldg(reinterpret_cast<const int4 *>(c.rec + node) + 1);
+        c.ptests += (unsigned)u.w;
         if (u.w == 1) {
             ++c.count;
         } else {
@@ -114,10 +123,14 @@ __global__ void __launch_bounds__(kBlock) pc_rec_kernel(const tt_pc_params P) {
         c.dp = (DIM + 3) & ~3;
         load_query<DIM>(c.q, P.q, pid, P.ld);
         c.r2 = P.r2;
-        c.count = c.visits = 0;
+        c.count = c.visits = c.ptests = 0;
+        c.pre = P.c.pre;
+        c.vh = VHash{};
         pc_rec<DIM>(c, 0);
         P.count[pid] = c.count;
         if (P.c.st_visits) P.c.st_visits[pid] = c.visits;
+        if (P.c.st_point_tests) P.c.st_point_tests[pid] = c.ptests;
+        if (c.pre) c.vh.store(P.c, pid);
     }
 }
 
@@ -131,7 +144,9 @@ struct KnnCtx {
     float q[DIM];
     float d[KT];
     unsigned i[KT];
-    unsigned visits;
+    unsigned visits, ptests;
+    const int32_t *pre;
+    VHash vh;
     __device__ void insert(float dd, unsigned ii) {
         d[KT - 1] = dd;
         i[KT - 1] = ii;
@@ -153,6 +168,7 @@ struct KnnCtx {
 template <int DIM, int KT>
 __device__ void knn_rec(KnnCtx<DIM, KT> &c, int node) {
     ++c.visits;
+    if (c.pre) c.vh.add(c.pre, node);
     if (c.d[KT - 1] < __int_as_float(0x7f800000)) {  // list full: can_correlate (R5a)
         float lo[DIM], hi[DIM];
         load_row_nc<DIM>(lo, c.box + (size_t)node * 2 * c.dp);
@@ -162,6 +178,7 @@ __device__ void knn_rec(KnnCtx<DIM, KT> &c, int node) {
     const int4 t = __ldg(reinterpret_cast<const int4 *>(c.rec + node));
     const int4 u = __ldg(reinterpret_cast<const int4 *>(c.rec + node) + 1);
     if (t.x < 0) {  // update_closest
+        c.ptests += (unsigned)u.w;
         for (int j = u.z; j < u.z + u.w; ++j) {
             float p[DIM];
             load_row_nc<DIM>(p, c.pts + (size_t)j * c.dp);
@@ -197,7 +214,9 @@ __global__ void __launch_bounds__(kBlock) knn_rec_kernel(const tt_knn_params P) 
             c.d[j] = j >= KT - P.k ? __int_as_float(0x7f800000) : __int_as_float(0xff800000);
             c.i[j] = 0xffffffffu;
         }
-        c.visits = 0;
+        c.visits = c.ptests = 0;
+        c.pre = P.c.pre;
+        c.vh = VHash{};
         knn_rec<DIM, KT>(c, 0);
         for (int j = KT - P.k; j < KT; ++j) {
             const int slot = j - (KT - P.k);
@@ -205,6 +224,8 @@ __global__ void __launch_bounds__(kBlock) knn_rec_kernel(const tt_knn_params P) 
             P.d2[pid * P.k + slot] = c.d[j];
         }
         if (P.c.st_visits) P.c.st_visits[pid] = c.visits;
+        if (P.c.st_point_tests) P.c.st_point_tests[pid] = c.ptests;
+        if (c.pre) c.vh.store(P.c, pid);
     }
 }
 
@@ -217,11 +238,14 @@ struct VpCtx {
     float q[DIM];
     float best, tau;
     unsigned best_i, visits;
+    const int32_t *pre;
+    VHash vh;
 };
 
 template <int DIM>
 __device__ void vp_rec(VpCtx<DIM> &c, int node, float lb, float sc) {
     ++c.visits;
+    if (c.pre) c.vh.add(c.pre, node);
     if (__fsub_rn(lb, c.tau) > __fmul_rn(TT_VP_EPS_R, __fadd_rn(sc, c.tau))) return;
     const int4 t = __ldg(reinterpret_cast<const int4 *>(c.rec + node));
     float v[DIM];
@@ -257,10 +281,13 @@ __global__ void __launch_bounds__(kBlock) vp_rec_kernel(const tt_vp_params P) {
         c.best = c.tau = __int_as_float(0x7f800000);
         c.best_i = 0xffffffffu;
         c.visits = 0;
+        c.pre = P.c.pre;
+        c.vh = VHash{};
         vp_rec<DIM>(c, 0, __int_as_float(0xff800000), 0.f);
         P.idx[pid] = c.best_i == 0xffffffffu ? -1 : (int)c.best_i;
         P.d2[pid] = c.best;
         if (P.c.st_visits) P.c.st_visits[pid] = c.visits;
+        if (c.pre) c.vh.store(P.c, pid);
     }
 }
 

@@ -112,6 +112,8 @@ __global__ void __launch_bounds__(kBlock) bh_stack_kernel(const tt_bh_params P, 
         L.ax = L.ay = L.az = 0.f;
         L.AX = L.AY = L.AZ = 0.0;
         unsigned visits = 0, fetches = 0, steps = 0;
+        VHash vh;
+        const bool hashing = STATS && P.c.pre;
         if (lock) {
             // Fig.8 with the stack in shared memory, once per warp; lane 0 owns
             // the stack, the popped entry is broadcast with __shfl_sync
@@ -138,17 +140,20 @@ __global__ void __launch_bounds__(kBlock) bh_stack_kernel(const tt_bh_params P, 
                 const bool active = (e.mask >> lane) & 1u;
                 bool open = false;
                 if (active) {
-                    if (STATS) ++visits;
+                    if (STATS) {
+                        ++visits;
+                        if (hashing) vh.add(P.c.pre, e.node);
+                    }
                     open = bh_visit(L, g, t, s_dsq, P.eps2);
+                    if (++k == kFlush) {  // per lane, after each kFlush own visits (as N)
+                        L.flush();
+                        k = 0;
+                    }
                 }
                 const unsigned cmask = __ballot_sync(TT_FULL, open);
                 if (cmask) {
                     if (lane == 0) ws[sp] = WarpEntry{t.x, t.y, cmask};
                     ++sp;
-                }
-                if (++k == kFlush) {
-                    L.flush();
-                    k = 0;
                 }
                 __syncwarp();
             }
@@ -164,7 +169,10 @@ __global__ void __launch_bounds__(kBlock) bh_stack_kernel(const tt_bh_params P, 
                 const int2 e = gpop(gstack, --sp, stride, gtid);
                 const float4 g = __ldg(reinterpret_cast<const float4 *>(&rec[e.x].gx));
                 const int4 t = __ldg(reinterpret_cast<const int4 *>(&rec[e.x].first_child));
-                if (STATS) ++visits;
+                if (STATS) {
+                    ++visits;
+                    if (hashing) vh.add(P.c.pre, e.x);
+                }
                 if (t.y != e.y) gpush(gstack, sp++, stride, gtid, t.y, e.y);
                 if (bh_visit(L, g, t, s_dsq, P.eps2)) gpush(gstack, sp++, stride, gtid, t.x, t.y);
                 if (++k == kFlush) {
@@ -181,6 +189,7 @@ __global__ void __launch_bounds__(kBlock) bh_stack_kernel(const tt_bh_params P, 
         if (valid) {
             P.acc[pid] = make_float4((float)L.AX, (float)L.AY, (float)L.AZ, 0.f);
             if (STATS && P.c.st_visits) P.c.st_visits[pid] = visits;
+            if (hashing) vh.store(P.c, pid);
         }
         if (STATS) write_warp_stats(P.c, tile, fetches, steps, lock);
     }
@@ -193,13 +202,14 @@ __global__ void __launch_bounds__(kBlock) bh_stack_kernel(const tt_bh_params P, 
 // Returns true iff the lane descends into the node's children.
 template <int DIM>
 __device__ __forceinline__ bool pc_visit(const tt_pc_params &P, const tt_kd_rec *rec, int node, int4 t, int dp,
-                                         const float (&q)[DIM], unsigned &count) {
+                                         const float (&q)[DIM], unsigned &count, unsigned &ptests) {
     float lo[DIM], hi[DIM];
     load_row_nc<DIM>(lo, P.c.tree.box + (size_t)node * 2 * dp);
     load_row_nc<DIM>(hi, P.c.tree.box + (size_t)node * 2 * dp + dp);
     if (pinned_boxd2<DIM>(q, lo, hi) > P.r2) return false;  // !can_correlate
     if (t.x >= 0) return true;
     const int4 u = __ldg(reinterpret_cast<const int4 *>(rec + node) + 1);
+    ptests += (unsigned)u.w;
     for (int j = u.z; j < u.z + u.w; ++j) {  // update_correlation over the bucket
         float p[DIM];
         load_row_nc<DIM>(p, P.c.tree.pts + (size_t)j * dp);
@@ -230,7 +240,9 @@ __global__ void __launch_bounds__(kBlock) pc_stack_kernel(const tt_pc_params P, 
         else
 #pragma unroll
             for (int d = 0; d < DIM; ++d) q[d] = 0.f;
-        unsigned count = 0, visits = 0, fetches = 0, steps = 0;
+        unsigned count = 0, visits = 0, fetches = 0, steps = 0, ptests = 0;
+        VHash vh;
+        const bool hashing = STATS && P.c.pre;
         if (lock) {
             const unsigned vmask = __ballot_sync(TT_FULL, valid);
             if (lane == 0) ws[0] = WarpEntry{0, TT_END, vmask};
@@ -250,8 +262,11 @@ __global__ void __launch_bounds__(kBlock) pc_stack_kernel(const tt_pc_params P, 
                 }
                 bool down = false;
                 if ((e.mask >> lane) & 1u) {
-                    if (STATS) ++visits;
-                    down = pc_visit<DIM>(P, rec, e.node, t, DP, q, count);
+                    if (STATS) {
+                        ++visits;
+                        if (hashing) vh.add(P.c.pre, e.node);
+                    }
+                    down = pc_visit<DIM>(P, rec, e.node, t, DP, q, count, ptests);
                 }
                 const unsigned cmask = __ballot_sync(TT_FULL, down);
                 if (cmask) {
@@ -270,9 +285,12 @@ __global__ void __launch_bounds__(kBlock) pc_stack_kernel(const tt_pc_params P, 
             while (sp > 0) {
                 const int2 e = gpop(gstack, --sp, stride, gtid);
                 const int4 t = __ldg(reinterpret_cast<const int4 *>(rec + e.x));
-                if (STATS) ++visits;
+                if (STATS) {
+                    ++visits;
+                    if (hashing) vh.add(P.c.pre, e.x);
+                }
                 if (t.z != e.y) gpush(gstack, sp++, stride, gtid, t.z, e.y);
-                if (pc_visit<DIM>(P, rec, e.x, t, DP, q, count)) gpush(gstack, sp++, stride, gtid, t.x, t.z);
+                if (pc_visit<DIM>(P, rec, e.x, t, DP, q, count, ptests)) gpush(gstack, sp++, stride, gtid, t.x, t.z);
             }
             if (STATS) {
                 fetches = warp_sum(visits);
@@ -282,6 +300,8 @@ __global__ void __launch_bounds__(kBlock) pc_stack_kernel(const tt_pc_params P, 
         if (valid) {
             P.count[pid] = count;
             if (STATS && P.c.st_visits) P.c.st_visits[pid] = visits;
+            if (STATS && P.c.st_point_tests) P.c.st_point_tests[pid] = ptests;
+            if (hashing) vh.store(P.c, pid);
         }
         if (STATS) write_warp_stats(P.c, tile, fetches, steps, lock);
     }
@@ -322,7 +342,7 @@ int launch_with_stack(Kern kern, const Params &p, const tt_launch_cfg &cfg) {
 
 template <int DIM>
 int launch_pc_dim(const tt_pc_params &p, const tt_launch_cfg &cfg) {
-    const bool stats = p.c.st_visits || p.c.st_warp_fetches || p.c.st_warp_steps || p.c.st_warp_mode;
+    const bool stats = stats_on(p.c);
     return stats ? launch_with_stack(pc_stack_kernel<DIM, true>, p, cfg)
                  : launch_with_stack(pc_stack_kernel<DIM, false>, p, cfg);
 }
@@ -331,7 +351,7 @@ int launch_pc_dim(const tt_pc_params &p, const tt_launch_cfg &cfg) {
 
 int tt_launch_bh_stack(const tt_bh_params &p, const tt_launch_cfg &cfg) {
     if (p.c.height + 2 > TT_MAX_HEIGHT + 2) return -1;
-    const bool stats = p.c.st_visits || p.c.st_warp_fetches || p.c.st_warp_steps || p.c.st_warp_mode;
+    const bool stats = stats_on(p.c);
     return stats ? launch_with_stack(bh_stack_kernel<true>, p, cfg) : launch_with_stack(bh_stack_kernel<false>, p, cfg);
 }
 

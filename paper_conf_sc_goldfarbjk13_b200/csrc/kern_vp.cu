@@ -141,12 +141,17 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
         float best_d = POS_INF, tau = POS_INF;
         unsigned best_i = 0xffffffffu;
         unsigned visits = 0, fetches = 0, steps = 0;
+        VHash vh;
+        const bool hashing = STATS && P.c.pre;
         if (!lock) {
             int sp = 0;
             int cur = valid ? 0 : TT_END;
             float lb = NEG_INF, sc = 0.f;
             while (cur != TT_END) {
-                if (STATS) ++visits;
+                if (STATS) {
+                    ++visits;
+                    if (hashing) vh.add(P.c.pre, cur);
+                }
                 if (!vp_prune(lb, sc, tau)) {
                     int4 t;
                     float v[DIM];
@@ -199,6 +204,7 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
                 if (STATS) {
                     ++steps;
                     visits += in;
+                    if (hashing) vh.add_if(in, P.c.pre, cur);
                 }
                 const bool active = in && !vp_prune(lb, sc, tau);
                 const unsigned act = __ballot_sync(TT_FULL, active);
@@ -256,6 +262,7 @@ __global__ void __launch_bounds__(kBlock) vp_kernel(const tt_vp_params P, int ca
             P.idx[pid] = best_i == 0xffffffffu ? -1 : (int)best_i;
             P.d2[pid] = best_d;
             if (STATS && P.c.st_visits) P.c.st_visits[pid] = visits;
+            if (hashing) vh.store(P.c, pid);
         }
         if (STATS) write_warp_stats(P.c, tile, fetches, steps, lock);
         __syncwarp();
@@ -300,7 +307,7 @@ int launch(const tt_vp_params &p, const tt_launch_cfg &cfg) {
 
 template <int DIM>
 int launch_dim(const tt_vp_params &p, const tt_launch_cfg &cfg) {
-    const bool stats = p.c.st_visits || p.c.st_warp_fetches || p.c.st_warp_steps || p.c.st_warp_mode;
+    const bool stats = stats_on(p.c);
     return stats ? launch<DIM, true>(p, cfg) : launch<DIM, false>(p, cfg);
 }
 

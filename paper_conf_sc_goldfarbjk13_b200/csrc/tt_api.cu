@@ -57,6 +57,58 @@ constexpr int kAutoBH = 3, kAutoPC = 255, kAutoKNN = 4, kAutoVP = 4, kAutoNN = 4
 // the budget trades staged levels against occupancy.
 constexpr int kTopBH = 32 * 1024, kTopPC = 32 * 1024, kTopKNN = 16 * 1024, kTopVP = 4 * 1024, kTopNN = 8 * 1024;
 
+// Canonical preorder id of every device node (for the stats hashes): the
+// blob numbers the top levels level by level, so the map is rebuilt on the
+// host from the records' child links (first child first, the Fig.2 order)
+// once per tree and kept on the device.  Stats-only; synchronous.
+tt_status ensure_preorder(tt_tree *t) {
+    std::lock_guard<std::mutex> lk(t->grp_mu);
+    if (t->d_pre) return TT_OK;
+    const int64_t N = t->hdr.n_nodes;
+    const size_t rb = (size_t)t->hdr.rec_bytes;
+    std::vector<int32_t> rec;
+    std::vector<int32_t> pre;
+    try {
+        rec.resize((size_t)N * rb / 4);
+        pre.assign((size_t)N, -1);
+    } catch (const std::bad_alloc &) {
+        return TT_ERR_OOM;
+    }
+    cudaError_t e = cudaMemcpy(rec.data(), t->dev.rec, (size_t)N * rb, cudaMemcpyDeviceToHost);
+    if (e != cudaSuccess) return cuda_fail(e);
+    const size_t w = rb / 4;  // int32 words per record
+    auto at = [&](int64_t v, int f) { return rec[(size_t)v * w + (size_t)f]; };
+    std::vector<int32_t> stk;
+    stk.push_back(0);
+    int32_t next = 0;
+    std::vector<int32_t> kids;
+    while (!stk.empty()) {
+        const int32_t v = stk.back();
+        stk.pop_back();
+        if (v < 0 || v >= N || pre[(size_t)v] >= 0) return TT_ERR_INVALID_ARG;  // not a tree
+        pre[(size_t)v] = next++;
+        kids.clear();
+        if (t->hdr.kind == TT_KIND_OCT) {  // first_child (word 4), then the skip chain (word 5)
+            const int32_t end = at(v, 5);
+            for (int32_t c = at(v, 4); c >= 0 && c != end; c = at(c, 5)) kids.push_back(c);
+        } else {  // KD {left, right, ...}, VP {in, out, ...}, NN {left, right, ...}
+            for (int f = 0; f < 2; ++f)
+                if (at(v, f) >= 0) kids.push_back(at(v, f));
+        }
+        for (size_t i = kids.size(); i-- > 0;) stk.push_back(kids[i]);
+    }
+    if (next != N) return TT_ERR_INVALID_ARG;
+    int32_t *d = nullptr;
+    e = cudaMalloc((void **)&d, sizeof(int32_t) * (size_t)N);
+    if (e == cudaSuccess) e = cudaMemcpy(d, pre.data(), sizeof(int32_t) * (size_t)N, cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) {
+        if (d) cudaFree(d);
+        return cuda_fail(e);
+    }
+    t->d_pre = d;
+    return TT_OK;
+}
+
 tt_status setup_common(const tt_tree *t, int kind, int64_t n, const tt_traverse_opts *o, int default_amd,
                        int stage_bytes_per_node, int stage_budget, tt_common_params &c, tt_launch_cfg &cfg,
                        tt_stream s, bool allow_switch = false) {
@@ -88,6 +140,14 @@ tt_status setup_common(const tt_tree *t, int kind, int64_t n, const tt_traverse_
             c.st_warp_fetches = o->stats->warp_fetches;
             c.st_warp_steps = o->stats->warp_steps;
             c.st_warp_mode = o->stats->warp_mode;
+            c.st_hash = o->stats->visit_hash;
+            c.st_set = o->stats->visit_set;
+            c.st_point_tests = o->stats->point_tests;
+            if (c.st_hash || c.st_set) {
+                tt_status ps = ensure_preorder(const_cast<tt_tree *>(t));
+                if (ps != TT_OK) return ps;
+                c.pre = t->d_pre;
+            }
         }
         if (o->block_threads != 0 && o->block_threads != 256) return TT_ERR_UNSUPPORTED;
         if (o->ctas_per_sm < 0) return TT_ERR_INVALID_ARG;
@@ -423,6 +483,7 @@ tt_status tt_tree_free(tt_tree *t) {
     if (idle) tt_bh_groups_release(t->d_grp);
     else tt_bh_groups_discard(t->d_grp);
     if (t->grp_ready) cudaEventDestroy(t->grp_ready);
+    if (t->d_pre) cudaFree(t->d_pre);
     delete t;
     return idle ? TT_OK : cuda_fail(e1);
 }

@@ -102,6 +102,11 @@ struct tt_common_params {
     // stats (nullable)
     uint32_t *st_visits, *st_warp_fetches, *st_warp_steps;
     uint8_t *st_warp_mode;
+    // per-point visit hashes (nullable; `pre` = canonical preorder id of every
+    // device node, set whenever a hash is requested) and leaf-point tests
+    uint64_t *st_hash, *st_set;
+    const int32_t *pre;
+    uint32_t *st_point_tests;
     // root cube (OCT AUTO mode)
     double root_center[3], root_side;
 };
@@ -149,6 +154,7 @@ struct tt_tree {
     tt_dev_tree dev;
     uint32_t *d_counters;  // [TT_COUNTER_SLOTS][2]
     unsigned slot_next;
+    int32_t *d_pre = nullptr;  // canonical preorder id of every device node (stats hashes), built on first use
     void *d_grp = nullptr;  // OCT: child-group records (kern_bh_group.cu), built on first use
     cudaEvent_t grp_ready = nullptr;  // recorded on the stream of that build
     std::mutex grp_mu;

@@ -261,14 +261,24 @@ class Stats:
     warp_fetches: torch.Tensor
     warp_steps: torch.Tensor
     warp_mode: torch.Tensor
+    visit_hash: torch.Tensor | None = None   # int64 storage of the uint64 hashes
+    visit_set: torch.Tensor | None = None
+    point_tests: torch.Tensor | None = None
 
     @staticmethod
-    def alloc(n: int, device) -> "Stats":
+    def alloc(n: int, device, hashes: bool = False, point_tests: bool = False) -> "Stats":
         nw = (n + 31) // 32
         return Stats(torch.zeros(n, dtype=torch.int32, device=device),
                      torch.zeros(nw, dtype=torch.int32, device=device),
                      torch.zeros(nw, dtype=torch.int32, device=device),
-                     torch.zeros(nw, dtype=torch.uint8, device=device))
+                     torch.zeros(nw, dtype=torch.uint8, device=device),
+                     torch.zeros(n, dtype=torch.int64, device=device) if hashes else None,
+                     torch.zeros(n, dtype=torch.int64, device=device) if hashes else None,
+                     torch.zeros(n, dtype=torch.int32, device=device) if point_tests else None)
+
+    def hashes(self):
+        """(visit_hash, visit_set) as numpy uint64 arrays."""
+        return (self.visit_hash.cpu().numpy().view("uint64"), self.visit_set.cpu().numpy().view("uint64"))
 
 
 def _lanes(order, n):
@@ -289,8 +299,10 @@ def _opts(mode, auto_min_depth, order, stats, n, variant="autoropes", switch_bel
             raise ValueError("order must be a contiguous 1-D index tensor over the point rows")
         o.order = order.data_ptr()
     if stats is not None:
+        opt = lambda t: None if t is None else t.data_ptr()  # noqa: E731
         st = L.tt_stats(stats.visits.data_ptr(), stats.warp_fetches.data_ptr(), stats.warp_steps.data_ptr(),
-                        stats.warp_mode.data_ptr())
+                        stats.warp_mode.data_ptr(), opt(stats.visit_hash), opt(stats.visit_set),
+                        opt(stats.point_tests))
         keep.append(st)
         o.stats = C.addressof(st)
     return o, keep

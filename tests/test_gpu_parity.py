@@ -111,9 +111,11 @@ def test_bh_within_1e4_and_same_openings(bh_small, mode, sorted_):
 
 
 def test_bh_lockstep_equals_independent(bh_small):
-    """Fig.8 only masks: each lane makes the same opening decisions in both
-    modes (identical visit counts) and sums the same terms in the same order;
-    only the fp32->fp64 flush cadence differs (per warp step vs per lane)."""
+    """Default BH path: each body makes the same opening decisions in both
+    modes (identical visit counts); the child-group lockstep walk adds the
+    body's terms in DFS-over-groups order (reading R23), so L and N agree to
+    rounding.  (The per-node lockstep walks are bit-identical to N:
+    tests/test_gpu_order.py.)"""
     b, ot, ref, tree = bh_small
     bd = dev(b)
     sl, sn = P.Stats.alloc(len(b), "cuda"), P.Stats.alloc(len(b), "cuda")
