@@ -673,3 +673,18 @@ def test_guided_lockstep_lane_hash_equals_independent_when_alone(kind):
         ind, ls = getattr(oracle, kind)(t, q, stats=True), getattr(oracle, kind + "_lockstep")(t, q)
     assert ls.lane_visits[0] == ind.visits[0] and ls.lane_hash[0] == ind.hash[0]
     assert ls.warp_tests[0] == ind.visits[0]
+
+
+@pytest.mark.parametrize("dup", [9, 40])
+def test_bh_large_bucket_theta0_direct_sum(dup):
+    """A depth-32 bucket (R9) holds any number of coincident bodies, one leaf
+    child each: at theta = 0 the walk still equals the O(n^2) direct sum."""
+    from tests import brute
+    b = ttgen.plummer(1200, seed=35 + dup)
+    b[100:100 + dup, :3] = b[3, :3]
+    t = oracle.build_oct(b)
+    assert t.height == 33
+    assert np.array_equal(np.sort(t.tree_order()), np.arange(len(b)))
+    a = oracle.bh(t, b, 0.0, 0.05, self_ids=np.arange(len(b))).out[0]
+    want = brute.direct_sum(b, 0.05)
+    assert (np.linalg.norm(a - want, axis=1) / np.linalg.norm(want, axis=1)).max() < 1e-11
