@@ -10,17 +10,28 @@ paper figure, see its header); this module only compiles it with
 ``-O2 -ffp-contract=off -fopenmp`` and marshals numpy arrays through ctypes.
 
 Parity status of each function:
-  build_kd / build_oct / build_vp  pinned: invariants + brute-force partition checks
+  build_kd / build_oct / build_vp  pinned: invariants + brute-force partition checks; oct
+                                   buckets of any size (R9) == direct sum at theta = 0
   linearise (skip/preorder)        pinned: Fig.2 worked example (tests/golden/fig2_ropes.txt)
   pc                               pinned: all-pairs brute force, symmetry, r=inf
-  bh                               pinned: theta=0 == O(n^2) direct sum, two-body closed form
+  bh                               pinned: theta=0 == O(n^2) direct sum, two-body closed form,
+                                   the R8 opening test by a hand-worked 10-node example
+                                   (visits, order hash, forces), error monotone in theta;
+                                   1M-Plummer visits/body and work expansion within 10% of
+                                   Tables 1-2 (sanity)
   knn                              pinned: brute-force partial sort on (d2, id)
   vp                               pinned: brute-force argmin on (d2, id)
   build_nn / nn (NEXT-3, R21)      pinned: brute-force argmin on (d2, id), == kNN k=1 == VP;
                                    builder: median/split/partition invariants
-  sort_keys                        pinned: Morton/preorder invariants, bijection
-  *_lockstep, unguided_warp_union  pinned: results == independent walks; fetches >= max lane
-                                   visits; absolute fetch counts parity unpinned
+  sort_keys                        pinned: kd/oct Morton/preorder invariants; vp/nn: a data
+                                   point's descent passes its own node except at checked
+                                   boundary ties; keys sort in preorder of the end node
+  visit hashes (stats=True)        pinned: order hash of a full walk == preorder sequence; set
+                                   hash == sum over all nodes; R8 example's order hash
+  *_lockstep, unguided_warp_union  pinned: results == independent walks; per warp, nodes tested
+                                   >= the longest lane; Table 2 work expansion >= 1 on average
+                                   (P:L2307-2313); a one-lane warp == the recursive walk;
+                                   absolute fetch counts on our inputs: parity unpinned
 """
 from __future__ import annotations
 

@@ -688,3 +688,80 @@ def test_bh_large_bucket_theta0_direct_sum(dup):
     a = oracle.bh(t, b, 0.0, 0.05, self_ids=np.arange(len(b))).out[0]
     want = brute.direct_sum(b, 0.05)
     assert (np.linalg.norm(a - want, axis=1) / np.linalg.norm(want, axis=1)).max() < 1e-11
+
+
+# ------------------------------------------------------ VP / NN sort keys (a1)
+def _decode_path(key, children):
+    """Nodes on the 2-bit-per-level descent code (01 = first child, 10 =
+    second, 00 = end; R18), starting at the root."""
+    path, v = [0], 0
+    for lvl in range(31):
+        c = (int(key) >> (62 - 2 * lvl)) & 3
+        if c == 0:
+            break
+        v = int(children[v, c - 1])
+        assert v >= 0
+        path.append(v)
+    return path
+
+
+def _ancestors(children, n):
+    par = np.full(n, -1, np.int64)
+    for v in range(n):
+        for c in children[v]:
+            if c >= 0:
+                par[c] = v
+    return par
+
+
+@pytest.mark.parametrize("kind", ["vp", "nn"])
+def test_sort_keys_vp_nn_descend_to_the_points_own_node(kind):
+    """Pins the VP / NN key paths (R18) against the builders' partitions
+    (pinned above by brute force): a data point's descent by the build's
+    rule -- VP: inside iff sqrt_rn(d2(vp, x)) <= r_in_max; NN: left iff
+    x[dim] < split -- passes through the node holding the point itself, the
+    node where it is the vantage / node point.  The only exceptions are the
+    boundary ties the rule cannot separate (VP: an outside point at exactly
+    r_in_max; NN: a left point with x[dim] == split), each checked to be one.
+    Keys sort in preorder of the path's end node (end 00 < 01 < 10)."""
+    d = 16 if kind == "vp" else 7
+    p = ttgen.gaussian_mixture(3000, d, seed=74, components=5)
+    p[40:44] = p[2]  # exact duplicates make boundary ties
+    t = oracle.build_vp(p) if kind == "vp" else oracle.build_nn(p)
+    keys = oracle.sort_keys(t, p)
+    ch = t.children()[:, :2]
+    own = np.full(len(p), -1, np.int64)
+    own[t.i64(oracle.F_VP)] = np.arange(t.n_nodes)
+    par = _ancestors(ch, t.n_nodes)
+    pre_end = np.empty(len(p), np.int64)
+    exceptions = 0
+    for x in range(len(p)):
+        path = _decode_path(keys[x], ch)
+        pre_end[x] = path[-1]
+        if own[x] in path:
+            continue
+        # walk up from the point's own node: find the ancestor where the rule
+        # sends x the other way, and check it is a boundary tie
+        v, tie = own[x], False
+        while par[v] >= 0:
+            a, side = par[v], int(np.where(ch[par[v]] == v)[0][0])
+            if kind == "vp":
+                dd = np.sqrt(brute.pinned_d2(p[[x]], p[[t.i64(oracle.F_VP)[a]]])[0, 0]).astype(np.float32)
+                goes_in = dd <= t.f32(oracle.F_RIN)[a]
+                if goes_in != (side == 0):
+                    tie = side == 1 and dd == t.f32(oracle.F_RIN)[a]
+                    break
+            else:
+                sd, sp = t.i64(oracle.F_SPLITDIM)[a], t.f32(oracle.F_SPLIT)[a]
+                goes_left = p[x, sd] < sp
+                if goes_left != (side == 0):
+                    tie = side == 0 and p[x, sd] == sp
+                    break
+            v = a
+        assert tie, x
+        exceptions += 1
+    assert exceptions < len(p) // 20
+    # key order = preorder of the end node (first child before second, a node
+    # before its subtree): non-decreasing preorder along the sorted keys
+    srt = np.argsort(keys, kind="stable")
+    assert np.all(np.diff(pre_end[srt]) >= 0)
