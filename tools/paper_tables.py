@@ -107,7 +107,8 @@ def main():
         if name != "nn":
             rec_ms = timed(lambda: launch(sorted_order, "independent", variant="recursive"), reps=1, warm=1)
         for oname, order in (("sorted", sorted_order), ("unsorted", None)):
-            for mode in ("lockstep", "independent"):
+            vis_n = None
+            for mode in ("independent", "lockstep"):
                 ms = timed(lambda: launch(order, mode))
                 st = P.Stats.alloc(m, dev)
                 launch(order, mode, stats=st)
@@ -115,13 +116,18 @@ def main():
                 vis = st.visits.to(torch.int64).cpu().numpy()
                 nodes = vis.mean()
                 we = None
-                if mode == "lockstep":
+                if mode == "independent":
+                    vis_n = vis
+                else:
+                    # Table 2: nodes the lockstep warp tests /
+                    # nodes of its longest non-lockstep traversal (N-mode
+                    # visits of the same points), per warp tile of T points
                     o = sorted_order.cpu().numpy() if order is not None else np.arange(m)
-                    v = vis[o]
+                    v = vis_n[o]
                     nt = m // T
                     longest = v[: nt * T].reshape(nt, T).max(1)
-                    wf = st.warp_fetches[:nt].to(torch.int64).cpu().numpy()
-                    we = float(np.mean(wf / np.maximum(longest, 1)))
+                    wt = st.warp_steps[:nt].to(torch.int64).cpu().numpy()
+                    we = float(np.mean(wt / np.maximum(longest, 1)))
                 pts_s = m / (ms / 1e3)
                 rows.append(dict(bench=name, workload=w["workload"], order=oname, mode="L" if mode == "lockstep" else "N",
                                  ms=ms, nodes=nodes, we=we, vs1=pts_s / rate1, vsN=pts_s / rateN,
@@ -132,7 +138,8 @@ def main():
              f"Host oracle threads: {ncpu} (`vs all`), 1 (`vs 1`); the paper's CPU columns used a 32-thread "
              "Opteron and a C2070 GPU (P:L1110-1117), context only.  L = lockstep, N = independent; "
              "avg # nodes = truncation tests per point; work expansion = mean over warp tiles of "
-             "fetches / longest lane (Table 2); improv. vs recurse = naive recursive GPU kernel time / "
+             "nodes the lockstep warp tests / the longest independent traversal among its points "
+             "(Table 2, P:L2307-2313; BH tiles hold 64 bodies, the others 32); improv. vs recurse = naive recursive GPU kernel time / "
              "autoropes time (N, sorted).", "",
              "| benchmark | order | mode | time (ms) | avg # nodes | work expansion | speedup vs 1 | speedup vs all | improv. vs recurse |",
              "|---|---|---|---|---|---|---|---|---|"]
