@@ -37,9 +37,15 @@ sys.path.insert(0, ROOT)
 import ttgen  # noqa: E402
 
 METRIC = "points traversed/sec and node visits/sec at 1/2/4/8 B200; % HBM peak"
-# algorithmic bytes per useful visit of each kernel's packed layout
-BYTES_PER_VISIT = {"bh": 32, "pc": 48, "knn": 96, "vp": 80, "nn": 48}
+# SURVEY §8(d) algorithmic bytes per useful visit (kNN: 16 B per node visit
+# plus 32 B per leaf-point distance, tt_stats.point_tests; NN, not in §8(d):
+# its 16-B header + the node's 32-B point) and per point of I/O
+BYTES_PER_VISIT = {"bh": 32, "pc": 32, "knn": 16, "vp": 80, "nn": 48}
+BYTES_PER_POINT_TEST = {"knn": 32}
 BYTES_PER_POINT_IO = {"bh": 32, "pc": 20, "knn": 28 + 64, "vp": 64 + 8, "nn": 28 + 8}
+# bytes of one fetched node in our packed layout (record + the side rows read
+# with it: kd boxes, kNN children's boxes, VP / NN points), for node_fetch
+FETCH_BYTES = {"bh": 32, "pc": 32 + 32, "knn": 32 + 128, "vp": 16 + 64, "nn": 16 + 64 + 32}
 L2_FLUSH_BYTES = 512 << 20  # > 126 MB L2
 
 
@@ -61,6 +67,9 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-chase", action="store_true", help="skip the live L2-latency (tt_diag_chase) roof")
     ap.add_argument("--points-per-rank", type=int, default=0, help="override M (testing)")
+    ap.add_argument("--no-strong", action="store_true",
+                    help="skip the fixed-config strong-scaling block (configs[4] BH 16M, every N)")
+    ap.add_argument("--strong-points", type=int, default=0, help="override the strong block's N (testing)")
     ap.add_argument("--auto-min-depth", type=int, default=None, help="AUTO-mode threshold (default: kernel's)")
     ap.add_argument("--switch-below", type=int, default=0,
                     help="kNN: dynamic L->N switch when fewer lanes are active (NEXT-3; 0 = never)")
@@ -278,6 +287,24 @@ def chase_ceiling(P, nrec: int, device, per_lane: bool, steps: int = 3000) -> fl
     return chains * n / statistics.median(ts)
 
 
+def l2_ceiling(P, device, nbytes: int = 64 << 20, reps: int = 20) -> float:
+    """L2 read GB/s of an L2-resident buffer (tt_diag_l2read), median of 3."""
+    import torch
+    buf = torch.ones(nbytes // 4, dtype=torch.float32, device=device)
+    s = torch.cuda.current_stream()
+    P.tt_diag_l2read(buf, reps)
+    ts = []
+    for _ in range(3):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(s)
+        P.tt_diag_l2read(buf, reps)
+        b.record(s)
+        torch.cuda.synchronize()
+        ts.append(a.elapsed_time(b) / 1e3)
+    del buf
+    return nbytes * reps / statistics.median(ts) / 1e9
+
+
 def measured_peaks():
     try:
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))), "measured"
@@ -398,6 +425,91 @@ def run_bh_steps(args, rank, world):
     print(json.dumps(line), flush=True)
 
 
+def run_strong16m(args, rank, world, device, P, PAR):
+    """configs[4]: one fixed Barnes-Hut problem (16M-body Plummer sphere,
+    theta 0.5) at every N -- strong scaling.  Rank 0 builds the tree on its
+    GPU (tt_build_oct_device, NEXT-1) and NCCL-broadcasts the packed blob
+    (tt_tree_copy_blob -> broadcast -> tt_tree_from_blob); every rank places
+    the bodies in global tree order once (data placement) and owns a
+    contiguous warp-aligned range; a timed step = a1 sort of the rank's shard
+    + traversal + all-gather of the accelerations.  Each phase is reported
+    separately; every time is the max over ranks (CUDA events)."""
+    import torch
+    import torch.distributed as dist
+    c = ttgen.CONFIGS["bh_16m_plummer"]
+    n = args.strong_points or c["n"]
+    if world > 1 and n % (64 * world):
+        raise SystemExit(f"bench: {n} bodies do not split into {world} equal warp-aligned shards")
+    data = ttgen.plummer(n, c["seed"])
+    bd_all = torch.from_numpy(data).to(device)
+    stream = torch.cuda.current_stream()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    tree = P.tt_build_oct_device(bd_all) if rank == 0 else None
+    torch.cuda.synchronize()
+    build_ms = 1e3 * (time.perf_counter() - t0)
+    bcast_ms = None
+    if world > 1:
+        dist.barrier()
+        t0 = time.perf_counter()
+        tree = PAR.broadcast_device_tree(tree, device)
+        torch.cuda.synchronize()
+        bcast_ms = PAR.max_over_ranks(1e3 * (time.perf_counter() - t0), device)
+    t0 = time.perf_counter()
+    gperm = P.tt_sort_points(tree, bd_all).long()
+    q = bd_all[gperm].contiguous()
+    ids = gperm.to(torch.int32)
+    del bd_all, gperm
+    torch.cuda.synchronize()
+    placement_ms = 1e3 * (time.perf_counter() - t0)
+    lo, hi = PAR.shard_range(n, rank, world)
+    q_shard, ids_shard = q[lo:hi], ids[lo:hi]
+    out = torch.zeros((n, 4), dtype=torch.float32, device=device)
+    out_shard = out[lo:hi]
+    order = torch.empty(hi - lo, dtype=torch.int32, device=device)
+
+    def step(ev=None):
+        if ev:
+            ev[0].record(stream)
+        P.tt_sort_points(tree, q_shard, out=order)
+        if ev:
+            ev[1].record(stream)
+        P.tt_traverse_bh(tree, q_shard, c["theta"], c["eps"], out=out_shard, self_ids=ids_shard, order=order)
+        if ev:
+            ev[2].record(stream)
+        if world > 1:
+            PAR.allgather_rows(out, world)
+        if ev:
+            ev[3].record(stream)
+
+    for _ in range(args.warmup):
+        step()
+    flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.float32, device=device)
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in range(args.steps)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    for i in range(args.steps):
+        flush.zero_()
+        step(evs[i])
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    mean = lambda a, b: statistics.mean(e[a].elapsed_time(e[b]) for e in evs)  # noqa: E731
+    ms, sort_ms, trav_ms, ag_ms = mean(0, 3), mean(0, 1), mean(1, 2), mean(2, 3)
+    if world > 1:
+        ms, sort_ms, trav_ms, ag_ms, placement_ms = (PAR.max_over_ranks(x, device) for x in
+                                                     (ms, sort_ms, trav_ms, ag_ms, placement_ms))
+    del flush, out, q, ids
+    return {"workload": "bh_16m_plummer", "scaling": "strong", "value": n / (ms / 1e3), "unit": "points/s",
+            "ms_per_step": ms, "sort_ms": sort_ms, "traverse_ms": trav_ms,
+            "allgather_ms": ag_ms if world > 1 else None, "points": n, "points_per_rank": hi - lo,
+            "tree_build_ms": build_ms, "tree_build": "device (tt_build_oct_device) on rank 0",
+            "bcast_ms": bcast_ms, "placement_ms": placement_ms,
+            "note": "configs[4] at every N: step = a1 sort of the rank's shard + traversal + all-gather; "
+                    "build, broadcast and placement outside the timed steps, reported here"}
+
+
 def run_ours(args, rank, world, local_rank):
     import torch
     import torch.distributed as dist
@@ -411,8 +523,11 @@ def run_ours(args, rank, world, local_rank):
     name = {"bh16m": "bh", "knn16m": "knn"}.get(args.workload, args.workload)
     c = w["cfg"]
     m = w["m"]
+    if world > 1 and len(w["queries"]) % (64 * world):
+        raise SystemExit(f"bench: {len(w['queries'])} points do not split into {world} equal warp-aligned "
+                         "shards (the in-place all-gather needs n % (64 * N) == 0)")
     lo, hi = PAR.shard_range(len(w["queries"]), rank, world)
-    m = hi - lo  # warp-aligned shard (strong-scaling workloads: the last may be shorter)
+    m = hi - lo  # warp-aligned equal shards
 
     # a0: tree (rank 0 builds; NCCL broadcast for N > 1) -- timed separately
     t0 = time.perf_counter()
@@ -442,6 +557,9 @@ def run_ours(args, rank, world, local_rank):
 
     q_all = torch.from_numpy(np.ascontiguousarray(w["queries"])).to(device)
     ids_all = None
+    bcast_ms = upload_ms if world > 1 and not args.device_build else None
+    torch.cuda.synchronize()
+    t_pl = time.perf_counter()
     if world > 1 and not args.unsorted:
         # Spatial decomposition (data placement, before the timed region, as a
         # time-stepping code keeps its bodies -- DESIGN.md §9): rank r owns a
@@ -451,6 +569,8 @@ def run_ours(args, rank, world, local_rank):
         q_all = q_all[gperm].contiguous()
         ids_all = gperm.to(torch.int32)
     q_shard = q_all[lo:hi]
+    torch.cuda.synchronize()
+    placement_ms = 1e3 * (time.perf_counter() - t_pl) if world > 1 and not args.unsorted else None
     n_all = len(w["queries"])
     stream = torch.cuda.current_stream()
     order_buf = torch.empty(m, dtype=torch.int32, device=device)
@@ -500,7 +620,7 @@ def run_ours(args, rank, world, local_rank):
     # a1b pays only when there are more tiles than resident warps (148 SMs x 32)
     lpt = not args.unsorted and not args.no_schedule and tree.kind != "oct" and m // 32 > 148 * 32
 
-    def step(kev=None, collective=True):
+    def step(kev=None, collective=True, agev=None):
         if not args.unsorted:
             P.tt_sort_points(tree, q_shard, out=order_buf)  # a1
             if lpt:
@@ -511,8 +631,12 @@ def run_ours(args, rank, world, local_rank):
         if kev:
             kev[1].record(stream)
         if world > 1 and collective:
+            if agev:
+                agev[0].record(stream)
             for o in (out if isinstance(out, tuple) else (out,)):
                 PAR.allgather_rows(o, world)
+            if agev:
+                agev[1].record(stream)
 
     clk = ClockSampler(gpu).__enter__()
     # stats pass (untimed): per-point useful visits, warp fetches, modes
@@ -520,10 +644,11 @@ def run_ours(args, rank, world, local_rank):
         P.tt_sort_points(tree, q_shard, out=order_buf)
         if lpt:
             P.tt_schedule_tiles(tree, q_shard, order_buf, out=order_buf)
-    st = P.Stats.alloc(m, device)
+    st = P.Stats.alloc(m, device, point_tests=name in BYTES_PER_POINT_TEST)
     traverse(q_shard, out_shard, order_buf, st)
     torch.cuda.synchronize()
     visits = int(st.visits.to(torch.int64).sum().item())
+    ptests = int(st.point_tests.to(torch.int64).sum().item()) if st.point_tests is not None else 0
     tile_pts = P._lib.TILE_POINTS[tree.kind] if args.variant in ("autoropes", "groups", "ropes") else 32
     tiles = -(-m // tile_pts)
     wf = int(st.warp_fetches[:tiles].to(torch.int64).sum().item())
@@ -539,13 +664,14 @@ def run_ours(args, rank, world, local_rank):
     flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.float32, device=device)
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     kevs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    agevs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
     for i in range(args.steps):
         flush.zero_()  # L2 flush between timed iterations (outside the events)
         evs[i][0].record(stream)
-        step(kevs[i])
+        step(kevs[i], agev=agevs[i])
         evs[i][1].record(stream)
     torch.cuda.synchronize()
     if world > 1:
@@ -554,9 +680,15 @@ def run_ours(args, rank, world, local_rank):
     kern_ms = [a.elapsed_time(b) for a, b in kevs]
     ms = statistics.mean(step_ms)
     kms = statistics.mean(kern_ms)
+    allgather_ms = statistics.mean(a.elapsed_time(b) for a, b in agevs) if world > 1 else None
     if world > 1:
         ms = PAR.max_over_ranks(ms, device)
         kms = PAR.max_over_ranks(kms, device)
+        allgather_ms = PAR.max_over_ranks(allgather_ms, device)
+        if bcast_ms is not None:
+            bcast_ms = PAR.max_over_ranks(bcast_ms, device)
+        if placement_ms is not None:
+            placement_ms = PAR.max_over_ranks(placement_ms, device)
         visits_all = torch.tensor([visits], dtype=torch.int64, device=PAR._wire(device))
         dist.all_reduce(visits_all)
         visits_tot = int(visits_all.item())
@@ -632,46 +764,75 @@ def run_ours(args, rank, world, local_rank):
         step()
         torch.cuda.synchronize()
     clk.__exit__(None, None, None)
+    # fixed-config strong scaling (configs[4], BH 16M): the same workload at
+    # every N, so the driver's 1/2/4/8-GPU lines are comparable
+    strong = None
+    if args.workload == "bh" and not args.no_strong and not args.unsorted:
+        del q_all, out, out_shard
+        torch.cuda.empty_cache()
+        strong = run_strong16m(args, rank, world, device, P, PAR)
     if rank != 0:
         return
     peaks, peak_src = measured_peaks()
     hbm = float(peaks.get("hbm_gbs", 6650.0))
     bpv = BYTES_PER_VISIT[name]
-    alg_bytes = visits * bpv + m * BYTES_PER_POINT_IO[name]  # per launch on rank 0
+    bpt = BYTES_PER_POINT_TEST.get(name, 0)
+    # SURVEY §8(d) algorithmic bytes per launch on rank 0
+    alg_bytes = visits * bpv + ptests * bpt + m * BYTES_PER_POINT_IO[name]
     achieved = alg_bytes / (kms / 1e3) / 1e9
     kernel_name = {"bh": "bh_group_kernel", "pc": "pc_kernel", "knn": "knn_kernel", "vp": "vp_kernel", "nn": "nn_kernel"}[name]
-    cnt = load_counts(name, args.mode) if not args.unsorted and args.variant == "autoropes" else None
+    cnt = load_counts(args.workload, args.mode) if not args.unsorted and args.variant == "autoropes" else None
+    cnt_ok = bool(cnt) and cnt.get("src_sha256") == kernel_sha256(name)
     clocks = clk.summary()
     sm_mhz = clocks.get("sm_mhz") or float(peaks.get("sm_max_mhz", 1965.0))
     nsm = torch.cuda.get_device_properties(device).multi_processor_count
-    # The kernels are not HBM-bound (trees L2-resident, lockstep broadcast):
-    # the binding roof is instruction issue (ncu issue-slot utilisation), so
-    # the primary roofline is executed warp instructions per second against
-    # 148 SMs x 4 schedulers x clock; SURVEY §8(d)'s effective node-fetch
-    # bandwidth (the north_star's "% HBM peak") is reported alongside.
+    # Three views of the dominant kernel, all measured live except the ncu
+    # instruction count:
+    #  * `roofline` (primary): executed warp instructions / s against the
+    #    issue ceiling 148 SMs x 4 schedulers x clock -- the binding roof
+    #    (ncu issue slots 73-79% busy; DRAM < 2% of peak);
+    #  * `hbm_effective`: SURVEY §8(d)'s algorithmic bytes / kernel time vs
+    #    the measured HBM copy bandwidth (the north_star's "effective
+    #    node-fetch bandwidth"); above 1 because warp fetches are broadcast
+    #    to the lanes and served from L1/L2, so it is NOT HBM evidence;
+    #  * `node_fetch`: bytes of the node records the warps actually fetch
+    #    (warp fetches x the layout's bytes per fetched node) / kernel time,
+    #    against the measured HBM bandwidth and a live L2 read ceiling
+    #    (tt_diag_l2read); `traffic` = ncu DRAM bytes of the same launch.
     hbm_eff = {"bound": "hbm", "achieved": round(achieved, 1), "peak": hbm, "unit": "GB/s",
                "frac": round(achieved / hbm, 4), "peak_source": peak_src,
                "alg_bytes_per_launch": int(alg_bytes),
-               "alg_bytes_def": f"useful visits x {bpv} B record + {BYTES_PER_POINT_IO[name]} B/point I/O "
-                                "(SURVEY 8(d)); served by L1/L2 and warp broadcast, not HBM",
-               "warp_fetch_bytes_per_launch": int(wf * bpv)}
+               "alg_bytes_def": f"useful visits x {bpv} B" + (f" + leaf-point tests x {bpt} B" if bpt else "")
+                                + f" + {BYTES_PER_POINT_IO[name]} B/point I/O (SURVEY 8(d)); "
+                                "served by L1/L2 and warp broadcast, not HBM"}
+    fetch_bytes = wf * FETCH_BYTES[name]
+    nf_gbs = fetch_bytes / (kms / 1e3) / 1e9
+    node_fetch = {"achieved": round(nf_gbs, 1), "unit": "GB/s", "fetch_bytes_per_launch": int(fetch_bytes),
+                  "def": f"warp node fetches (tt_stats) x {FETCH_BYTES[name]} B per fetched node of the packed "
+                         "layout / kernel time",
+                  "hbm_peak": hbm, "hbm_frac": round(nf_gbs / hbm, 4), "hbm_peak_source": peak_src}
+    if not args.no_chase:
+        l2 = l2_ceiling(P, device)
+        node_fetch.update({"l2_peak": round(l2, 1), "l2_frac": round(nf_gbs / l2, 4),
+                           "l2_peak_def": "tt_diag_l2read: 64 MiB L2-resident buffer, ld.global.cg, measured live"})
     common = {"kernel": kernel_name, "kernel_ms": round(kms, 4),
               "kernel_share_of_step": round(kms / ms, 4) if world == 1 else None,
-              "traffic": int(cnt["dram_bytes_per_point"] * m) if cnt else None,
-              "traffic_def": "ncu dram__bytes_read.sum + dram__bytes_write.sum per launch (scaled per point)"}
-    if cnt and cnt.get("src_sha256") == kernel_sha256(name):
+              "traffic": int(cnt["dram_bytes_per_point"] * m) if cnt_ok else None,
+              "traffic_def": "ncu dram__bytes_read.sum + dram__bytes_write.sum of this launch configuration"}
+    if cnt_ok:
         inst = cnt["warp_inst_per_point"] * m
         issue_peak = nsm * 4 * sm_mhz * 1e6 / 1e9  # warp instructions per ns -> G/s
         roofline = {"bound": "alu", "roof": "warp-instruction issue (ALU, LSU and branch instructions all issue here)",
                     "achieved": round(inst / (kms / 1e3) / 1e9, 1), "peak": round(issue_peak, 1),
                     "unit": "Gwarp-inst/s", "frac": round(inst / (kms / 1e3) / 1e9 / issue_peak, 4),
                     "inst_per_launch": int(inst),
-                    "achieved_def": f"ncu smsp__inst_executed of this kernel source ({cnt['round']}) / live kernel time",
+                    "achieved_def": f"ncu smsp__inst_executed of this kernel source and workload "
+                                    f"({args.workload}, {cnt['round']}) / live kernel time",
                     "peak_def": f"{nsm} SMs x 4 schedulers x 1 warp-inst/clk x {sm_mhz:.0f} MHz (B200_PROFILING)",
-                    **common, "hbm_effective": hbm_eff}
+                    **common, "hbm_effective": hbm_eff, "node_fetch": node_fetch}
     else:
-        roofline = {**hbm_eff, **common, "issue": None,
-                    "note": "no ncu instruction count for this kernel source: HBM-effective roofline only"}
+        roofline = {**hbm_eff, **common, "issue": None, "node_fetch": node_fetch,
+                    "note": "no ncu instruction count for this kernel source / workload: HBM-effective roofline only"}
     # L2-latency roof (live): a lockstep step is one 32-B record load whose
     # address comes from the previous record; tt_diag_chase runs that pure
     # dependent chase over as many records as the tree has nodes, with the
@@ -717,7 +878,9 @@ def run_ours(args, rank, world, local_rank):
         if visits and lock_frac > 0.99 else None,
         "warp_tile_points": tile_pts,
         "traverse_ms": kms, "upload_ms": upload_ms, "tree_build_ms": build_ms, "tree_build": build_where,
-        "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": (launches or 0) * args.steps,
+        "bcast_ms": bcast_ms, "placement_ms": placement_ms, "allgather_ms": allgather_ms,
+        "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "strong_16m": strong,
+        "gpu_launches": (launches or 0) * args.steps,
         "gpu_launches_per_step": launches,
         "clocks": clocks,
     }

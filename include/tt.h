@@ -182,6 +182,12 @@ tt_status tt_build_nn_device(const float *pts, int64_t n, int32_t dim, int32_t l
 /* Copy the packed device blob back to host memory (bytes >= device_bytes of
  * tt_tree_get_info); synchronous.  E.g. to checkpoint a tree.              */
 tt_status tt_tree_download(const tt_tree *t, void *host_blob, size_t bytes);
+/* Copy the packed blob to caller-owned memory: mem = TT_MEM_HOST (host, like
+ * tt_tree_download; synchronous) or TT_MEM_DEVICE (device, asynchronous on
+ * `s`) -- e.g. the send buffer of the NCCL broadcast of a GPU-built tree
+ * (§8(e)), adopted on the other ranks with tt_tree_from_blob(DEVICE).
+ * Errors: TT_ERR_INVALID_ARG (null, bytes < device_bytes, bad mem), TT_ERR_CUDA. */
+tt_status tt_tree_copy_blob(const tt_tree *t, void *dst, size_t bytes, int32_t mem, tt_stream s);
 tt_status tt_tree_free(tt_tree *t);
 
 typedef struct tt_tree_info {
@@ -263,7 +269,11 @@ typedef struct tt_traverse_opts {
                                 path) fewer than 8 times (0 = always lockstep,
                                 >= 64 = never); -1 = kernel default, measured on
                                 B200: BH 3, kNN 4, VP 4, PC never
-                                (10k-point PC is latency-bound: independent wins) */
+                                (10k-point PC is latency-bound: independent wins);
+                                PC AUTO with the default threshold and fewer
+                                32-point tiles than resident warps (SMs x 32)
+                                splits each point's walk over 16 lanes
+                                (TT_VARIANT_SPLIT; warp_* stats left untouched) */
     const uint32_t *order;   /* [n] device, nullable: lane j of the launch processes
                                 point order[j] (e.g. perm from tt_sort_points);
                                 results still go to the point's own slot        */
@@ -389,6 +399,13 @@ tt_status tt_kick_drift_permuted(const float *bodies, const float *vel, const fl
  * TT_ERR_INVALID_ARG, TT_ERR_CUDA.                                        */
 tt_status tt_diag_chase(const void *records, int64_t nrec, int32_t per_lane, int64_t steps, int32_t ctas_per_sm,
                         uint32_t *sink, tt_stream s);
+/* The L2 read-bandwidth ceiling: 8 x 256-thread CTAs per SM read `bytes`
+ * (a multiple of 32, smaller than L2 to be L2-resident) of `buf` `reps`
+ * times with ld.global.cg (L2 only, not L1), 32 B per thread per
+ * iteration; bytes * reps / time = L2 read GB/s.  buf: device, 32-B
+ * aligned; sink as above.  Asynchronous; the caller times it.
+ * Errors: TT_ERR_INVALID_ARG, TT_ERR_CUDA.                                 */
+tt_status tt_diag_l2read(const void *buf, int64_t bytes, int32_t reps, uint32_t *sink, tt_stream s);
 
 /* ------------------------------------------------------------------------ */
 const char *tt_status_string(tt_status s);

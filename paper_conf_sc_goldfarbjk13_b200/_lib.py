@@ -87,6 +87,7 @@ SIGNATURES = {
     "tt_build_vp_device": (I32, [P, I64, I32, I32, P, P]),
     "tt_build_nn_device": (I32, [P, I64, I32, I32, P, P]),
     "tt_tree_download": (I32, [P, P, SZ]),
+    "tt_tree_copy_blob": (I32, [P, P, SZ, I32, P]),
     "tt_kick_drift": (I32, [P, P, P, I64, F, F, P]),
     "tt_kick_drift_permuted": (I32, [P, P, P, P, P, I64, F, F, P, P, P, P]),
     "tt_tree_free": (I32, [P]),
@@ -99,6 +100,7 @@ SIGNATURES = {
     "tt_traverse_vp": (I32, [P, P, I64, I32, P, P, P, P]),
     "tt_traverse_nn": (I32, [P, P, I64, I32, P, P, P, P]),
     "tt_diag_chase": (I32, [P, I64, I32, I64, I32, P, P]),
+    "tt_diag_l2read": (I32, [P, I64, I32, P, P]),
     "tt_status_string": (C.c_char_p, [I32]),
     "tt_last_cuda_error": (I32, []),
     "tt_build_info": (C.c_char_p, []),

@@ -45,7 +45,33 @@ __global__ void __launch_bounds__(256, 4) chase_kernel(const unsigned char *rec,
     if (acc == 0x9e3779b9u) sink[0] = acc;  // keep the loads (practically never taken)
 }
 
+// L2-resident streaming read: every thread reads 32 B per iteration with two
+// ld.global.cg (cached in L2 only, not L1) over `nvec` 32-B vectors,
+// grid-strided, `reps` times.  A buffer smaller than L2 is then read from L2:
+// bytes / time is the L2 read bandwidth the traversal's record fetches draw on.
+__global__ void __launch_bounds__(256) l2read_kernel(const float4 *buf, long long nvec, int reps, unsigned *sink) {
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    float acc = 0.f;
+    for (int r = 0; r < reps; ++r) {
+#pragma unroll 4
+        for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < nvec; i += stride) {
+            const float4 a = __ldcg(buf + 2 * i), b = __ldcg(buf + 2 * i + 1);
+            acc += (a.x + a.y) + (a.z + a.w) + (b.x + b.y) + (b.z + b.w);
+        }
+    }
+    if (acc == 1.2345e-7f) sink[0] = __float_as_uint(acc);  // keep the loads
+}
+
 }  // namespace
+
+int tt_launch_l2read(const void *buf, long long bytes, int reps, unsigned *sink, void *stream) {
+    int dev = 0, nsm = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    l2read_kernel<<<(unsigned)(nsm * 8), 256, 0, (cudaStream_t)stream>>>(static_cast<const float4 *>(buf), bytes / 32,
+                                                                         reps, sink);
+    return (int)cudaGetLastError();
+}
 
 int tt_launch_chase(const void *rec, long long nrec, long long steps, int per_lane, int ctas_per_sm, unsigned *sink,
                     void *stream) {

@@ -449,6 +449,18 @@ tt_status tt_tree_download(const tt_tree *t, void *host_blob, size_t bytes) {
     return e == cudaSuccess ? TT_OK : cuda_fail(e);
 }
 
+tt_status tt_tree_copy_blob(const tt_tree *t, void *dst, size_t bytes, int32_t mem, tt_stream s) {
+    if (!t || !dst || bytes < t->bytes || (mem != TT_MEM_HOST && mem != TT_MEM_DEVICE)) return TT_ERR_INVALID_ARG;
+    cudaError_t e;
+    if (mem == TT_MEM_HOST) {
+        e = cudaMemcpyAsync(dst, t->d_blob, t->bytes, cudaMemcpyDeviceToHost, (cudaStream_t)s);
+        if (e == cudaSuccess) e = cudaStreamSynchronize((cudaStream_t)s);
+    } else {
+        e = cudaMemcpyAsync(dst, t->d_blob, t->bytes, cudaMemcpyDeviceToDevice, (cudaStream_t)s);
+    }
+    return e == cudaSuccess ? TT_OK : cuda_fail(e);
+}
+
 tt_status tt_tree_upload(const tt_tree_desc *d, tt_stream s, tt_tree **out) {
     if (!out) return TT_ERR_INVALID_ARG;
     size_t bytes = 0;
@@ -610,6 +622,23 @@ tt_status tt_traverse_pc(const tt_tree *t, const float *q, int64_t n, int32_t ld
     p.r2 = radius * radius;  // rn(r*r), reading R1
     p.count = count_out;
     if (cfg.variant == TT_VARIANT_GROUPS || cfg.variant == TT_VARIANT_ROPES) return TT_ERR_UNSUPPORTED;  // BH only
+    // AUTO with the default threshold: a launch with fewer 32-point tiles than
+    // resident warps (148 SMs x 32) cannot fill the GPU one lane per point --
+    // it is the latency of its longest walks -- so each point's walk is split
+    // over 16 lanes (TT_VARIANT_SPLIT; configs[0]: 0.10 vs
+    // 0.18 ms)
+    const bool default_amd = !opts || opts->auto_min_depth < 0;
+    if (cfg.variant == TT_VARIANT_AUTOROPES && p.c.mode == TT_MODE_AUTO && default_amd) {
+        static std::atomic<int> s_nsm{0};
+        int nsm = s_nsm.load();
+        if (nsm == 0) {
+            int dev = 0;
+            cudaGetDevice(&dev);
+            cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+            s_nsm.store(nsm);
+        }
+        if ((n + 31) / 32 < (int64_t)nsm * 32) cfg.variant = TT_VARIANT_SPLIT;
+    }
     return finish_launch(cfg.variant == TT_VARIANT_RECURSIVE ? tt_launch_pc_recursive(p, t->hdr.dim, cfg)
                          : cfg.variant == TT_VARIANT_STACK   ? tt_launch_pc_stack(p, t->hdr.dim, cfg)
                          : cfg.variant == TT_VARIANT_SPLIT   ? tt_launch_pc_split(p, t->hdr.dim, cfg)
@@ -696,6 +725,14 @@ tt_status tt_diag_chase(const void *records, int64_t nrec, int32_t per_lane, int
     tt_status st = have_device();
     if (st != TT_OK) return st;
     const int e = tt_launch_chase(records, nrec, steps, per_lane, ctas_per_sm, sink, s);
+    return e ? cuda_fail((cudaError_t)e) : TT_OK;
+}
+
+tt_status tt_diag_l2read(const void *buf, int64_t bytes, int32_t reps, uint32_t *sink, tt_stream s) {
+    if (!buf || !sink || bytes < 32 || reps < 1 || !aligned(buf, 32)) return TT_ERR_INVALID_ARG;
+    tt_status st = have_device();
+    if (st != TT_OK) return st;
+    const int e = tt_launch_l2read(buf, bytes, reps, sink, s);
     return e ? cuda_fail((cudaError_t)e) : TT_OK;
 }
 

@@ -217,6 +217,7 @@ int tt_build_vp_gpu_impl(const float *pts, long long n, int dim, int ld, void *s
                          void **blob);
 
 // Diagnostics (kern_diag.cu): dependent 32-B record chase.
+int tt_launch_l2read(const void *buf, long long bytes, int reps, unsigned *sink, void *stream);
 int tt_launch_chase(const void *rec, long long nrec, long long steps, int per_lane, int ctas_per_sm, unsigned *sink,
                     void *stream);
 

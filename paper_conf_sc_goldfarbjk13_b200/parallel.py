@@ -63,6 +63,27 @@ def broadcast_tree(host_tree, device, src: int = 0, group=None):
     return tt_tree_from_blob(buf)
 
 
+def broadcast_device_tree(tree, device, src: int = 0, group=None):
+    """Rank `src` passes a device Tree (e.g. built on the GPU with
+    tt_build_oct_device), the others None: its packed blob is copied device
+    to device into a send buffer (tt_tree_copy_blob), broadcast as bytes and
+    adopted on the other ranks (tt_tree_from_blob, DEVICE).  Rank `src`
+    keeps its own tree."""
+    from .tt import tt_tree_copy_blob, tt_tree_from_blob  # GPU path only
+    rank = dist.get_rank(group)
+    wire = _wire(device, group)
+    size = torch.zeros(1, dtype=torch.int64, device=wire)
+    if rank == src:
+        size[0] = int(tree.device_bytes)
+    dist.broadcast(size, src, group=group)
+    if rank == src:
+        buf = tt_tree_copy_blob(tree).to(wire)
+    else:
+        buf = torch.empty(int(size.item()), dtype=torch.uint8, device=wire)
+    dist.broadcast(buf, src, group=group)
+    return tree if rank == src else tt_tree_from_blob(buf.to(device))
+
+
 def allgather_rows(full: torch.Tensor, world: int, group=None) -> torch.Tensor:
     """In-place all-gather of equal-size contiguous row shards of `full`
     (rank r owns rows shard_range(n, r, world)); needs n % (64 * world) == 0."""

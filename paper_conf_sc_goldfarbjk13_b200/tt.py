@@ -24,7 +24,8 @@ __all__ = [
     "HostTree", "Tree", "Stats", "TTError",
     "build_kd", "build_oct", "build_vp", "build_nn", "tt_tree_pack", "tt_tree_from_blob", "tt_tree_upload",
     "tt_build_oct_device", "tt_build_kd_device", "tt_build_vp_device", "tt_build_nn_device", "tt_tree_download",
-    "tt_sort_points", "tt_schedule_tiles", "tt_traverse_bh", "tt_traverse_pc", "tt_traverse_knn", "tt_traverse_vp", "tt_traverse_nn", "chase_records", "tt_diag_chase",
+    "tt_tree_copy_blob",
+    "tt_sort_points", "tt_schedule_tiles", "tt_traverse_bh", "tt_traverse_pc", "tt_traverse_knn", "tt_traverse_vp", "tt_traverse_nn", "chase_records", "tt_diag_chase", "tt_diag_l2read",
     "build_info",
 ]
 
@@ -234,6 +235,18 @@ def tt_build_vp_device(pts: torch.Tensor, stream=None) -> Tree:
     check(L.load().tt_build_vp_device(pts.data_ptr(), pts.shape[0], pts.shape[1], pts.stride(0),
                                       C.c_void_p(_stream_handle(stream)), C.byref(h)), "tt_build_vp_device")
     return Tree(h)
+
+
+def tt_tree_copy_blob(tree: Tree, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """The packed device blob copied into a CUDA uint8 tensor (device to
+    device, async on the stream): the send buffer of a tree broadcast."""
+    if out is None:
+        out = torch.empty(tree.device_bytes, dtype=torch.uint8, device="cuda")
+    if not out.is_cuda or out.dtype != torch.uint8 or not out.is_contiguous():
+        raise ValueError("out must be a contiguous CUDA uint8 tensor")
+    check(L.load().tt_tree_copy_blob(tree._h, C.c_void_p(out.data_ptr()), out.numel(), L.MEM_DEVICE,
+                                     C.c_void_p(_stream_handle(stream))), "tt_tree_copy_blob")
+    return out
 
 
 def tt_tree_download(tree: Tree) -> np.ndarray:
@@ -449,3 +462,14 @@ def tt_diag_chase(records: torch.Tensor, steps: int, per_lane: bool = False, cta
     check(L.load().tt_diag_chase(records.data_ptr(), records.shape[0], int(bool(per_lane)), int(steps),
                                  int(ctas_per_sm), sink.data_ptr(), C.c_void_p(_stream_handle(stream))),
           "tt_diag_chase")
+
+
+def tt_diag_l2read(buf: torch.Tensor, reps: int, stream=None) -> None:
+    """L2-resident streaming read of `buf` (the L2 read-bandwidth ceiling;
+    include/tt.h).  Asynchronous; time it."""
+    if not buf.is_cuda or not buf.is_contiguous():
+        raise ValueError("buf must be a contiguous CUDA tensor")
+    sink = torch.zeros(1, dtype=torch.int32, device=buf.device)
+    nbytes = buf.numel() * buf.element_size() // 32 * 32
+    check(L.load().tt_diag_l2read(buf.data_ptr(), nbytes, int(reps), sink.data_ptr(),
+                                  C.c_void_p(_stream_handle(stream))), "tt_diag_l2read")

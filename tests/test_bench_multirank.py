@@ -1,0 +1,54 @@
+"""bench.py under torchrun with 2 ranks (the driver's N > 1 launch), on the
+gloo wire so both ranks can share one GPU: the JSON line, the fixed-config
+strong-scaling block (configs[4] shape, shrunk) and the separately reported
+broadcast / placement / all-gather times."""
+from __future__ import annotations
+
+import json
+import os
+import socket
+import subprocess
+import sys
+
+import pytest
+import torch
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def _torchrun(extra, env_extra=None, timeout=600):
+    env = dict(os.environ, TT_DIST_BACKEND="gloo", **(env_extra or {}))
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+           "--master-addr=127.0.0.1", f"--master-port={_free_port()}", os.path.join(ROOT, "bench.py"),
+           "--gpus", "2"] + extra
+    return subprocess.run(cmd, cwd=ROOT, env=env, capture_output=True, text=True, timeout=timeout)
+
+
+@pytest.mark.gpu
+def test_bench_two_ranks_line():
+    r = _torchrun(["--steps", "2", "--warmup", "3", "--points-per-rank", "64000", "--strong-points", "256000",
+                   "--no-cpu-baseline", "--no-e2e", "--no-chase"])
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, r.stdout  # rank 0 alone prints
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["value"] > 0 and d["scaling"] == "weak"
+    assert d["config"]["global_points"] == 128000
+    assert d["bcast_ms"] is not None and d["placement_ms"] is not None and d["allgather_ms"] is not None
+    s = d["strong_16m"]
+    assert s["scaling"] == "strong" and s["points"] == 256000 and s["points_per_rank"] == 128000
+    assert s["value"] > 0 and s["bcast_ms"] is not None and s["allgather_ms"] is not None
+
+
+@pytest.mark.gpu
+def test_bench_uneven_shards_fail_loudly():
+    r = _torchrun(["--steps", "1", "--warmup", "3", "--points-per-rank", "64000", "--strong-points", "100001",
+                   "--no-cpu-baseline", "--no-e2e", "--no-chase"])
+    assert r.returncode != 0
+    assert "equal warp-aligned shards" in (r.stdout + r.stderr)
