@@ -582,9 +582,25 @@ tt_status tt_traverse_bh(const tt_tree *t, const float *bodies, const int32_t *s
                 return cuda_fail((cudaError_t)e);
             }
             mt->d_grp = g;
+            mt->grp_stream = s;
+            mt->grp_done = false;
         }
-        const cudaError_t e = cudaStreamWaitEvent((cudaStream_t)s, mt->grp_ready, 0);
-        if (e) return cuda_fail(e);
+        // a launch on another stream waits for the build until it is known
+        // complete (then no further calls: nothing to wait for, and no event
+        // wait inside a later CUDA-graph capture)
+        if (!mt->grp_done) {
+            const cudaError_t q = cudaEventQuery(mt->grp_ready);
+            if (q == cudaSuccess) {
+                mt->grp_done = true;
+            } else if (q == cudaErrorNotReady) {
+                if (s != mt->grp_stream) {
+                    const cudaError_t e = cudaStreamWaitEvent((cudaStream_t)s, mt->grp_ready, 0);
+                    if (e) return cuda_fail(e);
+                }
+            } else {
+                return cuda_fail(q);
+            }
+        }
     }
     p.bodies = reinterpret_cast<const float4 *>(bodies);
     p.self_ids = self_ids;

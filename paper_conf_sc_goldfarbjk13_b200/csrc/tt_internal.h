@@ -157,6 +157,8 @@ struct tt_tree {
     int32_t *d_pre = nullptr;  // canonical preorder id of every device node (stats hashes), built on first use
     void *d_grp = nullptr;  // OCT: child-group records (kern_bh_group.cu), built on first use
     cudaEvent_t grp_ready = nullptr;  // recorded on the stream of that build
+    tt_stream grp_stream = nullptr;   // the stream of that build
+    bool grp_done = false;            // the build is known complete
     std::mutex grp_mu;
 };
 
