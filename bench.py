@@ -376,7 +376,7 @@ def run_reference(args, rank, world):
 # ------------------------------------------------------------------- ours
 def run_bh_steps(args, rank, world):
     """NEXT-4 workload: a bench step = one BH time step of configs[1]
-    (tt_build_oct_device + tt_sort_points + tt_traverse_bh + tt_kick_drift_permuted,
+    (tt_build_oct_device_order (tree + tree order) + tt_traverse_bh + tt_kick_drift_permuted,
     + all-gather of positions / velocities / ids for N > 1).  Strong scaling:
     the same 1M-body system on every N; each rank integrates its warp-aligned
     shard of the sorted order (nbody.simulate_sharded)."""
@@ -417,7 +417,7 @@ def run_bh_steps(args, rank, world):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": "bh_1m_plummer time steps", "bodies": n, "dt": dt,
-                       "step": "GPU build + sort + force (own shard) + gathered kick-drift (leapfrog KDK)"
+                       "step": "GPU build (+ tree order) + force (own shard) + gathered kick-drift (leapfrog KDK)"
                                + (" + all-gather of x, v, ids" if world > 1 else ""),
                        "parallelism": f"dp{world} (bodies sharded by sorted order, tree rebuilt on every rank)",
                        "params": c, "l2": "not flushed: a time step rewrites the bodies and rebuilds the tree"},

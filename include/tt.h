@@ -166,6 +166,14 @@ tt_status tt_tree_upload(const tt_tree_desc *d, tt_stream s, tt_tree **out);
  * (build rules R8a/R9).  Synchronises `s`.  Errors: TT_ERR_INVALID_ARG,
  * TT_ERR_TREE_TOO_DEEP (never for R9 trees: height <= 33), TT_ERR_CUDA/OOM. */
 tt_status tt_build_oct_device(const float *bodies, int64_t n, tt_stream s, tt_tree **out);
+/* The same build, also writing the bodies' tree order: order_out (device,
+ * n uint32, nullable) = body indices in leaf preorder (Fig.2 order of the
+ * leaves; the bodies of a depth-32 bucket by index, R9) -- the order the
+ * build has already sorted them into, so a time step can traverse in it
+ * without a separate tt_sort_points (§4.4: any order that makes
+ * neighbouring traversals similar; this one refines the 63-bit key of
+ * tt_sort_points to all 32 levels).  Synchronises `s` twice.               */
+tt_status tt_build_oct_device_order(const float *bodies, int64_t n, uint32_t *order_out, tt_stream s, tt_tree **out);
 /* NEXT-1: build a kd-tree (median splits, reading R3) on the GPU from device
  * points (n rows of `ld` floats, dim <= TT_MAX_DIM) straight into the packed
  * device layout -- the bytes tt_tree_pack produces for tt_build_kd.

@@ -83,6 +83,7 @@ SIGNATURES = {
     "tt_tree_from_blob": (I32, [P, SZ, I32, P, P]),
     "tt_tree_upload": (I32, [P, P, P]),
     "tt_build_oct_device": (I32, [P, I64, P, P]),
+    "tt_build_oct_device_order": (I32, [P, I64, P, P, P]),
     "tt_build_kd_device": (I32, [P, I64, I32, I32, I32, P, P]),
     "tt_build_vp_device": (I32, [P, I64, I32, I32, P, P]),
     "tt_build_nn_device": (I32, [P, I64, I32, I32, P, P]),

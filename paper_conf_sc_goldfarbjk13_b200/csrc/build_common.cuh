@@ -57,22 +57,28 @@ __global__ void level_assign_kernel(const int *level, const int *rank, long long
 // Fill h.height / top_levels / top_count / level_prefix from the node levels
 // (same plan as pack.cpp for `stage_bytes` per staged node) and compute the
 // device index newidx[v] of every canonical (preorder) node v.
+// known_hist (nullable): the level histogram, already on the host (no sync).
 inline cudaError_t renumber_top_first(const int *level, long long nn, int stage_bytes, tt_blob_header &h,
-                                      int *newidx, Scratch &W) {
+                                      int *newidx, Scratch &W, const unsigned *known_hist = nullptr) {
     cudaStream_t s = W.s;
     const unsigned GN = build_grid(nn);
-    unsigned *hist = W.get<unsigned>(64);
     int *flag = W.get<int>(nn + 1), *rank = W.get<int>(nn + 1);
     size_t sb = 0;
     cub::DeviceScan::ExclusiveSum(nullptr, sb, flag, rank, (int)nn, s);
     void *st = W.get<unsigned char>(sb);
     if (W.e) return W.e;
     cudaError_t e;
-    if ((e = cudaMemsetAsync(hist, 0, 64 * sizeof(unsigned), s))) return e;
-    level_hist_kernel<<<GN, 256, 0, s>>>(level, nn, hist);
     unsigned hh[64];
-    if ((e = cudaMemcpyAsync(hh, hist, sizeof(hh), cudaMemcpyDeviceToHost, s))) return e;
-    if ((e = cudaStreamSynchronize(s))) return e;
+    if (known_hist) {
+        std::memcpy(hh, known_hist, sizeof(hh));
+    } else {
+        unsigned *hist = W.get<unsigned>(64);
+        if (W.e) return W.e;
+        if ((e = cudaMemsetAsync(hist, 0, 64 * sizeof(unsigned), s))) return e;
+        level_hist_kernel<<<GN, 256, 0, s>>>(level, nn, hist);
+        if ((e = cudaMemcpyAsync(hh, hist, sizeof(hh), cudaMemcpyDeviceToHost, s))) return e;
+        if ((e = cudaStreamSynchronize(s))) return e;
+    }
     int height = 0;
     for (int l = 0; l < 64; ++l)
         if (hh[l]) height = l;

@@ -62,8 +62,35 @@ struct Cube {
     double c[3], side;
 };
 
-__global__ void digits_kernel(const float4 *b, long long n, Cube cube, unsigned long long *k0, unsigned long long *k1,
-                              unsigned *ids) {
+// What the host needs from the device, read back with ONE synchronisation:
+// the root cube (header), the node count (allocation sizes) and the level
+// histogram (top-levels-first plan).
+struct BuildInfo {
+    Cube cube;
+    int n_nodes, pad;
+    unsigned hist[64];
+};
+
+__global__ void box_init_kernel(float *box) {
+    if (threadIdx.x < 6) box[threadIdx.x] = threadIdx.x < 3 ? INFINITY : -INFINITY;
+}
+
+// root cube from the fp32 bounding box, in fp64 (R8a): centre = midpoint,
+// side = max extent (1 for a single point)
+__global__ void cube_kernel(const float *box, BuildInfo *info) {
+    if (threadIdx.x == 0) {
+        double side = 0.0;
+        for (int d = 0; d < 3; ++d) {
+            info->cube.c[d] = ((double)box[d] + (double)box[3 + d]) * 0.5;
+            side = fmax(side, (double)box[3 + d] - (double)box[d]);
+        }
+        info->cube.side = side == 0.0 ? 1.0 : side;
+    }
+}
+
+__global__ void digits_kernel(const float4 *b, long long n, const BuildInfo *info, unsigned long long *k0,
+                              unsigned long long *k1, unsigned *ids) {
+    const Cube cube = info->cube;
     for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
         const float4 p = b[i];
         const double x = p.x, y = p.y, z = p.z;
@@ -98,15 +125,29 @@ __device__ __forceinline__ int common_digits(unsigned long long a0, unsigned lon
 
 // d[i] = common digits of sorted bodies i and i+1 (-1 for the last); cnt[i] =
 // nodes started by body i.
+// ... and the level histogram of the nodes emit_kernel will write (cells at
+// levels dprev+1 .. min(dnext, 32), the leaf at max(dprev, dnext) + 1)
 __global__ void count_kernel(const unsigned long long *k0, const unsigned long long *k1, long long n, int *dn,
-                             int *cnt) {
+                             int *cnt, unsigned *hist) {
+    __shared__ unsigned sh[64];
+    if (threadIdx.x < 64) sh[threadIdx.x] = 0;
+    __syncthreads();
     for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
         const int dprev = i > 0 ? common_digits(k0[i - 1], k1[i - 1], k0[i], k1[i]) : -1;
         const int dnext = i + 1 < n ? common_digits(k0[i], k1[i], k0[i + 1], k1[i + 1]) : -1;
         dn[i] = dnext;
-        const int cells = max(0, min(dnext, kMaxDepth) - dprev);
+        const int top = min(dnext, kMaxDepth);
+        const int cells = max(0, top - dprev);
         cnt[i] = cells + 1;
+        for (int L = dprev + 1; L <= top; ++L) atomicAdd(sh + L, 1u);
+        atomicAdd(sh + min(max(dprev, dnext) + 1, kMaxDepth + 1), 1u);
     }
+    __syncthreads();
+    if (threadIdx.x < 64 && sh[threadIdx.x]) atomicAdd(hist + threadIdx.x, sh[threadIdx.x]);
+}
+
+__global__ void info_count_kernel(const int *base, long long n, BuildInfo *info) {
+    if (threadIdx.x == 0) info->n_nodes = base[n];
 }
 
 struct NodeArrays {
@@ -214,39 +255,34 @@ __global__ void gather_u64(const unsigned long long *src, const unsigned *perm, 
 }  // namespace
 
 // Build on `stream`: writes the host copy of the blob header and a cudaMalloc'd
-// device blob (caller owns it).  Synchronises the stream twice (the bounding
-// box and the node count / level histogram are needed on the host).
+// device blob (caller owns it).  Synchronises the stream twice: once to read
+// the root cube, node count and level histogram (one struct), once at the
+// end.  order_out (nullable, device [n]): the bodies' tree order (leaf
+// preorder), i.e. the sorted ids of step 2.
 int tt_build_oct_gpu_impl(const float *bodies_f, long long n, void *stream, tt_blob_header *hdr_out,
-                          void **blob_out) {
+                          void **blob_out, unsigned *order_out) {
     cudaStream_t s = (cudaStream_t)stream;
     const float4 *bodies = reinterpret_cast<const float4 *>(bodies_f);
     tt_keep_pool_memory();
     Scratch W{s};
     const unsigned G = build_grid(n);
 
-    // 1. root cube
+    // 1. root cube (on the device)
     float *d_box = W.get<float>(6);
-    float hbox[6] = {INFINITY, INFINITY, INFINITY, -INFINITY, -INFINITY, -INFINITY};
+    BuildInfo *d_info = W.get<BuildInfo>(1);
     if (W.e) return W.e;
-    cudaError_t e = cudaMemcpyAsync(d_box, hbox, sizeof(hbox), cudaMemcpyHostToDevice, s);
+    cudaError_t e = cudaMemsetAsync(d_info, 0, sizeof(BuildInfo), s);
     if (e) return e;
+    box_init_kernel<<<1, 32, 0, s>>>(d_box);
     bbox_kernel<<<G, 256, 0, s>>>(bodies, n, d_box);
-    if ((e = cudaMemcpyAsync(hbox, d_box, sizeof(hbox), cudaMemcpyDeviceToHost, s))) return e;
-    if ((e = cudaStreamSynchronize(s))) return e;
-    Cube cube;
-    double side = 0.0;
-    for (int d = 0; d < 3; ++d) {
-        cube.c[d] = ((double)hbox[d] + (double)hbox[3 + d]) * 0.5;
-        side = std::fmax(side, (double)hbox[3 + d] - (double)hbox[d]);
-    }
-    cube.side = side == 0.0 ? 1.0 : side;
+    cube_kernel<<<1, 32, 0, s>>>(d_box, d_info);
 
     // 2. digits + stable sort by (digits, id)
     auto *k0 = W.get<unsigned long long>(n), *k1 = W.get<unsigned long long>(n);
     auto *kt = W.get<unsigned long long>(n), *kt2 = W.get<unsigned long long>(n);
     auto *ids = W.get<unsigned>(n), *ids_t = W.get<unsigned>(n), *ids_s = W.get<unsigned>(n);
     if (W.e) return W.e;
-    digits_kernel<<<G, 256, 0, s>>>(bodies, n, cube, k0, k1, ids);
+    digits_kernel<<<G, 256, 0, s>>>(bodies, n, d_info, k0, k1, ids);
     size_t b1 = 0, b2 = 0;
     cub::DeviceRadixSort::SortPairs(nullptr, b1, k1, kt, ids, ids_t, (int)n, 0, 33, s);
     cub::DeviceRadixSort::SortPairs(nullptr, b2, kt, kt2, ids_t, ids_s, (int)n, 0, 63, s);
@@ -261,21 +297,28 @@ int tt_build_oct_gpu_impl(const float *bodies_f, long long n, void *stream, tt_b
     if (W.e) return W.e;
     gather_u64<<<G, 256, 0, s>>>(k0, ids_s, n, k0s);
     gather_u64<<<G, 256, 0, s>>>(k1, ids_s, n, k1s);
+    if (order_out && (e = cudaMemcpyAsync(order_out, ids_s, sizeof(unsigned) * (size_t)n, cudaMemcpyDeviceToDevice, s)))
+        return e;
 
-    // 3. node counts per body, preorder bases
+    // 3. node counts per body (and the level histogram), preorder bases
     int *dn = W.get<int>(n), *cnt = W.get<int>(n + 1), *base = W.get<int>(n + 1);
     if (W.e) return W.e;
-    count_kernel<<<G, 256, 0, s>>>(k0s, k1s, n, dn, cnt);
+    count_kernel<<<G, 256, 0, s>>>(k0s, k1s, n, dn, cnt, d_info->hist);
     if ((e = cudaMemsetAsync(cnt + n, 0, sizeof(int), s))) return e;
     size_t sb = 0;
     cub::DeviceScan::ExclusiveSum(nullptr, sb, cnt, base, (int)(n + 1), s);
     void *st = W.get<unsigned char>(sb);
     if (W.e) return W.e;
     if ((e = cub::DeviceScan::ExclusiveSum(st, sb, cnt, base, (int)(n + 1), s))) return e;
-    int nn = 0;
-    if ((e = cudaMemcpyAsync(&nn, base + n, sizeof(int), cudaMemcpyDeviceToHost, s))) return e;
+    info_count_kernel<<<1, 32, 0, s>>>(base, n, d_info);
+    BuildInfo info;
+    if ((e = cudaMemcpyAsync(&info, d_info, sizeof(info), cudaMemcpyDeviceToHost, s))) return e;
     if ((e = cudaStreamSynchronize(s))) return e;
-    const long long n_nodes = nn;
+    const long long n_nodes = info.n_nodes;
+    const Cube cube = info.cube;
+    int height = 0;
+    for (int l = 0; l < 64; ++l)
+        if (info.hist[l]) height = l;
 
     // 4. nodes in preorder
     NodeArrays A;
@@ -285,18 +328,9 @@ int tt_build_oct_gpu_impl(const float *bodies_f, long long n, void *stream, tt_b
     A.body = W.get<int>(n_nodes);
     A.m0 = W.get<double>(n_nodes);
     A.m1 = W.get<double>(3 * n_nodes);
-    unsigned *hist = W.get<unsigned>(64);
     if (W.e) return W.e;
     const unsigned GN = build_grid(n_nodes);
     emit_kernel<<<G, 256, 0, s>>>(k0s, k1s, ids_s, dn, base, n, n_nodes, A);
-    if ((e = cudaMemsetAsync(hist, 0, 64 * sizeof(unsigned), s))) return e;
-    level_hist_kernel<<<GN, 256, 0, s>>>(A.level, n_nodes, hist);
-    unsigned hh[64];
-    if ((e = cudaMemcpyAsync(hh, hist, sizeof(hh), cudaMemcpyDeviceToHost, s))) return e;
-    if ((e = cudaStreamSynchronize(s))) return e;
-    int height = 0;
-    for (int l = 0; l < 64; ++l)
-        if (hh[l]) height = l;
 
     // 5. moments bottom-up
     for (int l = height; l >= 0; --l) moments_kernel<<<GN, 256, 0, s>>>(bodies, n_nodes, l, A);
@@ -312,7 +346,7 @@ int tt_build_oct_gpu_impl(const float *bodies_f, long long n, void *stream, tt_b
     h.oct_flags = (height <= 32 ? TT_OCT_NARROW : 0) | TT_OCT_FEW_CELL_KIDS;
     int *newidx = W.get<int>(n_nodes);
     if (W.e) return W.e;
-    if ((e = renumber_top_first(A.level, n_nodes, 32, h, newidx, W))) return e;
+    if ((e = renumber_top_first(A.level, n_nodes, 32, h, newidx, W, info.hist))) return e;
     h.off_rec = align256(sizeof(tt_blob_header));
     h.total = align256(h.off_rec + (uint64_t)n_nodes * 32);
     void *blob = nullptr;

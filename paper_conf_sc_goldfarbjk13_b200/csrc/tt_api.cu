@@ -375,12 +375,16 @@ tt_status tt_tree_from_blob(const void *blob, size_t bytes, int32_t mem, tt_stre
 }
 
 tt_status tt_build_oct_device(const float *bodies, int64_t n, tt_stream s, tt_tree **out) {
+    return tt_build_oct_device_order(bodies, n, nullptr, s, out);
+}
+
+tt_status tt_build_oct_device_order(const float *bodies, int64_t n, uint32_t *order_out, tt_stream s, tt_tree **out) {
     if (!bodies || !out || n <= 0 || n > INT32_MAX / 3 || !aligned(bodies, 16)) return TT_ERR_INVALID_ARG;
     tt_status st = have_device();
     if (st != TT_OK) return st;
     tt_blob_header h;
     void *d_blob = nullptr;
-    const int e = tt_build_oct_gpu_impl(bodies, n, s, &h, &d_blob);
+    const int e = tt_build_oct_gpu_impl(bodies, n, s, &h, &d_blob, order_out);
     if (e) return cuda_fail((cudaError_t)e);
     if (h.height > TT_MAX_HEIGHT) {
         tt_blob_discard(d_blob);

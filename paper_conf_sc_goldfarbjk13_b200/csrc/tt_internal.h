@@ -206,7 +206,8 @@ inline int tt_stage_count(const tt_blob_header &h, int bytes_per_node, int budge
 
 // GPU oct-tree build (build_oct_gpu.cu): fills the host header copy and a
 // cudaMalloc'd device blob; returns a cudaError_t.
-int tt_build_oct_gpu_impl(const float *bodies, long long n, void *stream, tt_blob_header *hdr, void **blob);
+int tt_build_oct_gpu_impl(const float *bodies, long long n, void *stream, tt_blob_header *hdr, void **blob,
+                          unsigned *order_out = nullptr);
 
 int tt_launch_kick_drift(float *x, float *v, const float *a, long long n, float dtk, float dtd, void *stream);
 int tt_launch_kick_drift_permuted(const float *x, const float *v, const float *a, const int *perm, const int *ids,

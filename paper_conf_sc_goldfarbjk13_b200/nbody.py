@@ -6,7 +6,7 @@ mass, runs the force traversal and advances the bodies.  Every stage here is
 a libtt call on the current stream (no host round trip besides the node
 count the GPU build reads back):
 
-    tt_build_oct_device -> tt_sort_points -> tt_traverse_bh -> tt_kick_drift
+    tt_build_oct_device_order (tree + the bodies' tree order) -> tt_traverse_bh -> tt_kick_drift
 
 Integration is leapfrog kick-drift-kick, with consecutive half kicks merged:
   step 0:     kick(dt/2) + drift(dt), force
@@ -29,7 +29,7 @@ import torch
 
 from . import _lib as L
 from ._lib import check
-from .tt import _dev, _stream_handle, tt_build_oct_device, tt_sort_points, tt_traverse_bh
+from .tt import _dev, _stream_handle, tt_build_oct_device_order, tt_traverse_bh
 
 
 def tt_kick_drift(bodies: torch.Tensor, vel: torch.Tensor, acc: torch.Tensor, dt_kick: float, dt_drift: float,
@@ -71,8 +71,8 @@ def tt_kick_drift_permuted(bodies: torch.Tensor, vel: torch.Tensor, acc: torch.T
 def forces(bodies: torch.Tensor, theta: float, eps: float, out: torch.Tensor | None = None, mode="auto",
            stats=None):
     """One force pass on the current positions: GPU build, sort, traverse."""
-    tree = tt_build_oct_device(bodies)
-    perm = tt_sort_points(tree, bodies)
+    # the build's own sort is the tree order: no separate tt_sort_points
+    tree, perm = tt_build_oct_device_order(bodies)
     acc = tt_traverse_bh(tree, bodies, theta, eps, out=out, order=perm, mode=mode, stats=stats)
     return acc, tree
 
@@ -115,11 +115,11 @@ def simulate_sharded(bodies: torch.Tensor, vel: torch.Tensor, ids: torch.Tensor,
     x, v, i = bodies, vel, ids
     xo, vo, io = torch.empty_like(x), torch.empty_like(v), torch.empty_like(i)
     acc = torch.empty_like(x)
+    order_buf = torch.empty(n, dtype=torch.int32, device=x.device)
 
     def half(dtk, dtd):
         nonlocal x, v, i, xo, vo, io
-        tree = tt_build_oct_device(x)
-        perm = tt_sort_points(tree, x)
+        tree, perm = tt_build_oct_device_order(x, order_buf)  # tree order from the build's sort
         mine = perm[lo:hi]
         tt_traverse_bh(tree, x, theta, eps, out=acc, order=mine, mode=mode)
         tt_kick_drift_permuted(x, v, acc, mine, dtk, dtd, xo[lo:hi], vo[lo:hi], i, io[lo:hi])

@@ -23,7 +23,7 @@ from ._lib import TTError, check
 __all__ = [
     "HostTree", "Tree", "Stats", "TTError",
     "build_kd", "build_oct", "build_vp", "build_nn", "tt_tree_pack", "tt_tree_from_blob", "tt_tree_upload",
-    "tt_build_oct_device", "tt_build_kd_device", "tt_build_vp_device", "tt_build_nn_device", "tt_tree_download",
+    "tt_build_oct_device", "tt_build_oct_device_order", "tt_build_kd_device", "tt_build_vp_device", "tt_build_nn_device", "tt_tree_download",
     "tt_tree_copy_blob",
     "tt_sort_points", "tt_schedule_tiles", "tt_traverse_bh", "tt_traverse_pc", "tt_traverse_knn", "tt_traverse_vp", "tt_traverse_nn", "chase_records", "tt_diag_chase", "tt_diag_l2read",
     "build_info",
@@ -197,6 +197,24 @@ def tt_tree_from_blob(blob, stream=None) -> Tree:
                                         C.byref(h))
     check(st, "tt_tree_from_blob")
     return Tree(h)
+
+
+def tt_build_oct_device_order(bodies: torch.Tensor, order: torch.Tensor | None = None, stream=None):
+    """tt_build_oct_device that also returns the bodies' tree order (leaf
+    preorder; an int32 device tensor usable as a traversal `order`)."""
+    _dev(bodies, torch.float32, "bodies", 4)
+    if bodies.shape[1] != 4 or not bodies.is_contiguous():
+        raise ValueError("bodies must be a contiguous (n, 4) float32 tensor")
+    n = bodies.shape[0]
+    if order is None:
+        order = torch.empty(n, dtype=torch.int32, device=bodies.device)
+    _dev(order, torch.int32, "order")
+    if order.numel() < n or not order.is_contiguous():
+        raise ValueError("order needs n contiguous int32 entries")
+    h = C.c_void_p()
+    check(L.load().tt_build_oct_device_order(bodies.data_ptr(), n, order.data_ptr(), C.c_void_p(_stream_handle(stream)),
+                                             C.byref(h)), "tt_build_oct_device_order")
+    return Tree(h), order
 
 
 def tt_build_oct_device(bodies: torch.Tensor, stream=None) -> Tree:

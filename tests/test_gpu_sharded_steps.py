@@ -108,3 +108,25 @@ def test_two_ranks_bit_identical_to_one():
         assert not isinstance(x, str), x
         assert np.array_equal(ids, i1), rank
         assert np.array_equal(x, x1) and np.array_equal(u, u1), rank
+
+
+@pytest.mark.parametrize("n,dup", [(1, 0), (3001, 0), (20011, 12), (1_000_000, 0)])
+def test_build_tree_order_equals_oracle(n, dup):
+    """tt_build_oct_device_order's order = the bodies in leaf preorder: the
+    oracle builder's tree order (R8a / R9: depth-32 buckets by index), and a
+    traversal in that order matches the oracle."""
+    import oracle
+    import paper_conf_sc_goldfarbjk13_b200 as P
+    b = ttgen.plummer(n, seed=500 + n % 97)
+    if dup:
+        b[10:10 + dup, :3] = b[2, :3]
+    ot = oracle.build_oct(b)
+    tree, order = P.tt_build_oct_device_order(dev(b))
+    assert np.array_equal(order.cpu().numpy(), ot.tree_order())
+    if n == 1:
+        assert np.all(P.tt_traverse_bh(tree, dev(b), 0.5, 0.05, order=order).cpu().numpy() == 0)
+    elif n <= 20011:
+        acc = P.tt_traverse_bh(tree, dev(b), 0.5, 0.05, order=order).cpu().numpy()
+        ref = oracle.bh(ot, b, 0.5, 0.05, self_ids=np.arange(n)).out[0]
+        err = np.linalg.norm(acc[:, :3] - ref, axis=1) / np.linalg.norm(ref, axis=1)
+        assert err.max() <= 1e-4
