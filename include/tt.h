@@ -149,7 +149,10 @@ tt_status tt_host_tree_desc(const tt_host_tree *t, tt_tree_desc *out);
  * Errors: TT_ERR_INVALID_ARG (inconsistent desc), TT_ERR_TREE_TOO_DEEP
  * (height > TT_MAX_HEIGHT), TT_ERR_UNSUPPORTED (dim > TT_MAX_DIM),
  * TT_ERR_OOM, TT_ERR_CUDA.  The returned tree owns its device memory until
- * tt_tree_free; it is read-only, so concurrent traversals are safe.      */
+ * tt_tree_free; it is read-only, so concurrent traversals are safe (each
+ * launch takes one of 256 per-tree tile-scheduler slots round-robin and
+ * frees it when its last CTA finishes: at most 256 launches of one tree may
+ * be in flight at once).                                                  */
 typedef struct tt_tree tt_tree;
 
 tt_status tt_tree_pack_size(const tt_tree_desc *d, size_t *bytes);
