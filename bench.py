@@ -773,7 +773,9 @@ def run_ours(args, rank, world, local_rank):
         qds, rds, pms = [q_dev, torch.empty_like(q_dev)], [res_dev, like(res_dev)], [perm, torch.empty_like(perm)]
         rhs = [res_host, tuple(torch.empty(x.shape, dtype=x.dtype).pin_memory() for x in res_host)
                if isinstance(res_host, tuple) else torch.empty(res_host.shape, dtype=res_host.dtype).pin_memory()]
-        cs = torch.cuda.Stream(device)
+        # separate H2D and D2H streams: the next step's H2D must not queue
+        # behind this step's D2H (which waits for this step's compute)
+        cs, ds = torch.cuda.Stream(device), torch.cuda.Stream(device)
         ev = lambda: torch.cuda.Event()  # noqa: E731
         h2d_done, comp_done, d2h_done = [ev(), ev()], [ev(), ev()], [ev(), ev()]
 
@@ -788,10 +790,10 @@ def run_ours(args, rank, world, local_rank):
             flush.zero_()
             api_step(qds[b_], rds[b_], pms[b_])
             comp_done[b_].record(stream)
-            with torch.cuda.stream(cs):
-                cs.wait_event(comp_done[b_])
+            with torch.cuda.stream(ds):
+                ds.wait_event(comp_done[b_])
                 to_host(rhs[b_], rds[b_])
-                d2h_done[b_].record(cs)
+                d2h_done[b_].record(ds)
 
         for i in range(4):
             pipe_step(i)
@@ -799,6 +801,7 @@ def run_ours(args, rank, world, local_rank):
         t_a, t_b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         t_a.record(stream)
         cs.wait_stream(stream)
+        ds.wait_stream(stream)
         for i in range(args.steps):
             pipe_step(i)
         for b_ in range(2):
@@ -815,7 +818,7 @@ def run_ours(args, rank, world, local_rank):
                "serial_ms_per_step": serial_ms,
                "note": "public API (tt_sort_points + tt_schedule_tiles + tt_traverse_*) from / to pinned host "
                        "buffers: every step copies its points in (H2D) and its results out (D2H); the copies run "
-                       "on a second stream, overlapping the neighbouring steps' compute (double-buffered); "
+                       "on two copy streams, overlapping the neighbouring steps' compute (double-buffered); "
                        "L2 flushed before each step's compute inside the timed region.  serial_ms_per_step: "
                        "the same with H2D, compute and D2H serialised on one stream"}
 

@@ -425,10 +425,13 @@ void *grp_take(size_t bytes) {
             }
         }
     }
+    // slack (1/8, in 2-MiB steps): the next time step's tree is a little
+    // larger or smaller and should still fit [bytes, 2 * bytes]
+    const size_t alloc = ((bytes + bytes / 8) + (2u << 20) - 1) & ~(size_t)((2u << 20) - 1);
     void *p = nullptr;
-    if (cudaMalloc(&p, bytes) != cudaSuccess) return nullptr;
+    if (cudaMalloc(&p, alloc) != cudaSuccess) return nullptr;
     std::lock_guard<std::mutex> lk(g_grp_mu);
-    g_grp_info[p] = GrpInfo{bytes, dev};
+    g_grp_info[p] = GrpInfo{alloc, dev};
     return p;
 }
 

@@ -272,11 +272,13 @@ int tt_blob_take(size_t bytes, void **out) {
             }
         }
     }
+    // slack (1/8, in 2-MiB steps) so the next time step's tree fits too
+    const size_t alloc = ((bytes + bytes / 8) + (2u << 20) - 1) & ~(size_t)((2u << 20) - 1);
     void *p = nullptr;
-    cudaError_t e = cudaMalloc(&p, bytes);
+    cudaError_t e = cudaMalloc(&p, alloc);
     if (e) return e;
     std::lock_guard<std::mutex> lk(g_blob_mu);
-    g_blob_info[p] = BlobInfo{bytes, dev};
+    g_blob_info[p] = BlobInfo{alloc, dev};
     *out = p;
     return cudaSuccess;
 }
