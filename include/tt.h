@@ -213,12 +213,14 @@ tt_status tt_tree_get_info(const tt_tree *t, tt_tree_info *out);
 
 /* ------------------------------------------------------------------------ */
 /* a1: point sort (§4.4).  Key = where the point's descent of the
- * tree by the build's split rule ends, in tree (preorder) order: kd -> the
- * leaf's first tree-order point; oct -> 63-bit octant path (Morton order,
- * equal to the preorder of leaves); vp -> 2-bit-per-level path code; nn ->
- * the same code of the left-iff-x[dim]<split descent.  A
+ * tree by the build's split rule ends: kd -> the leaf's first tree-order
+ * point (tree order); oct -> the index, along the 3-D Hilbert curve of the
+ * root cube, of the point's 21-level cell of the cube hierarchy (octant bits
+ * from the build's fp64 comparisons; reading R18b: more compact warp tiles
+ * than the Morton / leaf-preorder order); vp -> 2-bit-per-level path code;
+ * nn -> the same code of the left-iff-x[dim]<split descent.  A
  * stable radix sort of (key, index) gives perm: perm[j] = original index of
- * the j-th point in tree order (ties by index).  pts: device, n rows of `ld`
+ * the j-th point in key order (ties by index).  pts: device, n rows of `ld`
  * floats (OCT: ld >= 4 or 3).  keys_out (nullable): the keys, in input order.
  * Temporary device memory is taken stream-ordered (cudaMallocAsync).      */
 tt_status tt_sort_points(const tt_tree *t, const float *pts, int64_t n, int32_t ld,

@@ -27,24 +27,64 @@ __global__ void iota_kernel(uint32_t *v, long long n) {
         v[i] = (uint32_t)i;
 }
 
+// Hilbert index (Skilling's transpose algorithm) of the 21-level cell whose
+// coordinate bits are (ix, iy, iz), bits interleaved x, y, z from the top
+__device__ __forceinline__ unsigned long long hilbert21(unsigned ix, unsigned iy, unsigned iz) {
+    unsigned X[3] = {ix, iy, iz};
+#pragma unroll 1
+    for (unsigned Q = 1u << 20; Q > 1; Q >>= 1) {
+        const unsigned P = Q - 1;
+#pragma unroll
+        for (int i = 0; i < 3; ++i) {
+            if (X[i] & Q) {
+                X[0] ^= P;
+            } else {
+                const unsigned t = (X[0] ^ X[i]) & P;
+                X[0] ^= t;
+                X[i] ^= t;
+            }
+        }
+    }
+    X[1] ^= X[0];
+    X[2] ^= X[1];
+    unsigned t = 0;
+#pragma unroll 1
+    for (unsigned Q = 1u << 20; Q > 1; Q >>= 1)
+        if (X[2] & Q) t ^= Q - 1;
+    X[0] ^= t;
+    X[1] ^= t;
+    X[2] ^= t;
+    unsigned long long h = 0;
+#pragma unroll 1
+    for (int b = 20; b >= 0; --b)
+        h = (h << 3) | ((unsigned long long)((X[0] >> b) & 1u) << 2) | ((unsigned long long)((X[1] >> b) & 1u) << 1) |
+            (unsigned long long)((X[2] >> b) & 1u);
+    return h;
+}
+
+// Oct sort key (reading R18b): the 21-level cell of the point's descent
+// through the cube hierarchy (octant bits from fp64 comparisons, as the
+// build), ordered along the Hilbert curve of the root cube.
 __global__ void oct_keys(const float *pts, long long n, int ld, double cx, double cy, double cz, double side,
                          unsigned long long *keys) {
     for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
         const float *p = pts + i * ld;
         const double x = p[0], y = p[1], z = p[2];
         double c0 = cx, c1 = cy, c2 = cz, s = side;
-        unsigned long long code = 0;
+        unsigned ix = 0, iy = 0, iz = 0;
 #pragma unroll 1
         for (int l = 0; l < 21; ++l) {
             const double h = s * 0.25;
             const int o = (x >= c0) | ((y >= c1) << 1) | ((z >= c2) << 2);
-            code = (code << 3) | (unsigned)o;
+            ix = (ix << 1) | (unsigned)(o & 1);
+            iy = (iy << 1) | (unsigned)((o >> 1) & 1);
+            iz = (iz << 1) | (unsigned)(o >> 2);
             c0 += (o & 1) ? h : -h;
             c1 += (o & 2) ? h : -h;
             c2 += (o & 4) ? h : -h;
             s *= 0.5;
         }
-        keys[i] = code;
+        keys[i] = hilbert21(ix, iy, iz);
     }
 }
 

@@ -338,14 +338,39 @@ def test_sort_keys_kd_reproduce_tree_order():
     assert np.array_equal(perm, t.tree_order())  # descent of a data point ends at its own leaf
 
 
-def test_sort_keys_oct_are_morton_and_tree_order():
-    b = ttgen.plummer(5000, seed=72)
+def test_sort_keys_oct_follow_the_hilbert_curve():
+    """Oct sort keys (reading R18b) order the points' 21-level cells of the
+    cube hierarchy along a Hilbert curve.  Pinned by the curve's defining
+    properties, not by its formula: (1) consecutive cells are face-adjacent
+    -- a grid of 8^3 bodies, one per level-3 cell of the unit root cube,
+    sorted by key steps by exactly one cell along one axis each time; (2)
+    the curve fills every dyadic cube before leaving it -- for Plummer bodies
+    each level-k cell (Morton prefix, the build's octant rule) is one
+    contiguous run of the sorted order, k = 1..7; (3) one key per cell."""
+    g = (np.stack(np.meshgrid(np.arange(8), np.arange(8), np.arange(8), indexing="ij"), -1).reshape(-1, 3) + 0.5) / 8
+    corners = np.array([[0, 0, 0], [1, 1, 1]], np.float64)  # make the root cube exactly [0, 1]^3
+    pts = np.concatenate([g, corners])
+    b = np.concatenate([pts, np.ones((len(pts), 1))], 1).astype(np.float32)
     t = oracle.build_oct(b)
     c, side = t.root_cube()
-    keys = oracle.sort_keys(t, b)
-    assert np.array_equal(keys, brute.morton63(b, c, side))
-    perm = np.argsort(keys, kind="stable")
-    assert np.array_equal(perm, t.tree_order())  # Morton order == preorder of leaves
+    assert side == 1.0 and np.array_equal(c, [0.5, 0.5, 0.5])
+    keys = oracle.sort_keys(t, b)[:512]
+    o = np.argsort(keys, kind="stable")
+    cells = np.floor(g[o] * 8).astype(int)
+    assert np.all(np.abs(np.diff(cells, axis=0)).sum(1) == 1)
+    assert len(np.unique(keys)) == 512
+
+    bp = ttgen.plummer(5000, seed=72)
+    t = oracle.build_oct(bp)
+    c, side = t.root_cube()
+    hk = oracle.sort_keys(t, bp)
+    mk = brute.morton63(bp, c, side)
+    o = np.argsort(hk, kind="stable")
+    for k in range(1, 8):
+        pre = (mk[o] >> np.uint64(63 - 3 * k))
+        starts = np.concatenate([[True], pre[1:] != pre[:-1]])
+        assert starts.sum() == len(np.unique(pre)), k  # each level-k cell is one run
+    assert len(np.unique(hk)) == len(np.unique(mk))  # one key per 21-level cell
 
 
 def test_sort_keys_vp_are_a_stable_bijection():
