@@ -242,7 +242,8 @@ def load_counts(workload: str, mode: str):
         return None
 
 
-KERNEL_SOURCE = {"bh": "kern_bh_group.cu", "pc": "kern_pc.cu", "knn": "kern_knn.cu", "vp": "kern_vp.cu", "nn": "kern_nn.cu"}
+KERNEL_SOURCE = {"bh": ["kern_bh_group.cu"], "pc": ["kern_pc.cu", "kern_pc_split.cu"], "knn": ["kern_knn.cu"],
+                 "vp": ["kern_vp.cu"], "nn": ["kern_nn.cu"]}
 
 
 def kernel_sha256(workload: str) -> str:
@@ -253,7 +254,7 @@ def kernel_sha256(workload: str) -> str:
     import hashlib
     kind = workload.rstrip("0123456789m").replace("steps", "")  # bh16m -> bh, bhsteps -> bh
     pkg = os.path.join(ROOT, "paper_conf_sc_goldfarbjk13_b200")
-    files = [os.path.join(pkg, "csrc", f) for f in (KERNEL_SOURCE[kind], "kern_common.cuh", "tt_internal.h")]
+    files = [os.path.join(pkg, "csrc", f) for f in (*KERNEL_SOURCE[kind], "kern_common.cuh", "tt_internal.h")]
     h = hashlib.sha256()
     for f in files:
         h.update(os.path.basename(f).encode())
@@ -845,6 +846,9 @@ def run_ours(args, rank, world, local_rank):
     alg_bytes = visits * bpv + ptests * bpt + m * BYTES_PER_POINT_IO[name]
     achieved = alg_bytes / (kms / 1e3) / 1e9
     kernel_name = {"bh": "bh_group_kernel", "pc": "pc_kernel", "knn": "knn_kernel", "vp": "vp_kernel", "nn": "nn_kernel"}[name]
+    if name == "pc" and args.mode == "auto" and args.variant == "autoropes" and args.auto_min_depth is None \
+            and -(-m // 32) < torch.cuda.get_device_properties(device).multi_processor_count * 32:
+        kernel_name = "pc_split_kernel"  # AUTO splits small launches over 16 lanes per point (tt.h)
     cnt = load_counts(args.workload, args.mode) if not args.unsorted and args.variant == "autoropes" else None
     cnt_ok = bool(cnt) and cnt.get("src_sha256") == kernel_sha256(name)
     clocks = clk.summary()

@@ -1,15 +1,20 @@
 #!/bin/bash
 # Run on the GPU box (gpurun): launch list of the bench command + one
-# `ncu --set full` capture of each traversal kernel.  Outputs in gpurun_out/.
+# `ncu --set full` capture of each traversal kernel (configs[0..4]).  Outputs in gpurun_out/.
 set -x
 mkdir -p gpurun_out
 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/launches_bh.csv \
-    python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e > /dev/null 2>&1
-for spec in "bh auto 1000000" "pc auto 10000" "knn auto 1000000" "vp auto 1000000" "vp independent 1000000" "knn independent 1000000" "nn auto 1000000"; do
+    python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e --no-strong > /dev/null 2>&1
+# <workload> <mode> <launches to skip: the a0 group-build trigger (BH) and the stats pass> <kernel>
+for spec in "bh auto 2 bh_group_kernel" "pc auto 1 pc_split_kernel" "knn auto 1 knn_kernel" "vp auto 1 vp_kernel" \
+            "vp independent 1 vp_kernel" "knn independent 1 knn_kernel" "nn auto 1 nn_kernel" \
+            "bh16m auto 2 bh_group_kernel" "knn16m auto 1 knn_kernel"; do
   set -- $spec
-  w=$1; m=$2; n=$3
-  ncu --set full --clock-control none --import-source on -k regex:$( [ $w = bh ] && echo bh_group_kernel || echo ${w}_kernel ) -s 1 -c 1 \
+  w=$1; m=$2; sk=$3; k=$4
+  extra=""
+  case $w in *16m) extra="--device-build";; esac
+  timeout 1200 ncu --set full --clock-control none --import-source on -k regex:$k -s $sk -c 1 \
       -o gpurun_out/prof_${w}_${m} python bench.py --workload $w --mode $m --steps 1 --warmup 1 \
-      --no-cpu-baseline --no-e2e --points-per-rank $n > gpurun_out/ncu_${w}_${m}.log 2>&1
+      --no-cpu-baseline --no-e2e --no-chase --no-strong $extra > gpurun_out/ncu_${w}_${m}.log 2>&1
 done
 ls -la gpurun_out
