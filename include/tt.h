@@ -215,7 +215,7 @@ tt_status tt_tree_get_info(const tt_tree *t, tt_tree_info *out);
 /* a1: point sort (§4.4).  Key = where the point's descent of the
  * tree by the build's split rule ends: kd -> the leaf's first tree-order
  * point (tree order); oct -> the index, along the 3-D Hilbert curve of the
- * root cube, of the point's 21-level cell of the cube hierarchy (octant bits
+ * root cube, of the point's 16-level cell of the cube hierarchy (octant bits
  * from the build's fp64 comparisons; reading R18b: more compact warp tiles
  * than the Morton / leaf-preorder order); vp -> 2-bit-per-level path code;
  * nn -> the same code of the left-iff-x[dim]<split descent.  A

@@ -27,12 +27,19 @@ __global__ void iota_kernel(uint32_t *v, long long n) {
         v[i] = (uint32_t)i;
 }
 
-// Hilbert index (Skilling's transpose algorithm) of the 21-level cell whose
-// coordinate bits are (ix, iy, iz), bits interleaved x, y, z from the top
-__device__ __forceinline__ unsigned long long hilbert21(unsigned ix, unsigned iy, unsigned iz) {
+// Levels of the oct sort key (reading R18b): cells of side root/2^16 -- for
+// the 1M / 16M Plummer configs fewer than 0.01 bodies per cell even in the
+// core, so the ties left to the index order are immaterial -- and a 48-bit
+// key: 6 radix passes instead of 8.
+constexpr int kOctKeyLevels = 16;
+
+// Hilbert index (Skilling's transpose algorithm) of the kOctKeyLevels-level
+// cell whose coordinate bits are (ix, iy, iz), bits interleaved x, y, z from
+// the top
+__device__ __forceinline__ unsigned long long hilbert_key(unsigned ix, unsigned iy, unsigned iz) {
     unsigned X[3] = {ix, iy, iz};
 #pragma unroll 1
-    for (unsigned Q = 1u << 20; Q > 1; Q >>= 1) {
+    for (unsigned Q = 1u << (kOctKeyLevels - 1); Q > 1; Q >>= 1) {
         const unsigned P = Q - 1;
 #pragma unroll
         for (int i = 0; i < 3; ++i) {
@@ -49,20 +56,20 @@ __device__ __forceinline__ unsigned long long hilbert21(unsigned ix, unsigned iy
     X[2] ^= X[1];
     unsigned t = 0;
 #pragma unroll 1
-    for (unsigned Q = 1u << 20; Q > 1; Q >>= 1)
+    for (unsigned Q = 1u << (kOctKeyLevels - 1); Q > 1; Q >>= 1)
         if (X[2] & Q) t ^= Q - 1;
     X[0] ^= t;
     X[1] ^= t;
     X[2] ^= t;
     unsigned long long h = 0;
 #pragma unroll 1
-    for (int b = 20; b >= 0; --b)
+    for (int b = kOctKeyLevels - 1; b >= 0; --b)
         h = (h << 3) | ((unsigned long long)((X[0] >> b) & 1u) << 2) | ((unsigned long long)((X[1] >> b) & 1u) << 1) |
             (unsigned long long)((X[2] >> b) & 1u);
     return h;
 }
 
-// Oct sort key (reading R18b): the 21-level cell of the point's descent
+// Oct sort key (reading R18b): the kOctKeyLevels-level cell of the point's descent
 // through the cube hierarchy (octant bits from fp64 comparisons, as the
 // build), ordered along the Hilbert curve of the root cube.
 __global__ void oct_keys(const float *pts, long long n, int ld, double cx, double cy, double cz, double side,
@@ -73,7 +80,7 @@ __global__ void oct_keys(const float *pts, long long n, int ld, double cx, doubl
         double c0 = cx, c1 = cy, c2 = cz, s = side;
         unsigned ix = 0, iy = 0, iz = 0;
 #pragma unroll 1
-        for (int l = 0; l < 21; ++l) {
+        for (int l = 0; l < kOctKeyLevels; ++l) {
             const double h = s * 0.25;
             const int o = (x >= c0) | ((y >= c1) << 1) | ((z >= c2) << 2);
             ix = (ix << 1) | (unsigned)(o & 1);
@@ -84,7 +91,7 @@ __global__ void oct_keys(const float *pts, long long n, int ld, double cx, doubl
             c2 += (o & 4) ? h : -h;
             s *= 0.5;
         }
-        keys[i] = hilbert21(ix, iy, iz);
+        keys[i] = hilbert_key(ix, iy, iz);
     }
 }
 
@@ -198,7 +205,7 @@ int tt_launch_sort(const tt_tree *t, const float *pts, int64_t n, int32_t ld, ui
         end_bit = 1;
         while (end_bit < 63 && (1ull << end_bit) <= (unsigned long long)t->hdr.n_points) ++end_bit;
     } else if (t->hdr.kind == TT_KIND_OCT) {
-        end_bit = 63;
+        end_bit = 3 * kOctKeyLevels;
     }
 #define TT_CK(x)                         \
     do {                                 \

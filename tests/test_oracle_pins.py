@@ -339,7 +339,7 @@ def test_sort_keys_kd_reproduce_tree_order():
 
 
 def test_sort_keys_oct_follow_the_hilbert_curve():
-    """Oct sort keys (reading R18b) order the points' 21-level cells of the
+    """Oct sort keys (reading R18b) order the points' 16-level cells of the
     cube hierarchy along a Hilbert curve.  Pinned by the curve's defining
     properties, not by its formula: (1) consecutive cells are face-adjacent
     -- a grid of 8^3 bodies, one per level-3 cell of the unit root cube,
@@ -370,7 +370,9 @@ def test_sort_keys_oct_follow_the_hilbert_curve():
         pre = (mk[o] >> np.uint64(63 - 3 * k))
         starts = np.concatenate([[True], pre[1:] != pre[:-1]])
         assert starts.sum() == len(np.unique(pre)), k  # each level-k cell is one run
-    assert len(np.unique(hk)) == len(np.unique(mk))  # one key per 21-level cell
+    lv16 = mk >> np.uint64(63 - 48)
+    assert len(np.unique(hk)) == len(np.unique(lv16))  # one key per 16-level cell
+    assert hk.max() < 2 ** 48
 
 
 def test_sort_keys_vp_are_a_stable_bijection():
