@@ -70,6 +70,8 @@ def parse():
     ap.add_argument("--no-strong", action="store_true",
                     help="skip the fixed-config strong-scaling block (configs[4] BH 16M, every N)")
     ap.add_argument("--strong-points", type=int, default=0, help="override the strong block's N (testing)")
+    ap.add_argument("--steps-order", default="build", choices=["build", "sort"],
+                    help="bhsteps traversal order: the GPU build's tree order, or tt_sort_points (Hilbert)")
     ap.add_argument("--auto-min-depth", type=int, default=None, help="AUTO-mode threshold (default: kernel's)")
     ap.add_argument("--switch-below", type=int, default=0,
                     help="kNN: dynamic L->N switch when fewer lanes are active (NEXT-3; 0 = never)")
@@ -395,7 +397,8 @@ def run_bh_steps(args, rank, world):
     ids = torch.arange(n, dtype=torch.int32, device=dev)
     dt = 1e-3
     for _ in range(args.warmup):
-        B, V, ids = nbody.simulate_sharded(B, V, ids, 1, dt, c["theta"], c["eps"], final_kick=False)
+        B, V, ids = nbody.simulate_sharded(B, V, ids, 1, dt, c["theta"], c["eps"], final_kick=False,
+                                           order=args.steps_order)
     torch.cuda.synchronize()
     stream = torch.cuda.current_stream()
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
@@ -404,7 +407,8 @@ def run_bh_steps(args, rank, world):
     with ClockSampler(torch.cuda.current_device()) as clk:
         for i in range(args.steps):
             evs[i][0].record(stream)
-            B, V, ids = nbody.simulate_sharded(B, V, ids, 1, dt, c["theta"], c["eps"], final_kick=False)
+            B, V, ids = nbody.simulate_sharded(B, V, ids, 1, dt, c["theta"], c["eps"], final_kick=False,
+                                               order=args.steps_order)
             evs[i][1].record(stream)
         torch.cuda.synchronize()
     if world > 1:
@@ -417,7 +421,7 @@ def run_bh_steps(args, rank, world):
     line = {"metric": METRIC, "value": n / (ms / 1e3), "unit": "points/s (body-steps/s)", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": {"workload": "bh_1m_plummer time steps", "bodies": n, "dt": dt,
+            "config": {"workload": "bh_1m_plummer time steps", "bodies": n, "dt": dt, "order": args.steps_order,
                        "step": "GPU build (+ tree order) + force (own shard) + gathered kick-drift (leapfrog KDK)"
                                + (" + all-gather of x, v, ids" if world > 1 else ""),
                        "parallelism": f"dp{world} (bodies sharded by sorted order, tree rebuilt on every rank)",

@@ -29,7 +29,7 @@ import torch
 
 from . import _lib as L
 from ._lib import check
-from .tt import _dev, _stream_handle, tt_build_oct_device_order, tt_traverse_bh
+from .tt import _dev, _stream_handle, tt_build_oct_device_order, tt_sort_points, tt_traverse_bh
 
 
 def tt_kick_drift(bodies: torch.Tensor, vel: torch.Tensor, acc: torch.Tensor, dt_kick: float, dt_drift: float,
@@ -92,7 +92,8 @@ def simulate(bodies: torch.Tensor, vel: torch.Tensor, steps: int, dt: float, the
 
 
 def simulate_sharded(bodies: torch.Tensor, vel: torch.Tensor, ids: torch.Tensor, steps: int, dt: float,
-                     theta: float = 0.5, eps: float = 0.05, mode="auto", group=None, final_kick: bool = True):
+                     theta: float = 0.5, eps: float = 0.05, mode="auto", group=None, final_kick: bool = True,
+                     order: str = "build"):
     """Leapfrog KDK over `steps` steps with the bodies sharded across the ranks
     of `group` (None and no process group: one rank).  Every rank passes the
     same full (n, 4) bodies / vel and (n,) int32 ids; n must be a multiple of
@@ -103,7 +104,12 @@ def simulate_sharded(bodies: torch.Tensor, vel: torch.Tensor, ids: torch.Tensor,
     Step s: tree = build(x); perm = sort(x); a = force(x) for the rank's lanes
     perm[lo:hi]; kick(dt/2 if s == 0 else dt) + drift(dt) gathered through
     perm[lo:hi] into rows [lo, hi); all-gather.  With final_kick, one more
-    force pass and the closing kick(dt/2) (drift 0)."""
+    force pass and the closing kick(dt/2) (drift 0).
+
+    order: the traversal order of a step -- "build": the tree order the GPU
+    build has already sorted the bodies into (no extra sort); "sort": the
+    Hilbert order of tt_sort_points (R18b: more compact warp tiles, one more
+    sort per step)."""
     import torch.distributed as dist
     from .parallel import allgather_rows, shard_range
     world = dist.get_world_size(group) if dist.is_initialized() else 1
@@ -120,6 +126,8 @@ def simulate_sharded(bodies: torch.Tensor, vel: torch.Tensor, ids: torch.Tensor,
     def half(dtk, dtd):
         nonlocal x, v, i, xo, vo, io
         tree, perm = tt_build_oct_device_order(x, order_buf)  # tree order from the build's sort
+        if order == "sort":
+            perm = tt_sort_points(tree, x, out=order_buf)
         mine = perm[lo:hi]
         tt_traverse_bh(tree, x, theta, eps, out=acc, order=mine, mode=mode)
         tt_kick_drift_permuted(x, v, acc, mine, dtk, dtd, xo[lo:hi], vo[lo:hi], i, io[lo:hi])
