@@ -70,7 +70,7 @@ def parse():
     ap.add_argument("--no-strong", action="store_true",
                     help="skip the fixed-config strong-scaling block (configs[4] BH 16M, every N)")
     ap.add_argument("--strong-points", type=int, default=0, help="override the strong block's N (testing)")
-    ap.add_argument("--steps-order", default="build", choices=["build", "sort"],
+    ap.add_argument("--steps-order", default="sort", choices=["build", "sort"],
                     help="bhsteps traversal order: the GPU build's tree order, or tt_sort_points (Hilbert)")
     ap.add_argument("--auto-min-depth", type=int, default=None, help="AUTO-mode threshold (default: kernel's)")
     ap.add_argument("--switch-below", type=int, default=0,
@@ -379,7 +379,7 @@ def run_reference(args, rank, world):
 # ------------------------------------------------------------------- ours
 def run_bh_steps(args, rank, world):
     """NEXT-4 workload: a bench step = one BH time step of configs[1]
-    (tt_build_oct_device_order (tree + tree order) + tt_traverse_bh + tt_kick_drift_permuted,
+    (tt_build_oct_device_order + tt_sort_points + tt_traverse_bh + tt_kick_drift_permuted,
     + all-gather of positions / velocities / ids for N > 1).  Strong scaling:
     the same 1M-body system on every N; each rank integrates its warp-aligned
     shard of the sorted order (nbody.simulate_sharded)."""
@@ -422,7 +422,7 @@ def run_bh_steps(args, rank, world):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": "bh_1m_plummer time steps", "bodies": n, "dt": dt, "order": args.steps_order,
-                       "step": "GPU build (+ tree order) + force (own shard) + gathered kick-drift (leapfrog KDK)"
+                       "step": "GPU build + sort + force (own shard) + gathered kick-drift (leapfrog KDK)"
                                + (" + all-gather of x, v, ids" if world > 1 else ""),
                        "parallelism": f"dp{world} (bodies sharded by sorted order, tree rebuilt on every rank)",
                        "params": c, "l2": "not flushed: a time step rewrites the bodies and rebuilds the tree"},

@@ -6,7 +6,8 @@ mass, runs the force traversal and advances the bodies.  Every stage here is
 a libtt call on the current stream (no host round trip besides the node
 count the GPU build reads back):
 
-    tt_build_oct_device_order (tree + the bodies' tree order) -> tt_traverse_bh -> tt_kick_drift
+    tt_build_oct_device_order -> tt_sort_points (Hilbert; or the build's tree order) -> tt_traverse_bh
+    -> tt_kick_drift
 
 Integration is leapfrog kick-drift-kick, with consecutive half kicks merged:
   step 0:     kick(dt/2) + drift(dt), force
@@ -68,11 +69,19 @@ def tt_kick_drift_permuted(bodies: torch.Tensor, vel: torch.Tensor, acc: torch.T
                                           iop, C.c_void_p(_stream_handle(stream))), "tt_kick_drift_permuted")
 
 
+# Traversal order of a time step: "sort" = tt_sort_points' Hilbert order
+# (R18b), "build" = the tree (Morton) order the GPU build already produced --
+# no extra sort, but less compact warp tiles: 5.25 vs 5.06 ms per 1M-body
+# step (bench --workload bhsteps --steps-order, same box), so "sort".
+DEFAULT_ORDER = "sort"
+
+
 def forces(bodies: torch.Tensor, theta: float, eps: float, out: torch.Tensor | None = None, mode="auto",
-           stats=None):
+           stats=None, order: str = DEFAULT_ORDER):
     """One force pass on the current positions: GPU build, sort, traverse."""
-    # the build's own sort is the tree order: no separate tt_sort_points
     tree, perm = tt_build_oct_device_order(bodies)
+    if order == "sort":
+        perm = tt_sort_points(tree, bodies, out=perm)
     acc = tt_traverse_bh(tree, bodies, theta, eps, out=out, order=perm, mode=mode, stats=stats)
     return acc, tree
 
@@ -93,7 +102,7 @@ def simulate(bodies: torch.Tensor, vel: torch.Tensor, steps: int, dt: float, the
 
 def simulate_sharded(bodies: torch.Tensor, vel: torch.Tensor, ids: torch.Tensor, steps: int, dt: float,
                      theta: float = 0.5, eps: float = 0.05, mode="auto", group=None, final_kick: bool = True,
-                     order: str = "build"):
+                     order: str = DEFAULT_ORDER):
     """Leapfrog KDK over `steps` steps with the bodies sharded across the ranks
     of `group` (None and no process group: one rank).  Every rank passes the
     same full (n, 4) bodies / vel and (n,) int32 ids; n must be a multiple of
