@@ -85,6 +85,15 @@ def parse():
 
 
 # ------------------------------------------------------------------ inputs
+_T0 = time.time()
+
+
+def _trace(msg: str):
+    """Phase trace on stderr (TT_BENCH_TRACE=1), rank-prefixed."""
+    if os.environ.get("TT_BENCH_TRACE"):
+        print(f"[bench r{os.environ.get('RANK', '0')} +{time.time() - _T0:7.2f}s] {msg}", file=sys.stderr, flush=True)
+
+
 def make_workload(name: str, world: int, per_rank: int = 0):
     """Global synthetic inputs (identical on every rank: seeded)."""
     if name == "bh16m":
@@ -430,29 +439,40 @@ def run_bh_steps(args, rank, world):
     print(json.dumps(line), flush=True)
 
 
-def run_strong16m(args, rank, world, device, P, PAR):
-    """configs[4]: one fixed Barnes-Hut problem (16M-body Plummer sphere,
-    theta 0.5) at every N -- strong scaling.  Rank 0 builds the tree on its
-    GPU (tt_build_oct_device, NEXT-1) and NCCL-broadcasts the packed blob
+def run_strong16m(args, rank, world, device, P, PAR, kind="bh"):
+    """configs[4]: one fixed problem at every N -- strong scaling.  kind "bh":
+    the 16M-body Plummer sphere, theta 0.5; kind "knn": k = 8 for 16M 7-D
+    queries over 16M 7-D mixture points.  Rank 0 builds the tree on its GPU
+    (tt_build_{oct,kd}_device, NEXT-1) and NCCL-broadcasts the packed blob
     (tt_tree_copy_blob -> broadcast -> tt_tree_from_blob); every rank places
-    the bodies in global tree order once (data placement) and owns a
+    the points in global sorted order once (data placement) and owns a
     contiguous warp-aligned range; a timed step = a1 sort of the rank's shard
-    + traversal + all-gather of the accelerations.  Each phase is reported
-    separately; every time is the max over ranks (CUDA events)."""
+    (+ a1b tile schedule for kNN) + traversal + all-gather of the results.
+    Each phase is reported separately; every time is the max over ranks
+    (CUDA events)."""
     import torch
     import torch.distributed as dist
-    c = ttgen.CONFIGS["bh_16m_plummer"]
-    n = args.strong_points or c["n"]
+    c = ttgen.CONFIGS["bh_16m_plummer" if kind == "bh" else "knn_16m_7d"]
+    n = args.strong_points or (c["n"] if kind == "bh" else c["m"])
     if world > 1 and n % (64 * world):
-        raise SystemExit(f"bench: {n} bodies do not split into {world} equal warp-aligned shards")
-    data = ttgen.plummer(n, c["seed"])
-    bd_all = torch.from_numpy(data).to(device)
+        raise SystemExit(f"bench: {n} points do not split into {world} equal warp-aligned shards")
+    if kind == "bh":
+        data = ttgen.plummer(n, c["seed"])
+        queries = data
+    else:
+        data = ttgen.gaussian_mixture(args.strong_points or c["n"], c["dim"], c["seed"])
+        queries = ttgen.gaussian_mixture(n, c["dim"], c["qseed"])
+    d_all = torch.from_numpy(np.ascontiguousarray(data)).to(device)
+    _trace(f"strong {kind}: inputs ready")
     stream = torch.cuda.current_stream()
     torch.cuda.synchronize()
     t0 = time.perf_counter()
-    tree = P.tt_build_oct_device(bd_all) if rank == 0 else None
+    tree = None
+    if rank == 0:
+        tree = P.tt_build_oct_device(d_all) if kind == "bh" else P.tt_build_kd_device(d_all, c["leaf"])
     torch.cuda.synchronize()
     build_ms = 1e3 * (time.perf_counter() - t0)
+    _trace(f"strong {kind}: built")
     bcast_ms = None
     if world > 1:
         dist.barrier()
@@ -460,30 +480,43 @@ def run_strong16m(args, rank, world, device, P, PAR):
         tree = PAR.broadcast_device_tree(tree, device)
         torch.cuda.synchronize()
         bcast_ms = PAR.max_over_ranks(1e3 * (time.perf_counter() - t0), device)
+    q_all = d_all if kind == "bh" else torch.from_numpy(np.ascontiguousarray(queries)).to(device)
+    del d_all
     t0 = time.perf_counter()
-    gperm = P.tt_sort_points(tree, bd_all).long()
-    q = bd_all[gperm].contiguous()
+    gperm = P.tt_sort_points(tree, q_all).long()
+    q = q_all[gperm].contiguous()
     ids = gperm.to(torch.int32)
-    del bd_all, gperm
+    del q_all, gperm
     torch.cuda.synchronize()
     placement_ms = 1e3 * (time.perf_counter() - t0)
+    _trace(f"strong {kind}: placed")
     lo, hi = PAR.shard_range(n, rank, world)
     q_shard, ids_shard = q[lo:hi], ids[lo:hi]
-    out = torch.zeros((n, 4), dtype=torch.float32, device=device)
-    out_shard = out[lo:hi]
+    if kind == "bh":
+        outs = (torch.zeros((n, 4), dtype=torch.float32, device=device),)
+    else:
+        outs = (torch.zeros((n, c["k"]), dtype=torch.int32, device=device),
+                torch.zeros((n, c["k"]), dtype=torch.float32, device=device))
     order = torch.empty(hi - lo, dtype=torch.int32, device=device)
+    lpt = kind == "knn" and (hi - lo) // 32 > 148 * 32
 
     def step(ev=None):
         if ev:
             ev[0].record(stream)
         P.tt_sort_points(tree, q_shard, out=order)
+        if lpt:
+            P.tt_schedule_tiles(tree, q_shard, order, out=order)
         if ev:
             ev[1].record(stream)
-        P.tt_traverse_bh(tree, q_shard, c["theta"], c["eps"], out=out_shard, self_ids=ids_shard, order=order)
+        if kind == "bh":
+            P.tt_traverse_bh(tree, q_shard, c["theta"], c["eps"], out=outs[0][lo:hi], self_ids=ids_shard, order=order)
+        else:
+            P.tt_traverse_knn(tree, q_shard, c["k"], out_idx=outs[0][lo:hi], out_d2=outs[1][lo:hi], order=order)
         if ev:
             ev[2].record(stream)
         if world > 1:
-            PAR.allgather_rows(out, world)
+            for o in outs:
+                PAR.allgather_rows(o, world)
         if ev:
             ev[3].record(stream)
 
@@ -500,19 +533,22 @@ def run_strong16m(args, rank, world, device, P, PAR):
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
+    _trace(f"strong {kind}: timed")
     mean = lambda a, b: statistics.mean(e[a].elapsed_time(e[b]) for e in evs)  # noqa: E731
     ms, sort_ms, trav_ms, ag_ms = mean(0, 3), mean(0, 1), mean(1, 2), mean(2, 3)
     if world > 1:
         ms, sort_ms, trav_ms, ag_ms, placement_ms = (PAR.max_over_ranks(x, device) for x in
                                                      (ms, sort_ms, trav_ms, ag_ms, placement_ms))
-    del flush, out, q, ids
-    return {"workload": "bh_16m_plummer", "scaling": "strong", "value": n / (ms / 1e3), "unit": "points/s",
+    del flush, outs, q, ids
+    return {"workload": "bh_16m_plummer" if kind == "bh" else "knn_16m_7d", "scaling": "strong",
+            "value": n / (ms / 1e3), "unit": "points/s",
             "ms_per_step": ms, "sort_ms": sort_ms, "traverse_ms": trav_ms,
             "allgather_ms": ag_ms if world > 1 else None, "points": n, "points_per_rank": hi - lo,
-            "tree_build_ms": build_ms, "tree_build": "device (tt_build_oct_device) on rank 0",
+            "tree_build_ms": build_ms,
+            "tree_build": f"device (tt_build_{'oct' if kind == 'bh' else 'kd'}_device) on rank 0",
             "bcast_ms": bcast_ms, "placement_ms": placement_ms,
-            "note": "configs[4] at every N: step = a1 sort of the rank's shard + traversal + all-gather; "
-                    "build, broadcast and placement outside the timed steps, reported here"}
+            "note": "configs[4] at every N: step = a1 sort of the rank's shard (+ LPT schedule, kNN) + traversal "
+                    "+ all-gather; build, broadcast and placement outside the timed steps, reported here"}
 
 
 def run_ours(args, rank, world, local_rank):
@@ -534,6 +570,7 @@ def run_ours(args, rank, world, local_rank):
     lo, hi = PAR.shard_range(len(w["queries"]), rank, world)
     m = hi - lo  # warp-aligned equal shards
 
+    _trace("workload ready")
     # a0: tree (rank 0 builds; NCCL broadcast for N > 1) -- timed separately
     t0 = time.perf_counter()
     if args.device_build:
@@ -558,6 +595,7 @@ def run_ours(args, rank, world, local_rank):
     torch.cuda.synchronize()
     t2 = time.perf_counter()
     build_ms, upload_ms = 1e3 * (t1 - t0), 1e3 * (t2 - t1)
+    _trace("tree ready")
     # a0 also includes BH's child-group array, derived from the uploaded blob
     # by the first traversal (kern_bh_group.cu): triggered and timed here, so
     # it is neither hidden in a traversal time nor left out of a0
@@ -671,9 +709,11 @@ def run_ours(args, rank, world, local_rank):
     lock_frac = float((st.warp_mode[:tiles] == 1).float().mean().item())
     del st
 
+    _trace("stats pass done")
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
+    _trace("warm-up done")
     # our kernels per step (the NCCL all-gather of N > 1 is not ours: excluded)
     launches = count_kernels(lambda: step(collective=False)) if rank == 0 else None
 
@@ -833,13 +873,16 @@ def run_ours(args, rank, world, local_rank):
         step()
         torch.cuda.synchronize()
     clk.__exit__(None, None, None)
+    _trace("main measurement done")
     # fixed-config strong scaling (configs[4], BH 16M): the same workload at
     # every N, so the driver's 1/2/4/8-GPU lines are comparable
-    strong = None
+    strong = strong_knn = None
     if args.workload == "bh" and not args.no_strong and not args.unsorted:
         del q_all, out, out_shard
         torch.cuda.empty_cache()
-        strong = run_strong16m(args, rank, world, device, P, PAR)
+        strong = run_strong16m(args, rank, world, device, P, PAR, "bh")
+        torch.cuda.empty_cache()
+        strong_knn = run_strong16m(args, rank, world, device, P, PAR, "knn")
     if rank != 0:
         return
     peaks, peak_src = measured_peaks()
@@ -952,7 +995,7 @@ def run_ours(args, rank, world, local_rank):
         "traverse_ms": kms, "upload_ms": upload_ms, "tree_build_ms": build_ms, "tree_build": build_where,
         "group_build_ms": group_build_ms, "bcast_ms": bcast_ms, "placement_ms": placement_ms,
         "allgather_ms": allgather_ms,
-        "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "strong_16m": strong,
+        "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "strong_16m": strong, "strong_16m_knn": strong_knn,
         "gpu_launches": (launches or 0) * args.steps,
         "gpu_launches_per_step": launches,
         "clocks": clocks,
@@ -976,6 +1019,8 @@ def main():
         import torch
         import torch.distributed as dist
         backend = os.environ.get("TT_DIST_BACKEND", "nccl")  # gloo: multi-rank flow test on one GPU
+        if backend == "gloo":
+            os.environ.setdefault("GLOO_SOCKET_IFNAME", "lo")  # loopback: the hostname may not resolve
         gpu = local_rank % torch.cuda.device_count()
         torch.cuda.set_device(gpu)
         if backend == "nccl":

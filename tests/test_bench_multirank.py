@@ -22,8 +22,9 @@ def _free_port():
         return s.getsockname()[1]
 
 
-def _torchrun(extra, env_extra=None, timeout=600):
-    env = dict(os.environ, TT_DIST_BACKEND="gloo", **(env_extra or {}))
+def _torchrun(extra, env_extra=None, timeout=300):
+    # gloo over the loopback interface (the box's hostname may not resolve)
+    env = dict(os.environ, TT_DIST_BACKEND="gloo", GLOO_SOCKET_IFNAME="lo", TT_BENCH_TRACE="1", **(env_extra or {}))
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
            "--master-addr=127.0.0.1", f"--master-port={_free_port()}", os.path.join(ROOT, "bench.py"),
            "--gpus", "2"] + extra
@@ -34,7 +35,7 @@ def _torchrun(extra, env_extra=None, timeout=600):
 def test_bench_two_ranks_line():
     r = _torchrun(["--steps", "2", "--warmup", "3", "--points-per-rank", "64000", "--strong-points", "256000",
                    "--no-cpu-baseline", "--no-e2e", "--no-chase"])
-    assert r.returncode == 0, r.stderr[-3000:]
+    assert r.returncode == 0, r.stderr[-3000:]  # (phase trace of both ranks in stderr)
     lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
     assert len(lines) == 1, r.stdout  # rank 0 alone prints
     d = json.loads(lines[0])
@@ -44,6 +45,9 @@ def test_bench_two_ranks_line():
     s = d["strong_16m"]
     assert s["scaling"] == "strong" and s["points"] == 256000 and s["points_per_rank"] == 128000
     assert s["value"] > 0 and s["bcast_ms"] is not None and s["allgather_ms"] is not None
+    sk = d["strong_16m_knn"]
+    assert sk["workload"] == "knn_16m_7d" and sk["points"] == 256000 and sk["points_per_rank"] == 128000
+    assert sk["value"] > 0 and sk["bcast_ms"] is not None and sk["allgather_ms"] is not None
 
 
 @pytest.mark.gpu
