@@ -870,7 +870,7 @@ def run_ours(args, rank, world, local_rank):
     # keep the GPU busy until the sampler has seen the load (>= 5 samples)
     t_soak = time.perf_counter()
     while len(clk.lines) < 5 and time.perf_counter() - t_soak < 3.0:
-        step()
+        step(collective=False)  # rank-local: the ranks may soak a different number of steps
         torch.cuda.synchronize()
     clk.__exit__(None, None, None)
     _trace("main measurement done")
