@@ -456,6 +456,7 @@ def run_strong16m(args, rank, world, device, P, PAR, kind="bh"):
     n = args.strong_points or (c["n"] if kind == "bh" else c["m"])
     if world > 1 and n % (64 * world):
         raise SystemExit(f"bench: {n} points do not split into {world} equal warp-aligned shards")
+    ids_shard = None
     if kind == "bh":
         data = ttgen.plummer(n, c["seed"])
         queries = data
@@ -490,13 +491,44 @@ def run_strong16m(args, rank, world, device, P, PAR, kind="bh"):
     torch.cuda.synchronize()
     placement_ms = 1e3 * (time.perf_counter() - t0)
     _trace(f"strong {kind}: placed")
-    lo, hi = PAR.shard_range(n, rank, world)
-    q_shard, ids_shard = q[lo:hi], ids[lo:hi]
     if kind == "bh":
         outs = (torch.zeros((n, 4), dtype=torch.float32, device=device),)
     else:
         outs = (torch.zeros((n, c["k"]), dtype=torch.int32, device=device),
                 torch.zeros((n, c["k"]), dtype=torch.float32, device=device))
+
+    def run(qs, oslices, order, stats=None):
+        if kind == "bh":
+            P.tt_traverse_bh(tree, qs, c["theta"], c["eps"], out=oslices[0], self_ids=ids_shard, order=order,
+                             stats=stats)
+        else:
+            P.tt_traverse_knn(tree, qs, c["k"], out_idx=oslices[0], out_d2=oslices[1], order=order, stats=stats)
+
+    # Cost-balanced shards: every rank traverses its
+    # equal-count shard once with stats (untimed), the per-point visit counts
+    # are all-gathered, and the shard boundaries are put where their prefix
+    # sum crosses r/N of the total (warp-aligned); results then travel by a
+    # padded all-gather.  N = 1: one shard.
+    ranges = [(0, n)]
+    imb_equal = imb_bal = 1.0
+    if world > 1:
+        lo, hi = PAR.shard_range(n, rank, world)
+        ids_shard = ids[lo:hi]
+        order = P.tt_sort_points(tree, q[lo:hi])
+        st = P.Stats.alloc(hi - lo, device)
+        run(q[lo:hi], tuple(o[lo:hi] for o in outs), order, st)
+        vis = torch.zeros((n, 1), dtype=torch.int32, device=device)
+        vis[lo:hi, 0] = st.visits
+        PAR.allgather_rows(vis, world)
+        cost = vis[:, 0].to(torch.float64)
+        ranges = PAR.balanced_ranges(cost, world)
+        per = lambda rs: [float(cost[a:b].sum()) for a, b in rs]  # noqa: E731
+        eq = per([PAR.shard_range(n, r, world) for r in range(world)])
+        bal = per(ranges)
+        imb_equal, imb_bal = max(eq) / (sum(eq) / world), max(bal) / (sum(bal) / world)
+        del st, vis, cost
+    lo, hi = ranges[rank]
+    q_shard, ids_shard = q[lo:hi], ids[lo:hi]
     order = torch.empty(hi - lo, dtype=torch.int32, device=device)
     lpt = kind == "knn" and (hi - lo) // 32 > 148 * 32
 
@@ -508,15 +540,12 @@ def run_strong16m(args, rank, world, device, P, PAR, kind="bh"):
             P.tt_schedule_tiles(tree, q_shard, order, out=order)
         if ev:
             ev[1].record(stream)
-        if kind == "bh":
-            P.tt_traverse_bh(tree, q_shard, c["theta"], c["eps"], out=outs[0][lo:hi], self_ids=ids_shard, order=order)
-        else:
-            P.tt_traverse_knn(tree, q_shard, c["k"], out_idx=outs[0][lo:hi], out_d2=outs[1][lo:hi], order=order)
+        run(q_shard, tuple(o[lo:hi] for o in outs), order)
         if ev:
             ev[2].record(stream)
         if world > 1:
             for o in outs:
-                PAR.allgather_rows(o, world)
+                PAR.allgather_rows_var(o, ranges)
         if ev:
             ev[3].record(stream)
 
@@ -547,6 +576,9 @@ def run_strong16m(args, rank, world, device, P, PAR, kind="bh"):
             "tree_build_ms": build_ms,
             "tree_build": f"device (tt_build_{'oct' if kind == 'bh' else 'kd'}_device) on rank 0",
             "bcast_ms": bcast_ms, "placement_ms": placement_ms,
+            "shards": "cost-balanced: prefix sum of a previous pass's per-point visit counts, warp-aligned"
+                      if world > 1 else "one",
+            "shard_cost_max_over_mean": {"equal_count": round(imb_equal, 4), "balanced": round(imb_bal, 4)},
             "note": "configs[4] at every N: step = a1 sort of the rank's shard (+ LPT schedule, kNN) + traversal "
                     "+ all-gather; build, broadcast and placement outside the timed steps, reported here"}
 

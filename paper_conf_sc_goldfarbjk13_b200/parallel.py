@@ -102,6 +102,47 @@ def allgather_rows(full: torch.Tensor, world: int, group=None) -> torch.Tensor:
     return full
 
 
+def balanced_ranges(costs: torch.Tensor, world: int, align: int = 64) -> list[tuple[int, int]]:
+    """Contiguous warp-aligned shards [lo, hi) of len(costs) points with
+    (nearly) equal total cost: the boundaries are where the prefix sum of the
+    per-point costs crosses r/world of the total, rounded to `align` points
+    (SURVEY §8(e)'s cost-weighted split; e.g. costs = the visit counts of a
+    previous pass).  Deterministic: every rank computes the same ranges from
+    the same costs."""
+    n = int(costs.numel())
+    c = torch.cumsum(costs.detach().to(torch.float64).cpu(), 0)
+    total = float(c[-1]) if n else 0.0
+    bounds = [0]
+    for r in range(1, world):
+        k = int(torch.searchsorted(c, torch.tensor([total * r / world], dtype=torch.float64)).item())
+        k = min(max(int(round(k / align)) * align, bounds[-1]), n)
+        bounds.append(k)
+    bounds.append(n)
+    return [(bounds[r], bounds[r + 1]) for r in range(world)]
+
+
+def allgather_rows_var(full: torch.Tensor, ranges: list[tuple[int, int]], group=None) -> torch.Tensor:
+    """All-gather of contiguous row shards of `full` whose lengths differ
+    (rank r owns rows ranges[r]): every rank contributes its rows padded to
+    the longest shard, one all_gather_into_tensor, then each shard is copied
+    to its place.  In place on `full`."""
+    world = len(ranges)
+    rank = dist.get_rank(group)
+    lens = [hi - lo for lo, hi in ranges]
+    mx = max(lens)
+    wire = _wire(full.device, group)
+    row = full.shape[1:]
+    mine = torch.zeros((mx, *row), dtype=full.dtype, device=wire)
+    lo, hi = ranges[rank]
+    mine[:hi - lo] = full[lo:hi].to(wire)
+    gathered = torch.empty((world * mx, *row), dtype=full.dtype, device=wire)
+    dist.all_gather_into_tensor(gathered, mine, group=group)
+    for r, (a, b) in enumerate(ranges):
+        if r != rank and b > a:
+            full[a:b] = gathered[r * mx:r * mx + (b - a)].to(full.device)
+    return full
+
+
 def max_over_ranks(x: float, device, group=None) -> float:
     t = torch.tensor([x], dtype=torch.float64, device=_wire(device, group))
     dist.all_reduce(t, op=dist.ReduceOp.MAX, group=group)

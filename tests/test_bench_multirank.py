@@ -55,9 +55,12 @@ def test_bench_two_ranks_line():
     s = d["strong_16m"]
     assert s["scaling"] == "strong" and s["points"] == 256000 and s["points_per_rank"] == 128000
     assert s["value"] > 0 and s["bcast_ms"] is not None and s["allgather_ms"] is not None
+    assert s["shards"].startswith("cost-balanced")
+    assert s["shard_cost_max_over_mean"]["balanced"] <= s["shard_cost_max_over_mean"]["equal_count"] + 1e-9
     sk = d["strong_16m_knn"]
     assert sk["workload"] == "knn_16m_7d" and sk["points"] == 256000 and sk["points_per_rank"] == 128000
     assert sk["value"] > 0 and sk["bcast_ms"] is not None and sk["allgather_ms"] is not None
+    assert sk["shard_cost_max_over_mean"]["balanced"] <= sk["shard_cost_max_over_mean"]["equal_count"] + 1e-9
 
 
 @pytest.mark.gpu

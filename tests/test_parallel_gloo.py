@@ -13,7 +13,7 @@ import torch
 import torch.distributed as dist
 import torch.multiprocessing as mp
 
-from paper_conf_sc_goldfarbjk13_b200.parallel import shard_range
+from paper_conf_sc_goldfarbjk13_b200.parallel import balanced_ranges, shard_range
 
 
 def _free_port():
@@ -49,6 +49,17 @@ def _worker(rank, world, port, q):
         ids[lo:hi] = torch.arange(lo, hi, dtype=torch.int32) * 3
         PAR.allgather_rows(ids.view(-1, 1), world)
         ok_gather = ok_gather and bool(torch.equal(ids, torch.arange(n, dtype=torch.int32) * 3))
+        # cost-balanced unequal shards + padded all-gather
+        costs = torch.ones(n)
+        costs[: n // 4] = 5.0  # the first quarter costs 5x
+        ranges = PAR.balanced_ranges(costs, world)
+        lo2, hi2 = ranges[rank]
+        full2 = torch.full((n, 3), -1.0)
+        full2[lo2:hi2] = torch.arange(lo2, hi2, dtype=torch.float32)[:, None] * torch.tensor([1.0, 2.0, 3.0])
+        PAR.allgather_rows_var(full2, ranges)
+        ok_gather = ok_gather and bool(torch.equal(
+            full2, torch.arange(n, dtype=torch.float32)[:, None] * torch.tensor([1.0, 2.0, 3.0])))
+        ok_gather = ok_gather and ranges[0][1] - ranges[0][0] < n // world  # the costly part gets fewer rows
         mx = PAR.max_over_ranks(float(rank + 1) * 1.5, "cpu")
         q.put((rank, ok_blob, ok_gather, mx))
         dist.destroy_process_group()
@@ -81,3 +92,22 @@ def test_shard_range_partitions_warp_aligned(n, world):
         assert lo % 64 == 0 or lo == n
         covered[lo:hi] += 1
     assert np.all(covered == 1)
+
+
+@pytest.mark.parametrize("world", [1, 2, 3, 8])
+def test_balanced_ranges_cover_aligned_and_balance(world):
+    """Contiguous, warp-aligned, covering; the per-shard cost is within one
+    warp of points of total/world (SURVEY §8(e) cost-weighted split)."""
+    rng = np.random.default_rng(world)
+    n = 64 * 1000 + 37
+    c = torch.from_numpy(rng.gamma(0.5, 2.0, n))
+    rs = balanced_ranges(c, world)
+    covered = np.zeros(n, np.int32)
+    for lo, hi in rs:
+        assert lo % 64 == 0 or lo == n
+        covered[lo:hi] += 1
+    assert np.all(covered == 1)
+    tot = float(c.sum())
+    per = [float(c[lo:hi].sum()) for lo, hi in rs]
+    worst = float(torch.topk(c, 64).values.sum())
+    assert max(per) - tot / world <= worst
