@@ -53,14 +53,19 @@ def test_bench_two_ranks_line():
     assert d["config"]["global_points"] == 128000
     assert d["bcast_ms"] is not None and d["placement_ms"] is not None and d["allgather_ms"] is not None
     s = d["strong_16m"]
-    assert s["scaling"] == "strong" and s["points"] == 256000 and s["points_per_rank"] == 128000
+    # cost-balanced shards: rank 0's is warp-aligned and near half
+    assert s["scaling"] == "strong" and s["points"] == 256000
+    assert s["points_per_rank"] % 64 == 0 and abs(s["points_per_rank"] - 128000) < 12800
     assert s["value"] > 0 and s["bcast_ms"] is not None and s["allgather_ms"] is not None
     assert s["shards"].startswith("cost-balanced")
-    assert s["shard_cost_max_over_mean"]["balanced"] <= s["shard_cost_max_over_mean"]["equal_count"] + 1e-9
+    # balanced within a warp of points of the ideal (the rounding can leave
+    # it a hair above an already even equal-count split)
+    assert s["shard_cost_max_over_mean"]["balanced"] <= max(s["shard_cost_max_over_mean"]["equal_count"], 1.01)
     sk = d["strong_16m_knn"]
-    assert sk["workload"] == "knn_16m_7d" and sk["points"] == 256000 and sk["points_per_rank"] == 128000
+    assert sk["workload"] == "knn_16m_7d" and sk["points"] == 256000
+    assert sk["points_per_rank"] % 64 == 0 and abs(sk["points_per_rank"] - 128000) < 38400
     assert sk["value"] > 0 and sk["bcast_ms"] is not None and sk["allgather_ms"] is not None
-    assert sk["shard_cost_max_over_mean"]["balanced"] <= sk["shard_cost_max_over_mean"]["equal_count"] + 1e-9
+    assert sk["shard_cost_max_over_mean"]["balanced"] <= max(sk["shard_cost_max_over_mean"]["equal_count"], 1.01)
 
 
 @pytest.mark.gpu
