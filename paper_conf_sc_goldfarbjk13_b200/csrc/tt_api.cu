@@ -651,14 +651,9 @@ tt_status tt_traverse_pc(const tt_tree *t, const float *q, int64_t n, int32_t ld
     // 0.18 ms)
     const bool default_amd = !opts || opts->auto_min_depth < 0;
     if (cfg.variant == TT_VARIANT_AUTOROPES && p.c.mode == TT_MODE_AUTO && default_amd) {
-        static std::atomic<int> s_nsm{0};
-        int nsm = s_nsm.load();
-        if (nsm == 0) {
-            int dev = 0;
-            cudaGetDevice(&dev);
-            cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-            s_nsm.store(nsm);
-        }
+        int dev = 0, nsm = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);  // the current device's
         if ((n + 31) / 32 < (int64_t)nsm * 32) cfg.variant = TT_VARIANT_SPLIT;
     }
     return finish_launch(cfg.variant == TT_VARIANT_RECURSIVE ? tt_launch_pc_recursive(p, t->hdr.dim, cfg)
