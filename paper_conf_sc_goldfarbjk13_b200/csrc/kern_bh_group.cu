@@ -24,6 +24,8 @@
 
 #include <cub/device/device_scan.cuh>
 
+#include <algorithm>
+#include <cstdlib>
 #include <mutex>
 #include <type_traits>
 #include <unordered_map>
@@ -44,6 +46,7 @@ constexpr int kBlock = 256;
 constexpr int kSmemHdr = 384;          // mbarrier + dsq table (as kern_bh.cu)
 constexpr int kBPL = TT_BH_POINTS_PER_LANE;
 constexpr int kStackPerWarp = 8 * 40;  // <= 8 children pushed per level, height <= 33 (R9) + slack
+constexpr int kStackSmall = 8 * 24;    // height <= 22: the 1M / 16M configs (heights 18-20)
 constexpr int kFlushEvery = 16;        // children between fp32 -> fp64 flushes
 
 struct GroupEntry {
@@ -99,13 +102,24 @@ __device__ __forceinline__ float dsq_at(int dsq_bits, int lvl) { return __int_as
 #endif
 // WIDE: some node has more than 8 children (a depth-32 bucket of more than 8
 // coincident bodies, R9, or a custom tree): groups are staged 8 at a time.
-template <bool STATS, bool EXP_DSQ, bool WIDE>
+// Shared memory: header (mbarrier, dsq table) | per-warp group stacks of
+// stk_cap entries (8 per level: sized by the tree height) | per-warp staging
+// buffers (8 32-B records) | the first n_top group records -- the root's and
+// the top levels' child groups, which every tile walks -- staged once per
+// CTA by one bulk copy (TMA, UBLKCP) on an mbarrier (shallow
+// data in fast shared memory).  A group lying inside the staged prefix is
+// read in place; any other is staged from global memory by the warp.
+template <bool STATS, bool EXP_DSQ, bool WIDE, int STK>
 __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_bh_params P, const tt_oct_rec *grp,
                                                                                  const int *leaf_of, long long np,
-                                                                                 const int *gsrc) {
+                                                                                 const int *gsrc, int n_top) {
+    constexpr int stk_cap = STK;  // compile-time stack stride
     extern __shared__ __align__(128) unsigned char smem[];
+    uint64_t *bar = reinterpret_cast<uint64_t *>(smem);
     float *s_dsq = reinterpret_cast<float *>(smem + 16);
     GroupEntry *s_stack = reinterpret_cast<GroupEntry *>(smem + kSmemHdr);
+    float4 *s_stage = reinterpret_cast<float4 *>(s_stack + (kBlock / 32) * stk_cap);
+    float4 *s_top = s_stage + (kBlock / 32) * 16;
     if (threadIdx.x == 0) {
         float d = P.dsq_root;
         for (int l = 0; l < 64; ++l) {
@@ -113,14 +127,16 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
             d = __fmul_rn(d, 0.25f);
         }
     }
-    __syncthreads();
+    StageChunk ch[1] = {{s_top, grp, (unsigned)n_top * 32u}};
+    stage_top(bar, ch);
 
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
-    GroupEntry *stk = s_stack + warp * kStackPerWarp;
-    // per-warp staging buffer of one child group (<= 8 records)
-    float4 *gbuf = reinterpret_cast<float4 *>(s_stack + (kBlock / 32) * kStackPerWarp) + warp * 16;
-    int4 *tbuf = reinterpret_cast<int4 *>(gbuf + 8);
+    GroupEntry *stk = s_stack + warp * stk_cap;
+    // per-warp staging buffer of one child group (<= 8 32-B records {g, t});
+    // 32-bit shared addresses (no generic-address rebuild in the loop)
+    const unsigned gbuf_a = smem_addr(s_stage + warp * 16);
+    const unsigned top_a = smem_addr(s_top);
     const tt_oct_rec *g_rec = static_cast<const tt_oct_rec *>(P.c.tree.rec);
     const long long n = P.c.n;
     const int dsq_bits = __float_as_int(P.dsq_root);
@@ -229,18 +245,26 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                     const int gall = gnk;
                     for (int c0 = 0;; c0 += 8) {
                     const int cn = WIDE ? min(gall - c0, 8) : gall;
-                    if (lane < cn) {
-                        float4 sg;
-                        int4 st4;
-                        ldg_rec256(grp + goff + c0 + lane, sg, st4);
-                        gbuf[lane] = sg;
-                        tbuf[lane] = st4;
+                    // a group of the staged top levels is read in place
+                    const bool staged = goff + c0 + cn <= n_top;
+                    if (!staged) {
+                        if (lane < cn) {
+                            float4 sg;
+                            int4 st4;
+                            ldg_rec256(grp + goff + c0 + lane, sg, st4);
+                            asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};\n\t"
+                                         "st.shared.v4.s32 [%0+16], {%5, %6, %7, %8};"
+                                         :: "r"(gbuf_a + 32u * (unsigned)lane), "f"(sg.x), "f"(sg.y), "f"(sg.z),
+                                            "f"(sg.w), "r"(st4.x), "r"(st4.y), "r"(st4.z), "r"(st4.w)
+                                         : "memory");
+                        }
+                        __syncwarp();
                     }
-                    __syncwarp();
+                    const unsigned rb = staged ? top_a + 32u * (unsigned)(goff + c0) : gbuf_a;
 #pragma unroll 1
                     for (int k = 0; k < cn; ++k) {
-                        const float4 g = gbuf[k];
-                        const int4 t = tbuf[k];
+                        const float4 g = lds_f4(rb + 32u * (unsigned)k);
+                        const int4 t = lds_i4(rb + 32u * (unsigned)k + 16u);
                         if (STATS) {
                             ++fetches;
                             ++steps;
@@ -374,16 +398,30 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
     cta_finish(P.c.counter);
 }
 
-template <bool STATS, bool EXP_DSQ, bool WIDE>
+template <bool STATS, bool EXP_DSQ, bool WIDE, bool BIG_STK>
 int launch(const tt_bh_params &p, const tt_oct_rec *grp, const int *leaf_of, long long np, const int *gsrc,
-           const tt_launch_cfg &cfg) {
-    const size_t smem = kSmemHdr + (size_t)(kBlock / 32) * kStackPerWarp * sizeof(GroupEntry) + (kBlock / 32) * 16 * 16;
-    auto kern = bh_group_kernel<STATS, EXP_DSQ, WIDE>;
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return (int)e;
-    int dev = 0, nsm = 0, occ = 0;
+           long long n_groups, const tt_launch_cfg &cfg) {
+    // group stacks sized by the height: at most 8 cell children pushed per
+    // level of the current path (oct_flags TT_OCT_FEW_CELL_KIDS)
+    // (two compile-time sizes: 192 entries -- height <= 22, every config --
+    // or the 33-level maximum)
+    constexpr int STK = BIG_STK ? kStackPerWarp : kStackSmall;
+    const int stk_cap = STK;
+    const size_t base = kSmemHdr + (size_t)(kBlock / 32) * stk_cap * sizeof(GroupEntry) + (kBlock / 32) * 16 * 16;
+    // the staged top-level groups get what is left of the shared memory of
+    // TT_BHG_MINB CTAs per SM (TT_STAGE_BYTES overrides: tuning sweeps)
+    int dev = 0, nsm = 0, smem_sm = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev);
+    long long budget = (long long)smem_sm / TT_BHG_MINB - 1024 - (long long)base;  // 1 KB reserved per CTA
+    if (const char *ev = std::getenv("TT_STAGE_BYTES")) budget = std::atoll(ev);
+    long long n_top = std::max(0LL, std::min(n_groups, budget / 32));
+    const size_t smem = base + (size_t)n_top * 32;
+    auto kern = bh_group_kernel<STATS, EXP_DSQ, WIDE, STK>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return (int)e;
+    int occ = 0;
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kBlock, smem);
     if (e != cudaSuccess) return (int)e;
     if (cfg.ctas_per_sm > 0 && cfg.ctas_per_sm < occ) occ = cfg.ctas_per_sm;
@@ -393,7 +431,7 @@ int launch(const tt_bh_params &p, const tt_oct_rec *grp, const int *leaf_of, lon
     const long long need = (ntiles + kBlock / 32 - 1) / (kBlock / 32);
     if (grid > need) grid = need;
     if (grid < 1) grid = 1;
-    kern<<<(unsigned)grid, kBlock, smem, (cudaStream_t)cfg.stream>>>(p, grp, leaf_of, np, gsrc);
+    kern<<<(unsigned)grid, kBlock, smem, (cudaStream_t)cfg.stream>>>(p, grp, leaf_of, np, gsrc, (int)n_top);
     return (int)cudaGetLastError();
 }
 
@@ -509,10 +547,17 @@ int tt_launch_bh_group(const tt_bh_params &p, const void *grp, long long nn, lon
     const tt_oct_rec *g = static_cast<const tt_oct_rec *>(grp);
     const int *lf = reinterpret_cast<const int *>(g + nn);
     const int *gs = lf + np;
+    const bool big = 8 * (p.c.height + 2) > kStackSmall;
     if (wide) {  // rare (buckets of > 8 coincident bodies): no specialisations beyond stats
-        if (stats) return launch<true, false, true>(p, g, lf, np, gs, cfg);
-        return launch<false, false, true>(p, g, lf, np, gs, cfg);
+        if (stats) return launch<true, false, true, true>(p, g, lf, np, gs, nn, cfg);
+        return launch<false, false, true, true>(p, g, lf, np, gs, nn, cfg);
     }
-    if (stats) return exp_ok ? launch<true, true, false>(p, g, lf, np, gs, cfg) : launch<true, false, false>(p, g, lf, np, gs, cfg);
-    return exp_ok ? launch<false, true, false>(p, g, lf, np, gs, cfg) : launch<false, false, false>(p, g, lf, np, gs, cfg);
+    if (big) {
+        if (stats) return launch<true, false, false, true>(p, g, lf, np, gs, nn, cfg);
+        return launch<false, false, false, true>(p, g, lf, np, gs, nn, cfg);
+    }
+    if (stats) return exp_ok ? launch<true, true, false, false>(p, g, lf, np, gs, nn, cfg)
+                             : launch<true, false, false, false>(p, g, lf, np, gs, nn, cfg);
+    return exp_ok ? launch<false, true, false, false>(p, g, lf, np, gs, nn, cfg)
+                  : launch<false, false, false, false>(p, g, lf, np, gs, nn, cfg);
 }
