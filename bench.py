@@ -47,6 +47,15 @@ BYTES_PER_POINT_IO = {"bh": 32, "pc": 20, "knn": 28 + 64, "vp": 64 + 8, "nn": 28
 # with it: kd boxes, kNN children's boxes, VP / NN points), for node_fetch
 FETCH_BYTES = {"bh": 32, "pc": 32 + 32, "knn": 32 + 128, "vp": 16 + 64, "nn": 16 + 64 + 32}
 L2_FLUSH_BYTES = 256 << 20  # 2x the 126 MB L2
+# The paper's own numbers, other hardware (Tesla C2070: 14 SMs, vs 4 AMD
+# Opteron 6176, 32 threads): context only, never a ratio.
+PAPER_CONTEXT = {
+    "bh": {"claim": "speedups of up to 38x over 32-thread CPU versions (P:L29-31)",
+           "paper_traversal_ms": 669.07, "paper_visits_per_point": 3345,
+           "paper_speedup_vs_32_threads": 7.18,
+           "what": "Table 1, Barnes-Hut Plummer 1M bodies, sorted, lockstep (P:L1150)",
+           "hardware": "NVIDIA Tesla C2070 vs 4x AMD Opteron 6176 (P:L1096-1108)"},
+}
 
 
 def parse():
@@ -1028,6 +1037,7 @@ def run_ours(args, rank, world, local_rank):
         "group_build_ms": group_build_ms, "bcast_ms": bcast_ms, "placement_ms": placement_ms,
         "allgather_ms": allgather_ms,
         "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "strong_16m": strong, "strong_16m_knn": strong_knn,
+        "paper_context": PAPER_CONTEXT.get(name),
         "gpu_launches": (launches or 0) * args.steps,
         "gpu_launches_per_step": launches,
         "clocks": clocks,
