@@ -79,6 +79,7 @@ def parse():
     ap.add_argument("--no-strong", action="store_true",
                     help="skip the fixed-config strong-scaling block (configs[4] BH 16M, every N)")
     ap.add_argument("--strong-points", type=int, default=0, help="override the strong block's N (testing)")
+    ap.add_argument("--leaf", type=int, default=0, help="override the kd bucket size (tuning sweeps only)")
     ap.add_argument("--steps-order", default="sort", choices=["build", "sort"],
                     help="bhsteps traversal order: the GPU build's tree order, or tt_sort_points (Hilbert)")
     ap.add_argument("--auto-min-depth", type=int, default=None, help="AUTO-mode threshold (default: kernel's)")
@@ -604,6 +605,8 @@ def run_ours(args, rank, world, local_rank):
     w = make_workload(args.workload, world, args.points_per_rank)
     name = {"bh16m": "bh", "knn16m": "knn"}.get(args.workload, args.workload)
     c = w["cfg"]
+    if args.leaf:
+        c["leaf"] = args.leaf
     m = w["m"]
     if world > 1 and len(w["queries"]) % (64 * world):
         raise SystemExit(f"bench: {len(w['queries'])} points do not split into {world} equal warp-aligned "
