@@ -693,23 +693,24 @@ def run_ours(args, rank, world, local_rank):
     if name == "bh":  # the bodies' ids in the tree (original indices)
         self_ids = ids_all[lo:hi] if ids_all is not None else torch.arange(lo, hi, dtype=torch.int32, device=device)
 
-    def traverse(pts, res, order, stats=None):
+    def traverse(pts, res, order, stats=None, mode=None):
+        mode = mode or args.mode
         if name == "bh":
             P.tt_traverse_bh(tree, pts, c["theta"], c["eps"], out=res, self_ids=self_ids, order=order,
-                             mode=args.mode, auto_min_depth=args.auto_min_depth, stats=stats,
+                             mode=mode, auto_min_depth=args.auto_min_depth, stats=stats,
                              variant=args.variant)
         elif name == "knn":
-            P.tt_traverse_knn(tree, pts, c["k"], out_idx=res[0], out_d2=res[1], order=order, mode=args.mode,
+            P.tt_traverse_knn(tree, pts, c["k"], out_idx=res[0], out_d2=res[1], order=order, mode=mode,
                               auto_min_depth=args.auto_min_depth, stats=stats, variant=args.variant,
                               switch_below=args.switch_below)
         elif name == "vp":
-            P.tt_traverse_vp(tree, pts, out_idx=res[0], out_d2=res[1], order=order, mode=args.mode,
+            P.tt_traverse_vp(tree, pts, out_idx=res[0], out_d2=res[1], order=order, mode=mode,
                              auto_min_depth=args.auto_min_depth, stats=stats, variant=args.variant)
         elif name == "nn":
-            P.tt_traverse_nn(tree, pts, out_idx=res[0], out_d2=res[1], order=order, mode=args.mode,
+            P.tt_traverse_nn(tree, pts, out_idx=res[0], out_d2=res[1], order=order, mode=mode,
                              auto_min_depth=args.auto_min_depth, stats=stats)
         else:
-            P.tt_traverse_pc(tree, pts, c["radius"], out=res, order=order, mode=args.mode,
+            P.tt_traverse_pc(tree, pts, c["radius"], out=res, order=order, mode=mode,
                              auto_min_depth=args.auto_min_depth, stats=stats, variant=args.variant)
 
     if args.unsorted:
@@ -751,6 +752,22 @@ def run_ours(args, rank, world, local_rank):
     tiles = -(-m // tile_pts)
     wf = int(st.warp_fetches[:tiles].to(torch.int64).sum().item())
     lock_frac = float((st.warp_mode[:tiles] == 1).float().mean().item())
+    # Table 2's work expansion (reading R22): per lockstep warp
+    # tile, the nodes the warp tested / the longest independent traversal of
+    # its points (an extra, untimed independent-mode stats pass)
+    we_table2 = None
+    if lock_frac > 0 and args.variant in ("autoropes", "groups", "ropes"):
+        sn = P.Stats.alloc(m, device)
+        traverse(q_shard, out_shard, order_buf, sn, mode="independent")
+        torch.cuda.synchronize()
+        lanes = order_buf.long() if not args.unsorted else torch.arange(m, device=device)
+        vn = sn.visits.to(torch.float64)[lanes]
+        vn = torch.cat([vn, torch.zeros(tiles * tile_pts - m, dtype=torch.float64, device=device)])
+        longest = vn.view(tiles, tile_pts).max(1).values
+        lk = st.warp_mode[:tiles] == 1
+        tested = st.warp_steps[:tiles].to(torch.float64)
+        we_table2 = float((tested[lk] / longest[lk].clamp(min=1)).mean().item())
+        del sn, vn
     del st
 
     _trace("stats pass done")
@@ -1035,6 +1052,7 @@ def run_ours(args, rank, world, local_rank):
         # lane-slots offered by the warp fetches / useful visits (lockstep tiles)
         "work_expansion_fetch_over_visits": (wf * tile_pts / visits)
         if visits and lock_frac > 0.99 else None,
+        "work_expansion_table2": we_table2,
         "warp_tile_points": tile_pts,
         "traverse_ms": kms, "upload_ms": upload_ms, "tree_build_ms": build_ms, "tree_build": build_where,
         "group_build_ms": group_build_ms, "bcast_ms": bcast_ms, "placement_ms": placement_ms,
