@@ -17,7 +17,11 @@
 //
 // Group record (32 B, like tt_oct_rec): {com.xyz, mass} +
 // {group offset of the node's children | -1, number of children, body | -1,
-// level << 24}; entry 0 is the root, the children of a cell are contiguous.
+// level << 24 for a cell, kLeafLevel for a leaf}; entry 0 is the root, the
+// children of a cell are contiguous.  kLeafLevel makes a leaf's opening
+// distance negative (exponent path: dsq_bits - 0x7fffffff is a negative
+// float for every finite dsq_root > 0; table path: entry 127 is -1), so
+// `drsq < dl` alone is the opening test -- no separate "is a cell" compare.
 #include <climits>
 #include <cfloat>
 #include <cmath>
@@ -43,7 +47,8 @@ namespace {
 using namespace tt;
 
 constexpr int kBlock = 256;
-constexpr int kSmemHdr = 384;          // mbarrier + dsq table (as kern_bh.cu)
+constexpr int kSmemHdr = 640;          // mbarrier + dsq table of 128 levels (>= 64: leaves, -1)
+constexpr int kLeafLevel = 0x7fffffff; // level field of a leaf group record
 constexpr int kBPL = TT_BH_POINTS_PER_LANE;
 constexpr int kStackPerWarp = 8 * 40;  // <= 8 children pushed per level, height <= 33 (R9) + slack
 constexpr int kStackSmall = 8 * 24;    // height <= 22: the 1M / 16M configs (heights 18-20)
@@ -74,7 +79,7 @@ __global__ void groups_fill_kernel(const tt_oct_rec *rec, long long nn, const in
             tt_oct_rec r = rec[0];
             r.first_child = nk[0] > 0 ? 1 + goff[0] : -1;
             r.skip = nk[0];
-            r.level <<= 24;
+            r.level = r.first_child < 0 ? kLeafLevel : r.level << 24;
             grp[0] = r;
             gsrc[0] = 0;
             if (r.first_child < 0 && r.body >= 0 && r.body < np) leaf_of[r.body] = 0;
@@ -85,7 +90,8 @@ __global__ void groups_fill_kernel(const tt_oct_rec *rec, long long nn, const in
             tt_oct_rec r = rec[c];
             r.first_child = nk[c] > 0 ? 1 + goff[c] : -1;
             r.skip = nk[c];
-            r.level <<= 24;  // the exponent step of dsq_L (level * 2^24): one IADD per child
+            // the exponent step of dsq_L (level * 2^24): one IADD per child
+            r.level = r.first_child < 0 ? kLeafLevel : r.level << 24;
             grp[1 + goff[v] + k] = r;
             gsrc[1 + goff[v] + k] = c;  // the device node (stats hashes map it to its preorder id)
             if (r.first_child < 0 && r.body >= 0 && r.body < np) leaf_of[r.body] = 1 + goff[v] + k;
@@ -126,6 +132,7 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
             s_dsq[l] = d;
             d = __fmul_rn(d, 0.25f);
         }
+        for (int l = 64; l < 128; ++l) s_dsq[l] = -1.f;  // kLeafLevel >> 24 = 127
     }
     StageChunk ch[1] = {{s_top, grp, (unsigned)n_top * 32u}};
     stage_top(bar, ch);
@@ -238,6 +245,8 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                 constexpr bool SELF = decltype(self_chk)::value;
                 for (;;) {
                     const bool in0 = (m0 >> lane) & 1u, in1 = (m1 >> lane) & 1u;
+                    const float2 e2m = make_float2(in0 ? P.eps2 : __int_as_float(0x7f800000),
+                                                   in1 ? P.eps2 : __int_as_float(0x7f800000));
                     // stage the group: lane k loads child k (one request for the
                     // whole group, one round trip), the warp reads them back from
                     // shared memory with broadcast loads; the buffer holds 8
@@ -261,10 +270,9 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                         __syncwarp();
                     }
                     const unsigned rb = staged ? top_a + 32u * (unsigned)(goff + c0) : gbuf_a;
-#pragma unroll 1
-                    for (int k = 0; k < cn; ++k) {
-                        const float4 g = lds_f4(rb + 32u * (unsigned)k);
-                        const int4 t = lds_i4(rb + 32u * (unsigned)k + 16u);
+                    auto child = [&](unsigned a, int k) {
+                        const float4 g = lds_f4(a);
+                        const int4 t = lds_i4(a + 16u);
                         if (STATS) {
                             ++fetches;
                             ++steps;
@@ -279,23 +287,33 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                                 if (in1) vh[1].s += m;
                             }
                         }
+                        // a leaf's dl is negative (kLeafLevel): drsq < dl is the whole test
                         const float dl = EXP_DSQ ? __int_as_float(dsq_bits - t.w) : s_dsq[t.w >> 24];
                         const float2 dx = add2_rn(make_float2(g.x, g.x), nbx);
                         const float2 dy = add2_rn(make_float2(g.y, g.y), nby);
                         const float2 dz = add2_rn(make_float2(g.z, g.z), nbz);
                         const float2 drsq = add2_rn(add2_rn(sqr2_rn(dx, nz), sqr2_rn(dy, nz)), sqr2_rn(dz, nz));
-                        const bool cell = t.x >= 0;
-                        const bool o0 = in0 && cell && drsq.x < dl;
-                        const bool o1 = in1 && cell && drsq.y < dl;
-                        const bool k0 = in0 && !o0 && (!SELF || t.z != self[0]);
-                        const bool k1 = in1 && !o1 && (!SELF || t.z != self[1]);
-                        const float2 mw = make_float2(k0 ? g.w : 0.f, k1 ? g.w : 0.f);
-                        const float2 r = add2_rn(drsq, e22);
-                        const float2 inv = make_float2(rsqrt_ftz(r.x), rsqrt_ftz(r.y));
-                        float2 f = mul2_rn(mul2_rn(mw, mul2_rn(inv, inv)), inv);
-                        // the checked walk also serves eps = 0, where a skipped
-                        // leaf at distance 0 has inv = inf (0 * inf): select
-                        if (SELF) f = make_float2(k0 ? f.x : 0.f, k1 ? f.y : 0.f);
+                        const bool o0 = in0 && drsq.x < dl;
+                        const bool o1 = in1 && drsq.y < dl;
+                        float2 f;
+                        if (SELF) {
+                            const bool k0 = in0 && !o0 && t.z != self[0];
+                            const bool k1 = in1 && !o1 && t.z != self[1];
+                            const float2 mw = make_float2(k0 ? g.w : 0.f, k1 ? g.w : 0.f);
+                            const float2 r = add2_rn(drsq, e22);
+                            const float2 inv = make_float2(rsqrt_ftz(r.x), rsqrt_ftz(r.y));
+                            f = mul2_rn(mul2_rn(mw, mul2_rn(inv, inv)), inv);
+                            // the checked walk also serves eps = 0, where a skipped
+                            // leaf at distance 0 has inv = inf (0 * inf): select
+                            f = make_float2(k0 ? f.x : 0.f, k1 ? f.y : 0.f);
+                        } else {
+                            // a body outside the group's mask has r = inf, so inv = 0
+                            // and f = 0 exactly (eps > 0 here: active inv is finite)
+                            const float2 mw = make_float2(o0 ? 0.f : g.w, o1 ? 0.f : g.w);
+                            const float2 r = add2_rn(drsq, e2m);
+                            const float2 inv = make_float2(rsqrt_ftz(r.x), rsqrt_ftz(r.y));
+                            f = mul2_rn(mul2_rn(mw, mul2_rn(inv, inv)), inv);
+                        }
                         ax = fma2_rn(f, dx, ax);
                         ay = fma2_rn(f, dy, ay);
                         az = fma2_rn(f, dz, az);
@@ -306,7 +324,16 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                             if (lane == 0) stk[sp] = GroupEntry{t.x, t.y, om0, om1};
                             ++sp;
                         }
+                    };
+                    // two children per trip (the loop control and address
+                    // arithmetic of one trip serve both); pushes stay in child order
+                    int k = 0;
+#pragma unroll 1
+                    for (; k + 1 < cn; k += 2) {
+                        child(rb + 32u * (unsigned)k, k);
+                        child(rb + 32u * (unsigned)k + 32u, k + 1);
                     }
+                    if (k < cn) child(rb + 32u * (unsigned)k, k);
                     __syncwarp();  // the group buffer is reused by the next chunk / pop
                     if (!WIDE || c0 + 8 >= gall) break;
                     }
