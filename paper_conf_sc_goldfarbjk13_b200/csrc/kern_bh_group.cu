@@ -52,7 +52,8 @@ constexpr int kLeafLevel = 0x7fffffff; // level field of a leaf group record
 constexpr int kBPL = TT_BH_POINTS_PER_LANE;
 constexpr int kStackPerWarp = 8 * 40;  // <= 8 children pushed per level, height <= 33 (R9) + slack
 constexpr int kStackSmall = 8 * 24;    // height <= 22: the 1M / 16M configs (heights 18-20)
-constexpr int kFlushEvery = 16;        // children between fp32 -> fp64 flushes
+constexpr int kFlushEvery = 16;        // independent walk: steps between fp32 -> fp64 flushes
+constexpr int kFlushEveryL = 32;       // lockstep group walk: >= children between flushes
 
 struct GroupEntry {
     int off, nk;
@@ -125,7 +126,8 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
     float *s_dsq = reinterpret_cast<float *>(smem + 16);
     GroupEntry *s_stack = reinterpret_cast<GroupEntry *>(smem + kSmemHdr);
     float4 *s_stage = reinterpret_cast<float4 *>(s_stack + (kBlock / 32) * stk_cap);
-    float4 *s_top = s_stage + (kBlock / 32) * 16;
+    double *s_accb = reinterpret_cast<double *>(s_stage + (kBlock / 32) * 16);  // [6][kBlock]
+    float4 *s_top = reinterpret_cast<float4 *>(s_accb + 6 * kBlock);
     if (threadIdx.x == 0) {
         float d = P.dsq_root;
         for (int l = 0; l < 64; ++l) {
@@ -142,8 +144,13 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
     GroupEntry *stk = s_stack + warp * stk_cap;
     // per-warp staging buffer of one child group (<= 8 32-B records {g, t});
     // 32-bit shared addresses (no generic-address rebuild in the loop)
-    const unsigned gbuf_a = smem_addr(s_stage + warp * 16);
+    // (warp-uniform by construction; the shuffles let the compiler keep them
+    // in uniform registers, off the 64-register budget)
+    const unsigned gbuf_a = __shfl_sync(TT_FULL, smem_addr(s_stage + warp * 16), 0);
     const unsigned top_a = smem_addr(s_top);
+    const unsigned gbuf_l = gbuf_a + 32u * (unsigned)lane;  // this lane's staging slot
+    const tt_oct_rec *grp_l = grp + lane;                   // lane k stages child k
+    const unsigned lbit = 1u << lane;
     const tt_oct_rec *g_rec = static_cast<const tt_oct_rec *>(P.c.tree.rec);
     const long long n = P.c.n;
     const int dsq_bits = __float_as_int(P.dsq_root);
@@ -238,13 +245,27 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
             float2 ax = make_float2(0.f, 0.f), ay = ax, az = ax;
             int since_flush = 0;
             int sp = 0;
+            // the fp64 sums of the walk live in shared memory (this thread's
+            // column of s_acc[6][kBlock]): 12 registers fewer in the loop;
+            // a flush (every >= kFlushEveryL children) is 6 read-add-writes
+            double *s_acc = s_accb + threadIdx.x;
+#pragma unroll
+            for (int c = 0; c < 6; ++c) s_acc[c * kBlock] = 0.0;
+            auto flush_s = [&]() {
+                s_acc[0 * kBlock] += (double)ax.x;
+                s_acc[1 * kBlock] += (double)ay.x;
+                s_acc[2 * kBlock] += (double)az.x;
+                s_acc[3 * kBlock] += (double)ax.y;
+                s_acc[4 * kBlock] += (double)ay.y;
+                s_acc[5 * kBlock] += (double)az.y;
+            };
             // the root group: entry 0 alone, tested by every valid body
             int goff = 0, gnk = 1;
             unsigned m0 = __ballot_sync(TT_FULL, valid[0]), m1 = __ballot_sync(TT_FULL, valid[1]);
             auto walk = [&](auto self_chk) {
                 constexpr bool SELF = decltype(self_chk)::value;
                 for (;;) {
-                    const bool in0 = (m0 >> lane) & 1u, in1 = (m1 >> lane) & 1u;
+                    const bool in0 = (m0 & lbit) != 0u, in1 = (m1 & lbit) != 0u;
                     const float2 e2m = make_float2(in0 ? P.eps2 : __int_as_float(0x7f800000),
                                                    in1 ? P.eps2 : __int_as_float(0x7f800000));
                     // stage the group: lane k loads child k (one request for the
@@ -257,16 +278,16 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                     // a group of the staged top levels is read in place
                     const bool staged = goff + c0 + cn <= n_top;
                     if (!staged) {
-                        if (lane < cn) {
-                            float4 sg;
-                            int4 st4;
-                            ldg_rec256(grp + goff + c0 + lane, sg, st4);
-                            asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};\n\t"
-                                         "st.shared.v4.s32 [%0+16], {%5, %6, %7, %8};"
-                                         :: "r"(gbuf_a + 32u * (unsigned)lane), "f"(sg.x), "f"(sg.y), "f"(sg.z),
-                                            "f"(sg.w), "r"(st4.x), "r"(st4.y), "r"(st4.z), "r"(st4.w)
-                                         : "memory");
-                        }
+                        // lanes below cn: one 256-bit load, two 128-bit stores
+                        // (predicated, no divergent branch)
+                        asm volatile(
+                            "{\n\t.reg .pred p;\n\t.reg .b32 a<8>;\n\t"
+                            "setp.lt.s32 p, %0, %1;\n\t"
+                            "@p ld.global.nc.v8.b32 {a0, a1, a2, a3, a4, a5, a6, a7}, [%2];\n\t"
+                            "@p st.shared.v4.b32 [%3], {a0, a1, a2, a3};\n\t"
+                            "@p st.shared.v4.b32 [%3+16], {a4, a5, a6, a7};\n\t}"
+                            :: "r"(lane), "r"(cn), "l"(grp_l + (goff + c0)), "r"(gbuf_l)
+                            : "memory");
                         __syncwarp();
                     }
                     const unsigned rb = staged ? top_a + 32u * (unsigned)(goff + c0) : gbuf_a;
@@ -338,35 +359,36 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                     if (!WIDE || c0 + 8 >= gall) break;
                     }
                     since_flush += gall;
-                    if (since_flush >= kFlushEvery) {  // warp-uniform cadence
-                        X[0] += (double)ax.x;
-                        Y[0] += (double)ay.x;
-                        Z[0] += (double)az.x;
-                        X[1] += (double)ax.y;
-                        Y[1] += (double)ay.y;
-                        Z[1] += (double)az.y;
+                    if (since_flush >= kFlushEveryL) {  // warp-uniform cadence
+                        flush_s();
                         ax = ay = az = make_float2(0.f, 0.f);
                         since_flush = 0;
                     }
                     if (sp == 0) break;
                     --sp;
                     __syncwarp();
-                    int4 e = make_int4(0, 0, 0, 0);
-                    if (lane == 0) e = *reinterpret_cast<const int4 *>(stk + sp);
+                    // every lane reads the entry lane 0 pushed (one broadcast load);
+                    // the group's offset and size pass through a shuffle so the
+                    // compiler sees them warp-uniform (uniform loop control)
+                    // (a plain C++ load: ordered after lane 0's plain-store push
+                    // and the __syncwarp, which an asm load without a memory
+                    // clobber is not)
+                    const int4 e = *reinterpret_cast<const int4 *>(stk + sp);
                     goff = __shfl_sync(TT_FULL, e.x, 0);
                     gnk = __shfl_sync(TT_FULL, e.y, 0);
-                    m0 = (unsigned)__shfl_sync(TT_FULL, e.z, 0);
-                    m1 = (unsigned)__shfl_sync(TT_FULL, e.w, 0);
+                    m0 = (unsigned)e.z;
+                    m1 = (unsigned)e.w;
                 }
             };
             if (need_self) walk(std::true_type{});
             else walk(std::false_type{});
-            X[0] += (double)ax.x;
-            Y[0] += (double)ay.x;
-            Z[0] += (double)az.x;
-            X[1] += (double)ax.y;
-            Y[1] += (double)ay.y;
-            Z[1] += (double)az.y;
+            flush_s();
+            X[0] = s_acc[0 * kBlock];
+            Y[0] = s_acc[1 * kBlock];
+            Z[0] = s_acc[2 * kBlock];
+            X[1] = s_acc[3 * kBlock];
+            Y[1] = s_acc[4 * kBlock];
+            Z[1] = s_acc[5 * kBlock];
         } else {
             // independent: the stackless rope walk of kern_bh.cu over the
             // preorder records (through L1/L2)
@@ -434,7 +456,8 @@ int launch(const tt_bh_params &p, const tt_oct_rec *grp, const int *leaf_of, lon
     // or the 33-level maximum)
     constexpr int STK = BIG_STK ? kStackPerWarp : kStackSmall;
     const int stk_cap = STK;
-    const size_t base = kSmemHdr + (size_t)(kBlock / 32) * stk_cap * sizeof(GroupEntry) + (kBlock / 32) * 16 * 16;
+    const size_t base = kSmemHdr + (size_t)(kBlock / 32) * stk_cap * sizeof(GroupEntry) + (kBlock / 32) * 16 * 16 +
+                        6 * kBlock * sizeof(double);
     // the staged top-level groups get what is left of the shared memory of
     // TT_BHG_MINB CTAs per SM (TT_STAGE_BYTES overrides: tuning sweeps)
     int dev = 0, nsm = 0, smem_sm = 0;
