@@ -346,15 +346,23 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                             ++sp;
                         }
                     };
-                    // two children per trip (the loop control and address
-                    // arithmetic of one trip serve both); pushes stay in child order
-                    int k = 0;
-#pragma unroll 1
-                    for (; k + 1 < cn; k += 2) {
-                        child(rb + 32u * (unsigned)k, k);
-                        child(rb + 32u * (unsigned)k + 32u, k + 1);
+                    // straight-line: enter the unrolled sequence of 8 at 8 - cn
+                    // (one indirect jump per group, no per-child loop control;
+                    // pushes stay in child order).  3.18 vs 3.20 ms for a loop
+                    // of two children per trip, 3.32 for one.
+                    {
+                        const unsigned rb8 = rb - 32u * (unsigned)(8 - cn);
+                        switch (8 - cn) {
+                        case 0: child(rb8 + 0u, cn - 8); [[fallthrough]];
+                        case 1: child(rb8 + 32u, cn - 7); [[fallthrough]];
+                        case 2: child(rb8 + 64u, cn - 6); [[fallthrough]];
+                        case 3: child(rb8 + 96u, cn - 5); [[fallthrough]];
+                        case 4: child(rb8 + 128u, cn - 4); [[fallthrough]];
+                        case 5: child(rb8 + 160u, cn - 3); [[fallthrough]];
+                        case 6: child(rb8 + 192u, cn - 2); [[fallthrough]];
+                        default: child(rb8 + 224u, cn - 1);
+                        }
                     }
-                    if (k < cn) child(rb + 32u * (unsigned)k, k);
                     __syncwarp();  // the group buffer is reused by the next chunk / pop
                     if (!WIDE || c0 + 8 >= gall) break;
                     }
