@@ -138,11 +138,6 @@ __global__ void __launch_bounds__(kBlock, TT_KNN_MINB) knn_kernel(const tt_knn_p
     unsigned char *s_rec = smem + kSmemHdr;
     float *s_cbox = reinterpret_cast<float *>(s_rec + (size_t)top * 32);
     unsigned char *s_stack = reinterpret_cast<unsigned char *>(s_cbox) + (size_t)top * 16 * DP;
-    // each thread's query, [DIM][kBlock] (bank = lane for any dim): the split
-    // coordinate q[dim] of a node is one indexed load instead of a DIM-way
-    // select chain (the query stays in registers for the distance sums)
-    float *s_q = reinterpret_cast<float *>(s_stack + (size_t)kWarps * knn_stack_bytes(cap, g_lb == nullptr)) +
-                 threadIdx.x;
     const tt_kd_rec *g_rec = static_cast<const tt_kd_rec *>(P.c.tree.rec);
     const float *g_cbox = P.c.tree.cbox;
     StageChunk ch[2] = {{s_rec, g_rec, (unsigned)top * 32u}, {s_cbox, g_cbox, (unsigned)top * 16u * DP}};
@@ -181,8 +176,6 @@ __global__ void __launch_bounds__(kBlock, TT_KNN_MINB) knn_kernel(const tt_knn_p
 #pragma unroll
             for (int d = 0; d < DIM; ++d) q[d] = 0.f;
         const unsigned vmask = __ballot_sync(TT_FULL, valid);
-#pragma unroll
-        for (int d = 0; d < DIM; ++d) s_q[d * kBlock] = q[d];  // read back by this thread only
 
         bool lock = P.c.mode == TT_MODE_LOCKSTEP;
         if (P.c.mode == TT_MODE_AUTO && P.c.auto_min_depth >= 0 && P.c.auto_min_depth < 64) {
@@ -297,7 +290,7 @@ __global__ void __launch_bounds__(kBlock, TT_KNN_MINB) knn_kernel(const tt_knn_p
                     } else {
                         float lbl, lbr;
                         child_lbs<DIM>(s_cbox, g_cbox, DP, top, cur, q, lbl, lbr);
-                        const bool pref_left = active && s_q[u.y * kBlock] < __int_as_float(u.x);
+                        const bool pref_left = active && select_dim<DIM>(q, u.y) < __int_as_float(u.x);
                         const int votes = __popc(__ballot_sync(TT_FULL, pref_left));
                         const bool left_first = 2 * votes >= __popc(act);
                         if (lane == 0) {  // push second (warp-uniform entry)
@@ -347,7 +340,7 @@ __global__ void __launch_bounds__(kBlock, TT_KNN_MINB) knn_kernel(const tt_knn_p
                     } else {
                         float lbl, lbr;
                         child_lbs<DIM>(s_cbox, g_cbox, DP, top, cur, q, lbl, lbr);
-                        const bool left_near = s_q[u.y * kBlock] < __int_as_float(u.x);
+                        const bool left_near = select_dim<DIM>(q, u.y) < __int_as_float(u.x);
                         n_node[sp * 32 + lane] = left_near ? t.y : t.x;  // push far with its bound
                         n_lbs[sp * lbs_stride + lbs_lane] = left_near ? lbr : lbl;
                         ++sp;
@@ -396,8 +389,7 @@ int launch(const tt_knn_params &p, const tt_launch_cfg &cfg) {
     constexpr int DP = (DIM + 3) & ~3;
     const int cap = p.c.height + 2;
     const bool wide = p.c.mode == TT_MODE_INDEPENDENT;
-    const size_t smem = kSmemHdr + (size_t)p.c.top_count * (32 + 16 * DP) + (size_t)kWarps * knn_stack_bytes(cap, wide) +
-                        sizeof(float) * DIM * kBlock;
+    const size_t smem = kSmemHdr + (size_t)p.c.top_count * (32 + 16 * DP) + (size_t)kWarps * knn_stack_bytes(cap, wide);
     auto kern = knn_kernel<DIM, KT, STATS>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return (int)e;
