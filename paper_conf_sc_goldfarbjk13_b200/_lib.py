@@ -10,7 +10,9 @@ import ctypes as C
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libtt.so")
+# TT_LIB=checked loads the bounds-checked build (build.py --checked,
+# tt_check.cuh): the same C ABI with device-side asserts
+LIB_PATH = os.path.join(HERE, "libtt_checked.so" if os.environ.get("TT_LIB") == "checked" else "libtt.so")
 
 TT_OK = 0
 STATUS = {0: "TT_OK", -1: "TT_ERR_INVALID_ARG", -2: "TT_ERR_CUDA", -3: "TT_ERR_OOM",

@@ -36,6 +36,7 @@
 #include <vector>
 
 #include "kern_common.cuh"
+#include "tt_check.cuh"
 
 // a negative self id means "no self leaf": -2 matches no record's body field
 // (cells carry -1 there)
@@ -119,7 +120,8 @@ __device__ __forceinline__ float dsq_at(int dsq_bits, int lvl) { return __int_as
 template <bool STATS, bool EXP_DSQ, bool WIDE, int STK>
 __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_bh_params P, const tt_oct_rec *grp,
                                                                                  const int *leaf_of, long long np,
-                                                                                 const int *gsrc, int n_top) {
+                                                                                 const int *gsrc, int n_top,
+                                                                                 long long n_groups) {
     constexpr int stk_cap = STK;  // compile-time stack stride
     extern __shared__ __align__(128) unsigned char smem[];
     uint64_t *bar = reinterpret_cast<uint64_t *>(smem);
@@ -225,6 +227,7 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
             ok[j] = !valid[j] || self[j] < 0 || (long long)self[j] >= np;
             if (!ok[j]) {
                 const int lf = __ldg(leaf_of + self[j]);
+                TT_DCHECK(lf < n_groups);
                 if (lf < 0) {
                     ok[j] = true;  // no leaf is tested against this id
                 } else {
@@ -275,6 +278,7 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                     const int gall = gnk;
                     for (int c0 = 0;; c0 += 8) {
                     const int cn = WIDE ? min(gall - c0, 8) : gall;
+                    TT_DCHECK(cn >= 1 && cn <= 8 && goff >= 0 && goff + c0 + cn <= n_groups);
                     // a group of the staged top levels is read in place
                     const bool staged = goff + c0 + cn <= n_top;
                     if (!staged) {
@@ -342,6 +346,7 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                         // opens it (one vote: -1.5% vs two ballots per child)
                         if (__any_sync(TT_FULL, o0 || o1)) {
                             const unsigned om0 = __ballot_sync(TT_FULL, o0), om1 = __ballot_sync(TT_FULL, o1);
+                            TT_DCHECK(sp < stk_cap && t.x >= 1 && t.y >= 1);
                             if (lane == 0) stk[sp] = GroupEntry{t.x, t.y, om0, om1};
                             ++sp;
                         }
@@ -384,6 +389,8 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                     const int4 e = *reinterpret_cast<const int4 *>(stk + sp);
                     goff = __shfl_sync(TT_FULL, e.x, 0);
                     gnk = __shfl_sync(TT_FULL, e.y, 0);
+                    TT_DCHECK(sp >= 0 && gnk >= 1 && (WIDE || gnk <= 8) && goff >= 1 && goff + gnk <= n_groups &&
+                              __shfl_sync(TT_FULL, e.z, 0) == e.z && __shfl_sync(TT_FULL, e.w, 0) == e.w);
                     m0 = (unsigned)e.z;
                     m1 = (unsigned)e.w;
                 }
@@ -408,6 +415,7 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                 while (cur != TT_END) {
                     float4 g;
                     int4 t;
+                    TT_DCHECK(cur >= 0 && cur < n_groups);
                     ldg_rec256(g_rec + cur, g, t);
                     if (STATS) {
                         ++visits[j];
@@ -489,7 +497,7 @@ int launch(const tt_bh_params &p, const tt_oct_rec *grp, const int *leaf_of, lon
     const long long need = (ntiles + kBlock / 32 - 1) / (kBlock / 32);
     if (grid > need) grid = need;
     if (grid < 1) grid = 1;
-    kern<<<(unsigned)grid, kBlock, smem, (cudaStream_t)cfg.stream>>>(p, grp, leaf_of, np, gsrc, (int)n_top);
+    kern<<<(unsigned)grid, kBlock, smem, (cudaStream_t)cfg.stream>>>(p, grp, leaf_of, np, gsrc, (int)n_top, n_groups);
     return (int)cudaGetLastError();
 }
 
