@@ -151,7 +151,6 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
     const unsigned gbuf_a = __shfl_sync(TT_FULL, smem_addr(s_stage + warp * 16), 0);
     const unsigned top_a = smem_addr(s_top);
     const unsigned gbuf_l = gbuf_a + 32u * (unsigned)lane;  // this lane's staging slot
-    const tt_oct_rec *grp_l = grp + lane;                   // lane k stages child k
     const unsigned lbit = 1u << lane;
     const tt_oct_rec *g_rec = static_cast<const tt_oct_rec *>(P.c.tree.rec);
     const long long n = P.c.n;
@@ -283,14 +282,17 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                     const bool staged = goff + c0 + cn <= n_top;
                     if (!staged) {
                         // lanes below cn: one 256-bit load, two 128-bit stores
-                        // (predicated, no divergent branch)
+                        // (predicated, no divergent branch).  32-bit record index:
+                        // the launcher keeps groups to trees of < 2^27 nodes, so
+                        // index * 32 B fits 32 bits
+                        const unsigned gi = (unsigned)(goff + c0 + lane);
                         asm volatile(
                             "{\n\t.reg .pred p;\n\t.reg .b32 a<8>;\n\t"
                             "setp.lt.s32 p, %0, %1;\n\t"
                             "@p ld.global.nc.v8.b32 {a0, a1, a2, a3, a4, a5, a6, a7}, [%2];\n\t"
                             "@p st.shared.v4.b32 [%3], {a0, a1, a2, a3};\n\t"
                             "@p st.shared.v4.b32 [%3+16], {a4, a5, a6, a7};\n\t}"
-                            :: "r"(lane), "r"(cn), "l"(grp_l + (goff + c0)), "r"(gbuf_l)
+                            :: "r"(lane), "r"(cn), "l"(reinterpret_cast<const char *>(grp) + gi * 32u), "r"(gbuf_l)
                             : "memory");
                         __syncwarp();
                     }
