@@ -245,7 +245,7 @@ __global__ void __launch_bounds__(kBlock, 4) bh_kernel(const tt_bh_params P) {
                     const float2 dy = add2_rn(make_float2(g.y, g.y), nby[p]);
                     const float2 dz = add2_rn(make_float2(g.z, g.z), nbz[p]);
                     // rn(rn(rn(dx^2) + rn(dy^2)) + rn(dz^2)): the pinned order (R0)
-                    const float2 drsq = add2_rn(add2_rn(sqr2_rn(dx, nz), sqr2_rn(dy, nz)), sqr2_rn(dz, nz));
+                    const float2 drsq = fma2_rn(dz, dz, fma2_rn(dy, dy, sqr2_rn(dx, nz)));  // R8
                     const bool a0 = lvl <= w[2 * p], a1 = lvl <= w[2 * p + 1];
                     const bool o0 = a0 && cell && drsq.x < dl;
                     const bool o1 = a1 && cell && drsq.y < dl;
@@ -325,11 +325,10 @@ __global__ void __launch_bounds__(kBlock, 4) bh_kernel(const tt_bh_params P) {
                             ++bd[j].visits;
                             if (P.c.pre) vh.add(P.c.pre, cur);
                         }
-                        float dx, dy, sx, sy;
+                        float dx, dy;
                         sub2_rn(g.x, g.y, bd[j].b.x, bd[j].b.y, dx, dy);
-                        sqr2_rn(dx, dy, sx, sy);
                         const float dz = __fsub_rn(g.z, bd[j].b.z);
-                        const float drsq = __fadd_rn(__fadd_rn(sx, sy), __fmul_rn(dz, dz));
+                        const float drsq = __fmaf_rn(dz, dz, __fmaf_rn(dy, dy, __fmul_rn(dx, dx)));  // R8
                         const bool open = t.x >= 0 && drsq < dsq(t.w);
                         const float inv = rsqrt_ftz(__fadd_rn(drsq, eps2));
                         const float f = (!open && t.z != bd[j].self) ? g.w * (inv * inv) * inv : 0.0f;

@@ -319,7 +319,8 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                         const float2 dx = add2_rn(make_float2(g.x, g.x), nbx);
                         const float2 dy = add2_rn(make_float2(g.y, g.y), nby);
                         const float2 dz = add2_rn(make_float2(g.z, g.z), nbz);
-                        const float2 drsq = add2_rn(add2_rn(sqr2_rn(dx, nz), sqr2_rn(dy, nz)), sqr2_rn(dz, nz));
+                        // |dr|^2 = fma(dz, dz, fma(dy, dy, dx * dx)) (R8), 3 instructions
+                        const float2 drsq = fma2_rn(dz, dz, fma2_rn(dy, dy, sqr2_rn(dx, nz)));
                         const bool o0 = in0 && drsq.x < dl;
                         const bool o1 = in1 && drsq.y < dl;
                         float2 f;
@@ -425,7 +426,7 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                     }
                     const float dx = __fsub_rn(g.x, b[j].x), dy = __fsub_rn(g.y, b[j].y),
                                 dz = __fsub_rn(g.z, b[j].z);
-                    const float drsq = __fadd_rn(__fadd_rn(__fmul_rn(dx, dx), __fmul_rn(dy, dy)), __fmul_rn(dz, dz));
+                    const float drsq = __fmaf_rn(dz, dz, __fmaf_rn(dy, dy, __fmul_rn(dx, dx)));  // R8
                     const float dl = EXP_DSQ ? dsq_at(dsq_bits, t.w) : s_dsq[t.w];
                     const bool open = t.x >= 0 && drsq < dl;
                     const float inv = rsqrt_ftz(__fadd_rn(drsq, P.eps2));

@@ -42,7 +42,7 @@ __device__ void bh_rec(BhCtx &c, int node, float dsq) {
     const float4 g = __ldg(reinterpret_cast<const float4 *>(&c.rec[node].gx));
     const int4 t = __ldg(reinterpret_cast<const int4 *>(&c.rec[node].first_child));
     const float dx = __fsub_rn(g.x, c.b.x), dy = __fsub_rn(g.y, c.b.y), dz = __fsub_rn(g.z, c.b.z);
-    const float drsq = __fadd_rn(__fadd_rn(__fmul_rn(dx, dx), __fmul_rn(dy, dy)), __fmul_rn(dz, dz));
+    const float drsq = __fmaf_rn(dz, dz, __fmaf_rn(dy, dy, __fmul_rn(dx, dx)));  // R8
     if (t.x >= 0 && drsq < dsq) {  // !far_enough && type != LEAF (Fig.9a line 2)
         const float cd = __fmul_rn(dsq, 0.25f);
         // children of a cell: first_child, then the rope chain of siblings

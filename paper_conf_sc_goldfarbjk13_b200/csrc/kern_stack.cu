@@ -69,7 +69,7 @@ struct BhLane {
 // s_dsq[L] = dsq_root * 0.25^L ("dsq*0.25" per level, Fig.9a line 4).
 __device__ __forceinline__ bool bh_visit(BhLane &L, float4 g, int4 t, const float *s_dsq, float eps2) {
     const float dx = __fsub_rn(g.x, L.b.x), dy = __fsub_rn(g.y, L.b.y), dz = __fsub_rn(g.z, L.b.z);
-    const float drsq = __fadd_rn(__fadd_rn(__fmul_rn(dx, dx), __fmul_rn(dy, dy)), __fmul_rn(dz, dz));
+    const float drsq = __fmaf_rn(dz, dz, __fmaf_rn(dy, dy, __fmul_rn(dx, dx)));  // R8
     if (t.x >= 0 && drsq < s_dsq[t.w]) return true;
     if (t.z != L.self) {
         const float inv = rsqrt_ftz(__fadd_rn(drsq, eps2));
