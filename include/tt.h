@@ -345,7 +345,17 @@ typedef enum tt_variant {
  * point i skips (R9); a negative id skips nothing.  A cell is opened iff it is a cell and
  * |com - x|^2 < dsq_L, dsq_L = dsq_root * 0.25^L, dsq_root = (side/theta)^2
  * (theta == 0 -> +inf: every cell opened).  acc_out: float4 (ax,ay,az,0),
- * G = 1, softening eps.  Opening decisions use the pinned fp32 sequence R0. */
+ * G = 1, softening eps.  Opening decisions use pinned fp32 arithmetic:
+ * |com - x|^2 = fma(dz, dz, fma(dy, dy, dx*dx)) (reading R8).
+ * Variants: AUTOROPES (default) walks lockstep warps by child groups
+ * (TT_VARIANT_GROUPS) when the tree allows it -- height <= 38, <= 8 cell
+ * children per cell, < 2^27 nodes -- else by per-node ropes (ROPES);
+ * requesting GROUPS for a tree that does not allow it returns
+ * TT_ERR_TREE_TOO_DEEP (height / children) or TT_ERR_UNSUPPORTED (size).
+ * Opt-in, environment TT_L2_PERSIST_MB=<MiB>: an L2 persisting access-policy
+ * window over the top of the tree for each launch (device-wide set-aside;
+ * the stream's window is cleared after the launch; not inside a graph
+ * capture).  Results never depend on it. */
 tt_status tt_traverse_bh(const tt_tree *t, const float *bodies, const int32_t *self_ids, int64_t n,
                          float theta, float eps, float *acc_out, const tt_traverse_opts *opts,
                          tt_stream s);

@@ -627,12 +627,14 @@ tt_status tt_traverse_bh(const tt_tree *t, const float *bodies, const int32_t *s
     // oct_flags -- take the stackless per-node walk, or fail if groups were
     // requested; more than 8 children in all (depth-32 buckets) are staged 8
     // at a time by the WIDE kernel)
-    const bool groups_fit = 8 * (t->hdr.height + 2) <= 320 &&  // kStackPerWarp of kern_bh_group.cu
-                            (t->hdr.oct_flags & TT_OCT_FEW_CELL_KIDS) &&
-                            t->hdr.n_nodes < (1LL << 27);  // 32-bit byte offsets into the group array
+    const bool groups_shape = 8 * (t->hdr.height + 2) <= 320 &&  // kStackPerWarp of kern_bh_group.cu
+                              (t->hdr.oct_flags & TT_OCT_FEW_CELL_KIDS);
+    const bool groups_size = t->hdr.n_nodes < (1LL << 27);  // 32-bit byte offsets into the group array
+    const bool groups_fit = groups_shape && groups_size;
     const bool wide = !(t->hdr.oct_flags & TT_OCT_NARROW);
     if (cfg.variant == TT_VARIANT_AUTOROPES) cfg.variant = groups_fit ? TT_VARIANT_GROUPS : TT_VARIANT_ROPES;
-    if (cfg.variant == TT_VARIANT_GROUPS && !groups_fit) return TT_ERR_TREE_TOO_DEEP;
+    if (cfg.variant == TT_VARIANT_GROUPS && !groups_shape) return TT_ERR_TREE_TOO_DEEP;
+    if (cfg.variant == TT_VARIANT_GROUPS && !groups_size) return TT_ERR_UNSUPPORTED;
     if (cfg.variant == TT_VARIANT_GROUPS) {
         tt_tree *mt = const_cast<tt_tree *>(t);
         std::lock_guard<std::mutex> lk(mt->grp_mu);
