@@ -5,8 +5,9 @@
 // the same warp:
 //   kd : leaf reached by "left iff x[dim] < split" -> its first tree-order
 //        point index (leaves are numbered in preorder);
-//   oct: 63-bit octant path through the root cube (fp64 comparisons exactly as
-//        the build partitions bodies) = Morton order = preorder of leaves;
+//   oct: the point's 16-level cell of the cube hierarchy (octant bits from
+//        fp64 comparisons exactly as the build partitions bodies), ordered
+//        along the 3-D Hilbert curve (48-bit key, reading R18b);
 //   vp : 2-bit-per-level code (inside = 01, outside = 10, end = 00) of the
 //        inside-iff-d<=r_in_max descent; a node sorts before its subtree;
 //   nn : the same code (left = 01, right = 10) of the left-iff-x[dim]<split

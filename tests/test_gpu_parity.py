@@ -383,6 +383,20 @@ def test_sort_points_matches_oracle_for_every_kind():
         assert np.array_equal(perm.cpu().numpy(), oracle.sort_perm(ot, pts))
 
 
+@pytest.mark.parametrize("n", [1, 33, 16384, 16385])
+def test_kd_sort_sizes_with_equal_keys(n):
+    """kd sorts from one point to past 2^14 points (a one-CTA shared-memory
+    sort for <= 16384 points was tried there and measured no faster, DESIGN
+    §4.6) equal the oracle's stable (key, index) order, with many equal keys
+    (leaf 8)."""
+    p = ttgen.gaussian_mixture(20000, 3, seed=215, components=6)
+    host, ot = P.build_kd(p, 8), oracle.build_kd(p, 8)
+    tree = P.tt_tree_upload(host)
+    q = np.ascontiguousarray(p[np.random.default_rng(n).integers(0, len(p), n)])
+    perm = P.tt_sort_points(tree, dev(q))
+    assert np.array_equal(perm.cpu().numpy(), oracle.sort_perm(ot, q))
+
+
 # ------------------------------------------------------------ edges / misc
 def test_empty_and_partial_warp():
     p = ttgen.uniform(1000, 3, seed=214)
