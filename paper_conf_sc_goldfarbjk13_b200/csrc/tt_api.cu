@@ -279,9 +279,8 @@ struct L2Window {
         v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
         const cudaError_t e = cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &v);
         on = e == cudaSuccess;
-        static bool told = false;
-        if (!told) {  // asked for explicitly: say what was set
-            told = true;
+        static std::atomic<bool> told{false};
+        if (!told.exchange(true)) {  // asked for explicitly: say (once) what was set
             std::fprintf(stderr, "tt: L2 persisting window %s: %zu MiB of %zu MiB, hit ratio %.2f\n",
                          on ? "set" : cudaGetErrorString(e), limit >> 20,
                          (size_t)v.accessPolicyWindow.num_bytes >> 20, v.accessPolicyWindow.hitRatio);
