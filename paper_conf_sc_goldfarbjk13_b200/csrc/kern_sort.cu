@@ -34,40 +34,47 @@ __global__ void iota_kernel(uint32_t *v, long long n) {
 // key: 6 radix passes instead of 8.
 constexpr int kOctKeyLevels = 16;
 
+// spread the low 16 bits of v to every third bit (bit b -> bit 3b)
+__device__ __forceinline__ unsigned long long spread3(unsigned v) {
+    unsigned long long x = v & 0xffffull;
+    x = (x | (x << 16)) & 0x0000ff0000ffull;
+    x = (x | (x << 8)) & 0x00f00f00f00full;
+    x = (x | (x << 4)) & 0x0c30c30c30c3ull;
+    x = (x | (x << 2)) & 0x249249249249ull;
+    return x;
+}
+
 // Hilbert index (Skilling's transpose algorithm) of the kOctKeyLevels-level
 // cell whose coordinate bits are (ix, iy, iz), bits interleaved x, y, z from
-// the top
+// the top.  Branch-free and unrolled (the per-bit exchange as selects: lanes
+// of a warp take different branches), the interleave by bit spreading.
 __device__ __forceinline__ unsigned long long hilbert_key(unsigned ix, unsigned iy, unsigned iz) {
     unsigned X[3] = {ix, iy, iz};
-#pragma unroll 1
+#pragma unroll
     for (unsigned Q = 1u << (kOctKeyLevels - 1); Q > 1; Q >>= 1) {
         const unsigned P = Q - 1;
 #pragma unroll
         for (int i = 0; i < 3; ++i) {
-            if (X[i] & Q) {
-                X[0] ^= P;
+            // X[i] & Q: invert the low bits of X[0]; else exchange them with X[i]'s
+            const bool inv = (X[i] & Q) != 0;
+            const unsigned t = (X[0] ^ X[i]) & P;
+            if (i == 0) {
+                X[0] ^= inv ? P : 0u;  // (t == 0 for i == 0)
             } else {
-                const unsigned t = (X[0] ^ X[i]) & P;
-                X[0] ^= t;
-                X[i] ^= t;
+                X[0] ^= inv ? P : t;
+                X[i] ^= inv ? 0u : t;
             }
         }
     }
     X[1] ^= X[0];
     X[2] ^= X[1];
     unsigned t = 0;
-#pragma unroll 1
-    for (unsigned Q = 1u << (kOctKeyLevels - 1); Q > 1; Q >>= 1)
-        if (X[2] & Q) t ^= Q - 1;
+#pragma unroll
+    for (unsigned Q = 1u << (kOctKeyLevels - 1); Q > 1; Q >>= 1) t ^= (X[2] & Q) ? Q - 1 : 0u;
     X[0] ^= t;
     X[1] ^= t;
     X[2] ^= t;
-    unsigned long long h = 0;
-#pragma unroll 1
-    for (int b = kOctKeyLevels - 1; b >= 0; --b)
-        h = (h << 3) | ((unsigned long long)((X[0] >> b) & 1u) << 2) | ((unsigned long long)((X[1] >> b) & 1u) << 1) |
-            (unsigned long long)((X[2] >> b) & 1u);
-    return h;
+    return (spread3(X[0]) << 2) | (spread3(X[1]) << 1) | spread3(X[2]);
 }
 
 // Oct sort key (reading R18b): the kOctKeyLevels-level cell of the point's descent
