@@ -268,8 +268,13 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                 constexpr bool SELF = decltype(self_chk)::value;
                 for (;;) {
                     const bool in0 = (m0 & lbit) != 0u, in1 = (m1 & lbit) != 0u;
-                    const float2 e2m = make_float2(in0 ? P.eps2 : __int_as_float(0x7f800000),
-                                                   in1 ? P.eps2 : __int_as_float(0x7f800000));
+                    // the group's mask as the addend of the first square: +0 for
+                    // a body in the mask (fma(dx, dx, +0) = rn(dx^2), R8's value),
+                    // +inf outside it -- its |dr|^2 is then +inf, so it never
+                    // opens a child (no mask predicate per child) and its r is
+                    // +inf, inv = 0, f = 0 exactly
+                    const float2 zm = make_float2(in0 ? 0.f : __int_as_float(0x7f800000),
+                                                  in1 ? 0.f : __int_as_float(0x7f800000));
                     // stage the group: lane k loads child k (one request for the
                     // whole group, one round trip), the warp reads them back from
                     // shared memory with broadcast loads; the buffer holds 8
@@ -320,9 +325,10 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                         const float2 dy = add2_rn(make_float2(g.y, g.y), nby);
                         const float2 dz = add2_rn(make_float2(g.z, g.z), nbz);
                         // |dr|^2 = fma(dz, dz, fma(dy, dy, dx * dx)) (R8), 3 instructions
-                        const float2 drsq = fma2_rn(dz, dz, fma2_rn(dy, dy, sqr2_rn(dx, nz)));
-                        const bool o0 = in0 && drsq.x < dl;
-                        const bool o1 = in1 && drsq.y < dl;
+                        // (masked: +inf for a body outside the group's mask)
+                        const float2 drsq = fma2_rn(dz, dz, fma2_rn(dy, dy, SELF ? sqr2_rn(dx, nz) : fma2_rn(dx, dx, zm)));
+                        const bool o0 = (!SELF || in0) && drsq.x < dl;
+                        const bool o1 = (!SELF || in1) && drsq.y < dl;
                         float2 f;
                         if (SELF) {
                             const bool k0 = in0 && !o0 && t.z != self[0];
@@ -338,7 +344,7 @@ __global__ void __launch_bounds__(kBlock, TT_BHG_MINB) bh_group_kernel(const tt_
                             // a body outside the group's mask has r = inf, so inv = 0
                             // and f = 0 exactly (eps > 0 here: active inv is finite)
                             const float2 mw = make_float2(o0 ? 0.f : g.w, o1 ? 0.f : g.w);
-                            const float2 r = add2_rn(drsq, e2m);
+                            const float2 r = add2_rn(drsq, e22);
                             const float2 inv = make_float2(rsqrt_ftz(r.x), rsqrt_ftz(r.y));
                             f = mul2_rn(mul2_rn(mw, mul2_rn(inv, inv)), inv);
                         }
